@@ -1,0 +1,173 @@
+"""CPU ORACLE for the cuZ-Checker assessment hot path — TEST INFRASTRUCTURE ONLY.
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / `--impl reference` legs may
+import this package.  The product path (paper_conf_cluster_yudgtc21_b200) never imports it and
+fails loudly if its CUDA library is missing.  The oracle shares no code with the CUDA path.
+
+Thin ctypes wrapper over `liboracle.so` (built from czc_oracle.c by `build()` or on first use).
+All metric arithmetic lives in czc_oracle.c, each function citing the PAPER.md passage it
+implements.  Pinning status of every function:
+  p1        pinned  (closed forms: zero error, dyadic offset; statistical uniform-noise PSNR;
+                     numpy corrcoef / longdouble two-pass Pearson; brute-force numpy extrema)
+  deriv     pinned  (dyadic ramp / quadratic closed forms; numpy.gradient; scipy.ndimage.laplace)
+  autocorr  pinned  (checkerboard (-1)^tau; single-axis cosine; constant error -> NaN)
+  ssim      pinned  (zero error = 1; constant-field closed form; global-range mode equals the
+                     scipy uniform_filter formulation of scikit-image's SSIM; numpy brute force)
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+from typing import Dict, Sequence
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "liboracle.so")
+_SRC = os.path.join(_HERE, "czc_oracle.c")
+_lib = None
+
+DERIV_FIELDS = ("der1", "der2", "grad", "div", "lap")
+DERIV_STATS = ("maxabs", "mae", "mse", "rmse", "f_min", "f_max", "psnr")
+
+
+class _P1(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_uint64)] + [(k, ctypes.c_double) for k in (
+        "x_min", "x_max", "value_range", "err_min", "err_max", "err_maxabs", "err_mean",
+        "err_absmean", "mse", "rmse", "nrmse", "psnr", "snr", "max_rel_err", "pwr_min",
+        "pwr_max", "pwr_mean")] + [("n_pwr", ctypes.c_uint64), ("pearson", ctypes.c_double),
+                                   ("err_var", ctypes.c_double)]
+
+
+class _DF(ctypes.Structure):
+    _fields_ = [(k, ctypes.c_double) for k in DERIV_STATS]
+
+
+class _Deriv(ctypes.Structure):
+    _fields_ = [("n_interior", ctypes.c_uint64), ("f", _DF * 5)]
+
+
+def build(force: bool = False) -> str:
+    """Compile liboracle.so with gcc (-O2 -fopenmp -ffp-contract=off)."""
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
+        cmd = ["gcc", "-O2", "-fopenmp", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared",
+               "-std=c11", "-Wall", "-o", _SO, _SRC, "-lm"]
+        subprocess.check_call(cmd)
+    return _SO
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        build()
+        lib = ctypes.CDLL(_SO)
+        P = ctypes.c_void_p
+        I64P = ctypes.POINTER(ctypes.c_int64)
+        lib.czco_p1.argtypes = [P, P, ctypes.c_uint64, ctypes.POINTER(_P1)]
+        lib.czco_deriv.argtypes = [P, P, ctypes.c_int, I64P, ctypes.POINTER(_Deriv)]
+        lib.czco_autocorr.argtypes = [P, P, ctypes.c_int, I64P, ctypes.c_int,
+                                      ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_uint64)]
+        lib.czco_ssim_window.argtypes = [P, P, ctypes.c_int, I64P, I64P, I64P, ctypes.c_int, ctypes.c_double]
+        lib.czco_ssim_window.restype = ctypes.c_double
+        lib.czco_ssim.argtypes = [P, P, ctypes.c_int, I64P, I64P, I64P, ctypes.c_int,
+                                  ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_uint64)]
+        lib.czco_threads.restype = ctypes.c_int
+        _lib = lib
+    return _lib
+
+
+def _f32(a) -> np.ndarray:
+    if hasattr(a, "detach"):
+        a = a.detach().cpu().numpy()
+    a = np.ascontiguousarray(a, dtype=np.float32)
+    return a
+
+
+def _dims(a: np.ndarray, dims=None):
+    d = tuple(a.shape) if dims is None else tuple(int(v) for v in dims)
+    return len(d), (ctypes.c_int64 * len(d))(*d)
+
+
+def _i64(v: Sequence[int]):
+    return (ctypes.c_int64 * len(v))(*[int(t) for t in v])
+
+
+def threads() -> int:
+    return int(_load().czco_threads())
+
+
+def p1(x, y) -> Dict[str, float]:
+    x, y = _f32(x), _f32(y)
+    r = _P1()
+    rc = _load().czco_p1(x.ctypes.data, y.ctypes.data, x.size, ctypes.byref(r))
+    if rc:
+        raise ValueError(f"czco_p1 failed ({rc})")
+    return {k: getattr(r, k) for k, _ in _P1._fields_}
+
+
+def deriv(x, y, dims=None) -> Dict[str, float]:
+    x, y = _f32(x), _f32(y)
+    nd, d = _dims(x, dims)
+    r = _Deriv()
+    rc = _load().czco_deriv(x.ctypes.data, y.ctypes.data, nd, d, ctypes.byref(r))
+    if rc:
+        raise ValueError(f"czco_deriv failed ({rc})")
+    out = {"n_interior": r.n_interior}
+    for i, f in enumerate(DERIV_FIELDS):
+        for s in DERIV_STATS:
+            out[f"{f}_{s}"] = getattr(r.f[i], s)
+    return out
+
+
+def autocorr(x, y, max_lag: int = 10, dims=None):
+    """Returns (ac[0..max_lag], count[0..max_lag])."""
+    x, y = _f32(x), _f32(y)
+    nd, d = _dims(x, dims)
+    ac = (ctypes.c_double * (max_lag + 1))()
+    cnt = (ctypes.c_uint64 * (max_lag + 1))()
+    rc = _load().czco_autocorr(x.ctypes.data, y.ctypes.data, nd, d, max_lag, ac, cnt)
+    if rc:
+        raise ValueError(f"czco_autocorr failed ({rc})")
+    return np.array(ac[:], dtype=np.float64), np.array(cnt[:], dtype=np.uint64)
+
+
+def ssim_window(x, y, origin, window, range_mode: int = 0, global_range: float = 0.0, dims=None) -> float:
+    x, y = _f32(x), _f32(y)
+    nd, d = _dims(x, dims)
+    return float(_load().czco_ssim_window(x.ctypes.data, y.ctypes.data, nd, d, _i64(origin),
+                                          _i64(window), range_mode, global_range))
+
+
+def ssim(x, y, window, step=None, range_mode: int = 0, dims=None):
+    """Returns (ssim, n_windows).  window/step: one value per axis (slowest-first)."""
+    x, y = _f32(x), _f32(y)
+    nd, d = _dims(x, dims)
+    if step is None:
+        step = [1] * nd
+    out = ctypes.c_double()
+    nw = ctypes.c_uint64()
+    rc = _load().czco_ssim(x.ctypes.data, y.ctypes.data, nd, d, _i64(window), _i64(step), range_mode,
+                           ctypes.byref(out), ctypes.byref(nw))
+    if rc == 3:
+        return float("nan"), 0
+    if rc:
+        raise ValueError(f"czco_ssim failed ({rc})")
+    return out.value, int(nw.value)
+
+
+def assess(x, y, window=None, step=None, max_lag: int = 10, range_mode: int = 0) -> Dict[str, float]:
+    """All oracle metrics in one flat dict keyed like the CUDA binding's result."""
+    x, y = _f32(x), _f32(y)
+    nd = x.ndim
+    out = dict(p1(x, y))
+    out.update(deriv(x, y))
+    ac, cnt = autocorr(x, y, max_lag)
+    out["ac"] = ac
+    out["ac_count"] = cnt
+    if window is None:
+        window = [8] * nd
+    s, nw = ssim(x, y, window, step, range_mode)
+    out["ssim"] = s
+    out["n_windows"] = nw
+    return out

@@ -1,0 +1,321 @@
+"""Pins of the CPU oracle to things other than itself (no GPU needed).
+
+Each test fixes an oracle function against a closed form, an invariant, a library routine that
+implements the same definition independently (numpy / scipy), or brute force on tiny inputs —
+chosen so that a dropped term, a wrong sign or index, or a transposed operand fails one of them.
+Citations: PAPER.md line numbers (Lnnn); readings R1..R23 are DESIGN.md §2.
+"""
+import math
+
+import numpy as np
+import pytest
+import scipy.ndimage as ndi
+
+import synth
+
+rng = np.random.default_rng(1234)
+
+
+def dyadic_field(shape, scale=2.0 ** -20, lo=-(2 ** 18), hi=2 ** 18):
+    """Values on a 2^-20 grid with |x| < 1/4: float32-exact, and x + 2^-10 stays exact."""
+    return (rng.integers(lo, hi, size=shape).astype(np.float64) * scale).astype(np.float32)
+
+
+# ------------------------------------------------------------------------------------------ P1
+class TestP1:
+    def test_zero_error(self, orc):
+        """y = x: every error statistic is 0, PSNR = SNR = +inf, Pearson = 1 (north_star)."""
+        x = dyadic_field((9, 10, 11))
+        x[0, 0, :3] = 0.0
+        r = orc.p1(x, x)
+        for k in ("err_min", "err_max", "err_maxabs", "err_mean", "err_absmean", "mse", "rmse",
+                  "nrmse", "max_rel_err", "pwr_min", "pwr_max", "pwr_mean", "err_var"):
+            assert r[k] == 0.0, k
+        assert r["psnr"] == math.inf and r["snr"] == math.inf
+        assert abs(r["pearson"] - 1.0) < 1e-15
+        assert r["n_pwr"] == int(np.count_nonzero(x)) and r["n"] == x.size
+
+    def test_dyadic_offset_closed_form(self, orc):
+        """e == c exactly (dyadic grid): MSE = c^2 bit-exact, RMSE = c, PSNR = 20 log10(R/c)."""
+        x = dyadic_field((7, 13, 17))
+        c = 2.0 ** -10
+        y = (x.astype(np.float64) + c).astype(np.float32)
+        assert np.all(y.astype(np.float64) - x.astype(np.float64) == c)
+        r = orc.p1(x, y)
+        R = float(x.max()) - float(x.min())
+        assert r["mse"] == c * c and r["rmse"] == c and r["err_mean"] == c
+        assert r["err_min"] == c == r["err_max"] == r["err_maxabs"] == r["err_absmean"]
+        assert r["err_var"] == 0.0
+        assert r["value_range"] == R and r["max_rel_err"] == c / R
+        assert abs(r["psnr"] - 20 * math.log10(R / c)) < 1e-12
+        assert abs(r["nrmse"] - c / R) < 1e-18
+        assert abs(r["pearson"] - 1.0) < 1e-15
+
+    def test_uniform_noise_psnr_statistical(self, orc):
+        """C1 recipe, e ~ U[-a, a]: E[MSE] = a^2/3 (rel. sd 0.894/sqrt(N)), E[e] = 0 (sd a/sqrt(3N))."""
+        spec = synth.CONFIGS["C1"]
+        x, y = synth.make_pair(spec)
+        r = orc.p1(x, y)
+        a, N = spec.eb, x.numel()
+        assert abs(r["mse"] / (a * a / 3) - 1) < 4 * 0.894 / math.sqrt(N)
+        assert abs(r["err_mean"]) < 4 * a / math.sqrt(3 * N)
+        expect_psnr = 20 * math.log10(r["value_range"]) - 10 * math.log10(a * a / 3)
+        assert abs(r["psnr"] - expect_psnr) < 4 * 10 / math.log(10) * 0.894 / math.sqrt(N)
+        assert r["err_maxabs"] <= a * (1 + 1e-6)
+
+    @pytest.mark.parametrize("cfg", ["C1", "C2q"])
+    def test_against_numpy(self, orc, cfg):
+        """Independent numpy float64 formulations (pairwise sums) of every P1 definition."""
+        spec = synth.config(cfg, dims=(20, 30, 40))
+        x, y = synth.make_pair(spec)
+        x, y = x.numpy(), y.numpy()
+        r = orc.p1(x, y)
+        xd, yd = x.astype(np.float64), y.astype(np.float64)
+        e = yd - xd
+        assert r["x_min"] == float(x.min()) and r["x_max"] == float(x.max())
+        assert r["err_min"] == e.min() and r["err_max"] == e.max() and r["err_maxabs"] == np.abs(e).max()
+        nz = x != 0
+        q = np.abs(e[nz]) / np.abs(xd[nz])
+        assert r["n_pwr"] == int(nz.sum())
+        assert r["pwr_min"] == q.min() and r["pwr_max"] == q.max()
+        assert abs(r["pwr_mean"] - q.mean()) <= 1e-12 * q.mean()
+        assert abs(r["mse"] - np.mean(e * e)) <= 1e-12 * r["mse"]
+        assert abs(r["err_var"] - np.var(e)) <= 1e-10 * r["err_var"]
+        assert abs(r["err_absmean"] - np.mean(np.abs(e))) <= 1e-12 * r["err_absmean"]
+        assert abs(r["err_mean"] - np.mean(e)) <= 1e-12 * r["err_absmean"]
+        assert abs(r["pearson"] - np.corrcoef(xd.ravel(), yd.ravel())[0, 1]) < 1e-12
+        snr = 10 * np.log10(np.sum((xd - xd.mean()) ** 2) / np.sum(e * e))
+        assert abs(r["snr"] - snr) < 1e-9
+
+    def test_pearson_large_mean(self, orc):
+        """1e5 +- 100 field (condition ~ mean^2/var): two-pass Pearson vs numpy corrcoef (centred)."""
+        x = (1e5 + 100 * rng.standard_normal(4096)).astype(np.float32)
+        y = (x.astype(np.float64) + rng.uniform(-0.01, 0.01, 4096)).astype(np.float32)
+        r = orc.p1(x, y)
+        ref = np.corrcoef(x.astype(np.float64), y.astype(np.float64))[0, 1]
+        assert abs(r["pearson"] - ref) < 1e-13
+        assert 1 - ref > 1e-10            # the quantity really is resolved
+
+    def test_degenerate(self, orc):
+        """Constant original: R = 0 -> PSNR -inf when MSE > 0, Pearson NaN; all-zero x: pwr NaN."""
+        x = np.full(64, 3.0, np.float32)
+        y = x + np.float32(0.5)
+        r = orc.p1(x, y)
+        assert r["value_range"] == 0 and r["psnr"] == -math.inf and math.isnan(r["pearson"])
+        assert r["nrmse"] == math.inf
+        z = np.zeros(16, np.float32)
+        r = orc.p1(z, z + np.float32(1))
+        assert r["n_pwr"] == 0 and math.isnan(r["pwr_max"]) and math.isnan(r["pwr_mean"])
+
+
+# ------------------------------------------------------------------------------------------ P2
+def _interior(a):
+    return a[tuple(slice(1, -1) if n > 1 else slice(None) for n in a.shape)]
+
+
+def _fields_numpy(f):
+    """Derived fields via library routines: numpy.gradient (central /2) and scipy laplace."""
+    f = f.astype(np.float64)
+    axes = [a for a, n in enumerate(f.shape) if n > 1]
+    D = [np.gradient(f, axis=a) for a in axes]          # interior: (f(p+1) - f(p-1)) / 2
+    der1 = sum(2 * np.abs(d) for d in D)
+    grad = np.sqrt(sum(d * d for d in D))
+    div = sum(D)
+    lap = ndi.laplace(f, mode="nearest")                 # interior: sum_a f(+1) - 2 f + f(-1)
+    sec = []
+    for a in axes:
+        s = np.zeros_like(f)
+        sl = [slice(None)] * f.ndim
+        sl[a] = slice(1, -1)
+        hi = list(sl); hi[a] = slice(2, None)
+        lo = list(sl); lo[a] = slice(0, -2)
+        s[tuple(sl)] = f[tuple(hi)] - 2 * f[tuple(sl)] + f[tuple(lo)]
+        sec.append(s)
+    der2 = sum(np.abs(s) for s in sec)
+    return {k: _interior(v) for k, v in
+            dict(der1=der1, der2=der2, grad=grad, div=div, lap=lap).items()}
+
+
+class TestDeriv:
+    def test_dyadic_ramp(self, orc):
+        """f = sum_a c_a p_a: D_a = c_a, Delta_a = 0 -> Der1 = 2 sum|c|, Grad = |c|, Lap = 0 (L122, L129)."""
+        shape = (6, 7, 9)
+        p = np.indices(shape).astype(np.float64)
+        c = np.array([2 ** -3, -(2 ** -4), 2 ** -5])
+        cy = np.array([2 ** -3, 2 ** -4, 2 ** -6])
+        x = np.tensordot(c, p, 1).astype(np.float32) + np.float32(1)
+        y = np.tensordot(cy, p, 1).astype(np.float32) + np.float32(1)
+        r = orc.deriv(x, y)
+        assert r["n_interior"] == 4 * 5 * 7
+        assert r["der1_f_min"] == r["der1_f_max"] == 2 * np.abs(c).sum()
+        assert r["grad_f_min"] == pytest.approx(math.sqrt((c ** 2).sum()), abs=1e-15)
+        assert r["div_f_max"] == c.sum() and r["lap_f_max"] == 0 and r["der2_f_max"] == 0
+        d1 = 2 * (np.abs(cy).sum() - np.abs(c).sum())
+        assert r["der1_maxabs"] == abs(d1) and r["der1_mae"] == abs(d1) and r["der1_mse"] == d1 * d1
+        dd = cy.sum() - c.sum()
+        assert r["div_maxabs"] == abs(dd) and r["div_mse"] == dd * dd
+        assert r["lap_maxabs"] == 0 and r["lap_psnr"] == math.inf
+
+    def test_quadratic(self, orc):
+        """f = sum_a q_a p_a^2: Delta_a = 2 q_a exactly -> Lap = 2 sum q, Der2 = 2 sum |q|."""
+        shape = (5, 6, 7)
+        p = np.indices(shape).astype(np.float64)
+        q = np.array([2 ** -4, -(2 ** -5), 2 ** -3])
+        x = np.tensordot(q, p ** 2, 1).astype(np.float32)
+        r = orc.deriv(x, x)
+        assert r["lap_f_min"] == r["lap_f_max"] == 2 * q.sum()
+        assert r["der2_f_min"] == r["der2_f_max"] == 2 * np.abs(q).sum()
+        assert r["lap_mse"] == 0 and r["der1_maxabs"] == 0
+
+    @pytest.mark.parametrize("shape", [(12, 14, 16), (30, 40), (9, 1, 33)])
+    def test_against_numpy_scipy(self, orc, shape):
+        spec = synth.config("C1", dims=shape)
+        x, y = synth.make_pair(spec)
+        x, y = x.numpy(), y.numpy()
+        r = orc.deriv(x, y)
+        Fx, Fy = _fields_numpy(x), _fields_numpy(y)
+        assert r["n_interior"] == Fx["der1"].size
+        for k in Fx:
+            d = Fy[k] - Fx[k]
+            scale = max(1.0, float(np.abs(Fx[k]).max()))
+            assert abs(r[f"{k}_f_min"] - Fx[k].min()) < 1e-13 * scale, k
+            assert abs(r[f"{k}_f_max"] - Fx[k].max()) < 1e-13 * scale, k
+            assert abs(r[f"{k}_maxabs"] - np.abs(d).max()) < 1e-13 * scale, k
+            assert abs(r[f"{k}_mae"] - np.abs(d).mean()) < 1e-13 * scale, k
+            assert abs(r[f"{k}_mse"] - (d * d).mean()) < 1e-12 * max(r[f"{k}_mse"], 1e-30) + 1e-26, k
+
+    def test_no_interior(self, orc):
+        x = dyadic_field((2, 5, 5))
+        r = orc.deriv(x, x)
+        assert r["n_interior"] == 0 and math.isnan(r["der1_mae"])
+
+
+# ------------------------------------------------------------------------------------------ AC
+class TestAutocorr:
+    def _pair_with_error(self, e):
+        x = dyadic_field(e.shape)
+        y = (x.astype(np.float64) + e).astype(np.float32)
+        assert np.all(y.astype(np.float64) - x.astype(np.float64) == e)
+        return x, y
+
+    def test_checkerboard(self, orc):
+        """e = c (-1)^(z+y+x) on even dims: mu = 0, sigma^2 = c^2, AC(tau) = (-1)^tau exactly (Eq. 2)."""
+        shape = (8, 10, 12)
+        e = (2.0 ** -10) * (-1.0) ** np.indices(shape).sum(0)
+        ac, cnt = orc.autocorr(*self._pair_with_error(e), max_lag=6)
+        assert np.allclose(ac, [(-1.0) ** t for t in range(7)], rtol=0, atol=1e-15)
+        assert list(cnt[1:]) == [(8 - t) * (10 - t) * (12 - t) for t in range(1, 7)]
+
+    @pytest.mark.parametrize("axis", [0, 1, 2])
+    def test_single_axis_parity(self, orc, axis):
+        """e = c (-1)^(p_axis): the other two axis terms are +1, this one (-1)^tau -> (2 + (-1)^tau)/3."""
+        shape = (6, 8, 10)
+        e = (2.0 ** -9) * (-1.0) ** np.indices(shape)[axis]
+        ac, _ = orc.autocorr(*self._pair_with_error(e), max_lag=5)
+        want = [1.0] + [(2 + (-1.0) ** t) / 3 for t in range(1, 6)]
+        assert np.allclose(ac, want, rtol=0, atol=1e-15)
+
+    def test_2d_factor(self, orc):
+        """2-D field: 1/D = 1/2 (R12): e = c (-1)^x -> AC = (1 + (-1)^tau) / 2."""
+        e = (2.0 ** -9) * (-1.0) ** np.indices((10, 14))[1]
+        ac, cnt = orc.autocorr(*self._pair_with_error(e), max_lag=4)
+        assert np.allclose(ac, [1.0] + [(1 + (-1.0) ** t) / 2 for t in range(1, 5)], atol=1e-15)
+        assert list(cnt[1:]) == [(10 - t) * (14 - t) for t in range(1, 5)]
+
+    def test_brute_force_slices(self, orc):
+        """Random errors: vectorised slice formulation of Eq. 2 (population mu, sigma^2 over N)."""
+        x, y = synth.make_pair(synth.config("C1", dims=(11, 12, 13)))
+        x, y = x.numpy(), y.numpy()
+        e = y.astype(np.float64) - x.astype(np.float64)
+        mu, var = e.mean(), e.var()
+        ac, _ = orc.autocorr(x, y, max_lag=5)
+        for t in range(1, 6):
+            c = e[:-t, :-t, :-t] - mu
+            nb = (e[t:, :-t, :-t] - mu) + (e[:-t, t:, :-t] - mu) + (e[:-t, :-t, t:] - mu)
+            want = np.sum(c * nb / 3) / c.size / var
+            assert abs(ac[t] - want) < 1e-12, t
+
+    def test_degenerate(self, orc):
+        x = dyadic_field((6, 6, 6))
+        y = (x.astype(np.float64) + 2.0 ** -12).astype(np.float32)
+        ac, cnt = orc.autocorr(x, y, max_lag=7)
+        assert ac[0] == 1 and np.all(np.isnan(ac[1:]))         # sigma^2 = 0
+        assert cnt[6] == 0 and cnt[7] == 0 and cnt[5] == 1     # tau >= min n -> no pairs
+
+
+# ------------------------------------------------------------------------------------------ SSIM
+def ssim_uniform_filter(x, y, w, data_range):
+    """scikit-image's structural_similarity(win_size=w, data_range=R, gaussian_weights=False,
+    use_sample_covariance=False) restated with scipy.ndimage.uniform_filter and the crop of
+    (w-1)/2 it applies before averaging — valid windows, global dynamic range."""
+    x = x.astype(np.float64)
+    y = y.astype(np.float64)
+    ux, uy = ndi.uniform_filter(x, w), ndi.uniform_filter(y, w)
+    uxx, uyy, uxy = ndi.uniform_filter(x * x, w), ndi.uniform_filter(y * y, w), ndi.uniform_filter(x * y, w)
+    vx, vy, vxy = uxx - ux * ux, uyy - uy * uy, uxy - ux * uy
+    C1, C2 = (0.01 * data_range) ** 2, (0.03 * data_range) ** 2
+    S = (2 * ux * uy + C1) * (2 * vxy + C2) / ((ux ** 2 + uy ** 2 + C1) * (vx + vy + C2))
+    p = (w - 1) // 2
+    return S[tuple(slice(p, n - p) for n in S.shape)].mean()
+
+
+def ssim_brute_numpy(x, y, w, s=1):
+    """Per-window numpy moments (np.var, np.cov bias=True), local range of the original."""
+    vals = []
+    it = [range(0, n - w + 1, s) for n in x.shape]
+    for o in np.array(np.meshgrid(*it, indexing="ij")).reshape(x.ndim, -1).T:
+        sl = tuple(slice(a, a + w) for a in o)
+        a, b = x[sl].astype(np.float64).ravel(), y[sl].astype(np.float64).ravel()
+        L = a.max() - a.min()
+        L = 1.0 if L == 0 else L
+        C1, C2 = (0.01 * L) ** 2, (0.03 * L) ** 2
+        cxy = np.cov(a, b, bias=True)[0, 1]
+        vals.append((2 * a.mean() * b.mean() + C1) * (2 * cxy + C2) /
+                    ((a.mean() ** 2 + b.mean() ** 2 + C1) * (np.var(a) + np.var(b) + C2)))
+    return np.array(vals)
+
+
+class TestSSIM:
+    def test_zero_error_is_one(self, orc):
+        x, _ = synth.make_pair(synth.config("C2q", dims=(12, 16, 20)))
+        s, nw = orc.ssim(x, x, [5, 5, 5])
+        assert abs(s - 1) < 1e-15 and nw == 8 * 12 * 16
+
+    def test_constant_field_closed_form(self, orc):
+        """x = v, y = v + c: L = 0 -> 1, sigma = 0 -> SSIM = (2v(v+c)+C1)/(v^2+(v+c)^2+C1)."""
+        v, c = 0.75, 2.0 ** -8
+        x = np.full((9, 9, 9), v, np.float32)
+        y = np.full((9, 9, 9), v + c, np.float32)
+        s, nw = orc.ssim(x, y, [4, 4, 4])
+        C1 = 1e-4
+        assert nw == 6 ** 3
+        assert abs(s - (2 * v * (v + c) + C1) / (v * v + (v + c) ** 2 + C1)) < 1e-15
+
+    @pytest.mark.parametrize("shape,w", [((20, 22, 24), 7), ((40, 56), 7), ((15, 17, 19), 5)])
+    def test_global_range_equals_skimage_formulation(self, orc, shape, w):
+        x, y = synth.make_pair(synth.config("C1", dims=shape))
+        x, y = x.numpy(), y.numpy()
+        R = float(x.max()) - float(x.min())
+        s, _ = orc.ssim(x, y, [w] * len(shape), range_mode=1)
+        assert abs(s - ssim_uniform_filter(x, y, w, R)) < 1e-10
+
+    @pytest.mark.parametrize("cfg,shape,w,s", [("C1", (8, 9, 10), 4, 1), ("C2q", (9, 10, 12), 3, 2),
+                                               ("C4", (24, 30), 8, 3), ("C3", (7, 8, 9), 3, 1)])
+    def test_brute_force_numpy(self, orc, cfg, shape, w, s):
+        """Local-range SSIM, every window, against a numpy brute force; sparse zeros hit L := 1."""
+        x, y = synth.make_pair(synth.config(cfg, dims=shape))
+        x, y = x.numpy(), y.numpy()
+        ref = ssim_brute_numpy(x, y, w, s)
+        got, nw = orc.ssim(x, y, [w] * len(shape), [s] * len(shape))
+        assert nw == ref.size
+        assert abs(got - ref.mean()) < 1e-13
+        it = [range(0, n - w + 1, s) for n in shape]
+        origins = np.array(np.meshgrid(*it, indexing="ij")).reshape(len(shape), -1).T
+        for i in rng.choice(len(origins), size=min(20, len(origins)), replace=False):
+            v = orc.ssim_window(x, y, origins[i], [w] * len(shape))
+            assert abs(v - ref[i]) < 1e-13
+
+    def test_no_window(self, orc):
+        x = dyadic_field((5, 5, 5))
+        s, nw = orc.ssim(x, x, [6, 6, 6])
+        assert nw == 0 and math.isnan(s)
