@@ -38,7 +38,7 @@ extern "C" {
 #endif
 
 #define CZC_ABI_VERSION 1
-#define CZC_MAX_LAG 32           /* largest supported autocorrelation lag (paper uses <= 10, L345) */
+#define CZC_MAX_LAG 16           /* largest supported autocorrelation lag (paper uses <= 10, L345) */
 
 typedef enum czc_status {
   CZC_OK = 0,
@@ -159,6 +159,11 @@ const char* czc_last_error(const czc_ctx* ctx);
 /* ABI version (CZC_ABI_VERSION) and whether NCCL slab mode was compiled in (1/0). */
 int czc_abi_version(void);
 int czc_has_nccl(void);
+
+/* sizeof(czc_config) (what = 0), sizeof(czc_shape) (1), sizeof(czc_result) (2), bytes copied
+ * device->host per czc_assess call (3); 0 otherwise.  Lets bindings verify their struct mirrors
+ * against the compiled library. */
+uint64_t czc_sizeof(int what);
 
 #ifdef __cplusplus
 }

@@ -1,0 +1,538 @@
+// czc_api.cu — the C ABI (include/czc.h): context, validation, the "GPU module coordinator"
+// (L96: identify the requested metric categories, launch the matching fused kernels), one
+// device->host copy of the partial results, and the scalar finish math (derived metrics).
+#include <cuda_runtime.h>
+#include <math.h>
+#include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <algorithm>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "czc_internal.cuh"
+#include "czc_comm.h"
+
+namespace czc {
+cudaError_t launch_p1(const float* x, const float* y, int64_t n, int grid_cap, P1State* parts,
+                      DevResults* res, unsigned int* ticket, cudaStream_t st);
+cudaError_t launch_p1_combine(const P1State* states, int count, DevResults* res, cudaStream_t st);
+int p1_max_blocks_per_sm();
+int64_t deriv_blocks(const Field3& s, int zchunk);
+int64_t ac_blocks(const Field3& s, int zchunk);
+cudaError_t launch_deriv(const Field3& s, int zchunk, double* parts, DevResults* res,
+                         unsigned int* ticket, cudaStream_t st);
+cudaError_t launch_ac(const Field3& s, int T, int zchunk, double* parts, DevResults* res,
+                      unsigned int* ticket, cudaStream_t st);
+cudaError_t launch_ssim(int kind, int W, const Field3& f, const SsimParams& p,
+                        double* parts, DevResults* res, unsigned int* ticket, double* dbg,
+                        cudaStream_t st, int64_t* nblocks_out);
+}  // namespace czc
+
+using namespace czc;
+
+struct czc_ctx {
+  czc_config cfg;
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  int sm_count = 0;
+  int p1_grid_cap = 0;
+  DevResults* dres = nullptr;      // device
+  DevResults* hres = nullptr;      // pinned host
+  unsigned int* tickets = nullptr; // device
+  void* parts = nullptr;
+  size_t parts_cap = 0;
+  float* din[2] = {nullptr, nullptr};   // staging for czc_assess_host
+  size_t din_cap = 0;
+  cudaEvent_t ev[5] = {};
+  std::string last_error;
+  CommState* comm = nullptr;
+  // slab mode
+  void* dgather_in = nullptr;      // device, 64 B
+  void* dgather = nullptr;         // device, nranks * sizeof(DevResults)
+  void* hgather = nullptr;         // pinned host, nranks * sizeof(DevResults)
+  float* halo = nullptr;           // device halo planes (x lo, y lo, x hi, y hi)
+  size_t halo_cap = 0;
+};
+
+static const char* kStatusStr[] = {"ok", "invalid argument", "invalid shape", "unsupported dtype",
+                                   "CUDA error", "out of memory", "communication (NCCL) error",
+                                   "unsupported"};
+
+extern "C" const char* czc_strerror(czc_status s) {
+  const int i = (int)s;
+  return (i >= 0 && i < 8) ? kStatusStr[i] : "unknown status";
+}
+extern "C" const char* czc_last_error(const czc_ctx* ctx) { return ctx ? ctx->last_error.c_str() : ""; }
+extern "C" int czc_abi_version(void) { return CZC_ABI_VERSION; }
+extern "C" int czc_has_nccl(void) { return comm_available(); }
+extern "C" uint64_t czc_sizeof(int what) {
+  return what == 0 ? sizeof(czc_config) : what == 1 ? sizeof(czc_shape) : what == 2 ? sizeof(czc_result)
+       : what == 3 ? sizeof(DevResults) : 0;
+}
+
+static czc_status cuda_fail(czc_ctx* ctx, cudaError_t e, const char* where) {
+  if (ctx) ctx->last_error = std::string(where) + ": " + cudaGetErrorString(e);
+  (void)cudaGetLastError();
+  return e == cudaErrorMemoryAllocation ? CZC_ERR_NOMEM : CZC_ERR_CUDA;
+}
+#define CZC_CUDA(ctx, call)                                   \
+  do {                                                        \
+    cudaError_t _e = (call);                                  \
+    if (_e != cudaSuccess) return cuda_fail((ctx), _e, #call); \
+  } while (0)
+
+extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
+  if (!out) return CZC_ERR_INVALID;
+  *out = nullptr;
+  czc_config c;
+  memset(&c, 0, sizeof(c));
+  if (cfg) c = *cfg;
+  else c.device = -1;
+  if (c.ac_max_lag < 0 || c.ac_max_lag > CZC_MAX_LAG) return CZC_ERR_INVALID;
+  if (c.ssim_range_mode < 0 || c.ssim_range_mode > 1) return CZC_ERR_INVALID;
+  for (int i = 0; i < 3; i++)
+    if (c.ssim_window[i] < 0 || c.ssim_step[i] < 0) return CZC_ERR_INVALID;
+  if (c.nranks > 1 && (c.rank < 0 || c.rank >= c.nranks || !c.nccl_uid)) return CZC_ERR_INVALID;
+  if (c.nranks > 1 && !comm_available()) return CZC_ERR_UNSUPPORTED;
+
+  czc_ctx* ctx = new (std::nothrow) czc_ctx();
+  if (!ctx) return CZC_ERR_NOMEM;
+  ctx->cfg = c;
+  czc_status st = CZC_OK;
+  do {
+    int dev = c.device;
+    if (dev < 0) {
+      if (cudaGetDevice(&dev) != cudaSuccess) { st = cuda_fail(ctx, cudaGetLastError(), "cudaGetDevice"); break; }
+    }
+    ctx->device = dev;
+    cudaError_t e = cudaSetDevice(dev);
+    if (e != cudaSuccess) { st = cuda_fail(ctx, e, "cudaSetDevice"); break; }
+    cudaDeviceGetAttribute(&ctx->sm_count, cudaDevAttrMultiProcessorCount, dev);
+    ctx->p1_grid_cap = ctx->sm_count * p1_max_blocks_per_sm();
+    if (c.stream) {
+      ctx->stream = (cudaStream_t)c.stream;
+    } else {
+      e = cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking);
+      if (e != cudaSuccess) { st = cuda_fail(ctx, e, "cudaStreamCreate"); break; }
+      ctx->own_stream = true;
+    }
+    if ((e = cudaMalloc(&ctx->dres, sizeof(DevResults))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(res)"); break; }
+    if ((e = cudaMallocHost(&ctx->hres, sizeof(DevResults))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMallocHost"); break; }
+    if ((e = cudaMalloc(&ctx->tickets, TICKET_N * sizeof(unsigned int))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(tickets)"); break; }
+    if ((e = cudaMemset(ctx->tickets, 0, TICKET_N * sizeof(unsigned int))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMemset"); break; }
+    for (int i = 0; i < 5; i++)
+      if ((e = cudaEventCreate(&ctx->ev[i])) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaEventCreate"); break; }
+    if (st != CZC_OK) break;
+    if (c.nranks > 1) {
+      const size_t gb = (size_t)c.nranks * sizeof(DevResults);
+      if ((e = cudaMalloc(&ctx->dgather_in, 64)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(gather)"); break; }
+      if ((e = cudaMalloc(&ctx->dgather, gb)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(gather)"); break; }
+      if ((e = cudaMallocHost(&ctx->hgather, gb)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMallocHost(gather)"); break; }
+      ctx->comm = comm_create(c.nccl_uid, c.rank, c.nranks, &ctx->last_error);
+      if (!ctx->comm) { st = CZC_ERR_COMM; break; }
+    }
+  } while (0);
+  if (st != CZC_OK) {
+    czc_free(ctx);
+    return st;
+  }
+  *out = ctx;
+  return CZC_OK;
+}
+
+extern "C" void czc_free(czc_ctx* ctx) {
+  if (!ctx) return;
+  cudaSetDevice(ctx->device);
+  if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+  if (ctx->comm) comm_destroy(ctx->comm);
+  cudaFree(ctx->dres);
+  cudaFreeHost(ctx->hres);
+  cudaFree(ctx->tickets);
+  cudaFree(ctx->parts);
+  cudaFree(ctx->din[0]);
+  cudaFree(ctx->din[1]);
+  cudaFree(ctx->dgather_in);
+  cudaFree(ctx->dgather);
+  cudaFreeHost(ctx->hgather);
+  cudaFree(ctx->halo);
+  for (int i = 0; i < 5; i++)
+    if (ctx->ev[i]) cudaEventDestroy(ctx->ev[i]);
+  if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
+  delete ctx;
+}
+
+// ------------------------------------------------------------------------------------------------
+// Planning
+// ------------------------------------------------------------------------------------------------
+namespace {
+struct Plan {
+  int64_t n = 0;                  // local elements
+  int64_t d3[3] = {1, 1, 1};      // squeezed, right-aligned (nz, ny, nx) of the LOCAL field
+  int64_t g3[3] = {1, 1, 1};      // same for the GLOBAL field
+  int D = 0;                      // active axes
+  int W = 8, step[3] = {1, 1, 1}; // SSIM (per 3-D axis)
+  int win3[3] = {1, 1, 1};
+  int kind = 0;                   // 3, 2, 1 (active axes of the SSIM window)
+  int T = 10;
+  bool run_p1 = false, run_deriv = false, run_ac = false, run_ssim = false;
+  int32_t win_in[3] = {0, 0, 0}, step_in[3] = {0, 0, 0};  // reported per input axis
+};
+
+czc_status make_plan(const czc_ctx* ctx, const czc_shape* sh, uint64_t mask, Plan& P, std::string& why) {
+  const czc_config& c = ctx->cfg;
+  if (sh->ndim < 1 || sh->ndim > 3) { why = "ndim must be 1..3"; return CZC_ERR_SHAPE; }
+  int64_t gd[3], ld[3];
+  for (int i = 0; i < sh->ndim; i++) {
+    if (sh->dims[i] < 1) { why = "dims must be >= 1"; return CZC_ERR_SHAPE; }
+    gd[i] = ld[i] = sh->dims[i];
+  }
+  const int64_t nzl = sh->nz_local > 0 ? sh->nz_local : sh->dims[0];
+  if (sh->z0 < 0 || sh->z0 + nzl > sh->dims[0]) { why = "slab [z0, z0+nz_local) outside dims[0]"; return CZC_ERR_SHAPE; }
+  ld[0] = nzl;
+  if (ctx->cfg.nranks <= 1 && (sh->z0 != 0 || nzl != sh->dims[0])) { why = "slab shape needs nranks > 1"; return CZC_ERR_SHAPE; }
+  // squeeze inactive (extent-1) axes of the GLOBAL shape; C-order layout is unchanged by it
+  int act_in[3], na = 0;
+  for (int i = 0; i < sh->ndim; i++)
+    if (gd[i] > 1) act_in[na++] = i;
+  P.D = na;
+  for (int k = 0; k < na; k++) {
+    P.g3[3 - na + k] = gd[act_in[k]];
+    P.d3[3 - na + k] = ld[act_in[k]];
+  }
+  if (ctx->cfg.nranks > 1 && (na < 1 || act_in[0] != 0)) { why = "slab mode needs dims[0] > 1"; return CZC_ERR_SHAPE; }
+  P.n = P.d3[0] * P.d3[1] * P.d3[2];
+  P.T = c.ac_max_lag ? c.ac_max_lag : 10;
+  P.run_ssim = (mask & CZC_M_SSIM) != 0;
+  P.run_deriv = (mask & CZC_M_DERIV) != 0;
+  P.run_ac = (mask & CZC_M_AUTOCORR) != 0;
+  P.run_p1 = (mask & (CZC_M_P1 | CZC_M_AUTOCORR)) != 0 || (P.run_ssim && c.ssim_range_mode == 1);
+  // SSIM window per input axis -> per active axis
+  for (int i = 0; i < sh->ndim; i++) {
+    const int w = c.ssim_window[i] ? c.ssim_window[i] : 8;
+    const int s = c.ssim_step[i] ? c.ssim_step[i] : 1;
+    P.win_in[i] = gd[i] > 1 ? w : 1;
+    P.step_in[i] = gd[i] > 1 ? s : 1;
+  }
+  if (P.run_ssim) {
+    if (na == 0) { why = "SSIM needs at least one axis with extent > 1"; return CZC_ERR_SHAPE; }
+    int W = -1;
+    for (int k = 0; k < na; k++) {
+      const int w = P.win_in[act_in[k]];
+      if (W < 0) W = w;
+      if (w != W) { why = "SSIM fast path needs the same window extent on every active axis"; return CZC_ERR_UNSUPPORTED; }
+      if (w > gd[act_in[k]]) { why = "SSIM window larger than the field"; return CZC_ERR_SHAPE; }
+      P.win3[3 - na + k] = w;
+      P.step[3 - na + k] = P.step_in[act_in[k]];
+    }
+    if (W < 2 || W > kMaxWin) { why = "SSIM window extent must be 2..16"; return CZC_ERR_UNSUPPORTED; }
+    P.W = W;
+    P.kind = na;
+  }
+  return CZC_OK;
+}
+
+inline double nan_() { return NAN; }
+
+void finish_p1(const P1State& f, czc_result* o) {
+  const double n = f.n;
+  o->n = (uint64_t)n;
+  o->x_min = f.xmin;
+  o->x_max = f.xmax;
+  const double R = (double)f.xmax - (double)f.xmin;
+  o->value_range = R;
+  o->err_min = f.emin;
+  o->err_max = f.emax;
+  o->err_maxabs = fmax(fabs(f.emin), fabs(f.emax));
+  o->err_mean = f.me;
+  o->err_absmean = f.sae / n;
+  const double se2 = f.m2e + n * f.me * f.me;     // sum e^2 (positive terms)
+  const double mse = se2 / n;
+  o->mse = mse;
+  o->rmse = sqrt(mse);
+  o->nrmse = R > 0 ? sqrt(mse) / R : (mse > 0 ? INFINITY : nan_());
+  o->psnr = mse == 0 ? INFINITY : (R == 0 ? -INFINITY : 20.0 * log10(R) - 10.0 * log10(mse));
+  o->snr = se2 == 0 ? (f.m2x > 0 ? INFINITY : nan_()) : 10.0 * log10(f.m2x / se2);
+  o->max_rel_err = R > 0 ? o->err_maxabs / R : (o->err_maxabs > 0 ? INFINITY : nan_());
+  o->n_pwr = (uint64_t)f.npwr;
+  o->pwr_min = f.npwr > 0 ? f.pmin : nan_();
+  o->pwr_max = f.npwr > 0 ? f.pmax : nan_();
+  o->pwr_mean = f.npwr > 0 ? f.spwr / f.npwr : nan_();
+  o->pearson = (f.m2x > 0 && f.m2y > 0) ? f.cxy / sqrt(f.m2x * f.m2y) : nan_();
+  o->err_var = f.m2e / n;
+}
+
+// Derived metrics from the combined records (global shape in P.g3).
+void finish_all(const Plan& P, const DevResults& R, uint64_t mask, czc_result* out) {
+  uint64_t done = 0;
+  if (P.run_p1 && (mask & CZC_M_P1)) { finish_p1(R.p1, out); done |= CZC_M_P1; }
+  if (P.run_deriv) {
+    int64_t nI = P.D > 0 ? 1 : 0;
+    for (int a = 0; a < 3; a++)
+      if (P.g3[a] > 1) nI *= std::max<int64_t>(P.g3[a] - 2, 0);
+    out->n_interior = (uint64_t)nI;
+    for (int f = 0; f < CZC_NDERIV; f++) {
+      const double* r = R.deriv + f * kDerivStats;
+      czc_deriv_stats& d = out->deriv[f];
+      if (nI == 0) {
+        d.maxabs = d.mae = d.mse = d.rmse = d.f_min = d.f_max = d.psnr = NAN;
+        continue;
+      }
+      d.maxabs = r[0];
+      d.mae = r[1] / (double)nI;
+      d.mse = r[2] / (double)nI;
+      d.rmse = sqrt(d.mse);
+      d.f_min = r[3];
+      d.f_max = r[4];
+      const double rng = d.f_max - d.f_min;
+      d.psnr = d.mse == 0 ? INFINITY : (rng == 0 ? -INFINITY : 20.0 * log10(rng) - 10.0 * log10(d.mse));
+    }
+    done |= CZC_M_DERIV;
+  }
+  if (P.run_ac) {
+    out->ac_max_lag = P.T;
+    const double var = R.p1.m2e / R.p1.n;
+    int64_t nmin = INT64_MAX;
+    for (int a = 0; a < 3; a++)
+      if (P.g3[a] > 1) nmin = std::min(nmin, P.g3[a]);
+    out->ac[0] = 1.0;
+    out->ac_count[0] = (uint64_t)(P.g3[0] * P.g3[1] * P.g3[2]);
+    for (int t = 1; t <= CZC_MAX_LAG; t++) {
+      if (t > P.T || P.D == 0 || t >= nmin) { out->ac[t] = NAN; out->ac_count[t] = 0; continue; }
+      int64_t ne = 1;
+      for (int a = 0; a < 3; a++) ne *= P.g3[a] > 1 ? P.g3[a] - t : 1;
+      out->ac_count[t] = (uint64_t)ne;
+      out->ac[t] = var > 0 ? R.ac[t - 1] / (double)P.D / (double)ne / var : NAN;
+    }
+    done |= CZC_M_AUTOCORR;
+  }
+  if (P.run_ssim) {
+    for (int i = 0; i < 3; i++) { out->ssim_window[i] = P.win_in[i]; out->ssim_step[i] = P.step_in[i]; }
+    out->n_windows = (uint64_t)R.ssim[1];
+    out->ssim = R.ssim[1] > 0 ? R.ssim[0] / R.ssim[1] : NAN;
+    out->n_ssim_exact = (uint64_t)R.ssim[2];
+    done |= CZC_M_SSIM;
+  }
+  out->computed_mask = done;
+}
+}  // namespace
+
+static czc_status ensure_buf(czc_ctx* ctx, void** p, size_t* cap, size_t bytes) {
+  if (bytes <= *cap) return CZC_OK;
+  cudaFree(*p);
+  *p = nullptr;
+  *cap = 0;
+  CZC_CUDA(ctx, cudaMalloc(p, bytes));
+  *cap = bytes;
+  return CZC_OK;
+}
+
+// Slab-mode bookkeeping (nranks > 1): the per-rank slab table, halo buffers, gather buffers.
+struct SlabInfo {
+  int64_t z0, nzl;
+};
+
+static czc_status comm_err(czc_ctx* ctx) { return CZC_ERR_COMM; }
+
+static czc_status assess_core(czc_ctx* ctx, const float* x, const float* y, const czc_shape* shape,
+                              uint64_t mask, czc_result* out) {
+  Plan P;
+  czc_status st = make_plan(ctx, shape, mask, P, ctx->last_error);
+  if (st != CZC_OK) return st;
+  const cudaStream_t s = ctx->stream;
+  const bool timing = ctx->cfg.timing != 0;
+  const int zchunk_d = 32, zchunk_ac = 32, zchunk_ss = 32;
+  const bool slab = ctx->comm != nullptr;
+  const int nranks = slab ? comm_size(ctx->comm) : 1, rank = slab ? comm_rank(ctx->comm) : 0;
+  const int64_t plane = P.g3[1] * P.g3[2];
+
+  // ---- field view: owned planes + halo segments -------------------------------------------------
+  Field3 F{};
+  F.nz = P.g3[0]; F.ny = P.g3[1]; F.nx = P.g3[2];
+  const int64_t z0 = slab ? shape->z0 : 0, nzl = P.d3[0];
+  F.zown0 = z0; F.zown1 = z0 + nzl;
+  int64_t hlo = 0, hhi = 0;
+  if (slab) {
+    // slab table (every rank validates every slab identically -> collective decision)
+    int64_t mine[2] = {z0, nzl};
+    CZC_CUDA(ctx, cudaMemcpyAsync(ctx->dgather_in, mine, sizeof(mine), cudaMemcpyHostToDevice, s));
+    if (!comm_allgather(ctx->comm, ctx->dgather_in, ctx->dgather, sizeof(mine), s, &ctx->last_error)) return comm_err(ctx);
+    std::vector<SlabInfo> tab(nranks);
+    CZC_CUDA(ctx, cudaMemcpyAsync(tab.data(), ctx->dgather, nranks * sizeof(mine), cudaMemcpyDeviceToHost, s));
+    CZC_CUDA(ctx, cudaStreamSynchronize(s));
+    int64_t H = 0;
+    if (P.run_deriv) H = std::max<int64_t>(H, 1);
+    if (P.run_ac) H = std::max<int64_t>(H, P.T);
+    if (P.run_ssim) H = std::max<int64_t>(H, P.W - 1);
+    for (int r = 0; r < nranks; r++) {
+      const int64_t want_hi = std::min(H, F.nz - (tab[r].z0 + tab[r].nzl));
+      const bool contiguous = (r == 0 ? tab[r].z0 == 0 : tab[r].z0 == tab[r - 1].z0 + tab[r - 1].nzl);
+      if (!contiguous || tab[r].nzl < 1 || (r + 1 < nranks && tab[r + 1].nzl < want_hi) ||
+          (r == nranks - 1 && tab[r].z0 + tab[r].nzl != F.nz)) {
+        ctx->last_error = "slabs must tile dims[0] in rank order, each holding >= the halo depth";
+        return CZC_ERR_SHAPE;
+      }
+    }
+    hlo = (P.run_deriv && z0 > 0) ? 1 : 0;
+    hhi = std::min(H, F.nz - (z0 + nzl));
+    const int64_t prev_hhi = rank > 0 ? std::min(H, F.nz - z0) : 0;          // what rank-1 wants
+    const bool next_lo = P.run_deriv && rank + 1 < nranks;                  // rank+1 wants my last plane
+    const size_t pb = (size_t)plane * sizeof(float);
+    if ((st = ensure_buf(ctx, (void**)&ctx->halo, &ctx->halo_cap, 2 * (size_t)(hlo + hhi) * pb + 16)) != CZC_OK) return st;
+    float* xlo = ctx->halo;
+    float* ylo = xlo + hlo * plane;
+    float* xhi = ylo + hlo * plane;
+    float* yhi = xhi + hhi * plane;
+    if (!comm_group_begin(&ctx->last_error)) return comm_err(ctx);
+    bool ok = true;
+    if (rank > 0 && prev_hhi > 0) {
+      ok &= comm_send(ctx->comm, x, prev_hhi * pb, rank - 1, s, &ctx->last_error);
+      ok &= comm_send(ctx->comm, y, prev_hhi * pb, rank - 1, s, &ctx->last_error);
+    }
+    if (next_lo) {
+      ok &= comm_send(ctx->comm, x + (nzl - 1) * plane, pb, rank + 1, s, &ctx->last_error);
+      ok &= comm_send(ctx->comm, y + (nzl - 1) * plane, pb, rank + 1, s, &ctx->last_error);
+    }
+    if (hhi > 0) {
+      ok &= comm_recv(ctx->comm, xhi, hhi * pb, rank + 1, s, &ctx->last_error);
+      ok &= comm_recv(ctx->comm, yhi, hhi * pb, rank + 1, s, &ctx->last_error);
+    }
+    if (hlo > 0) {
+      ok &= comm_recv(ctx->comm, xlo, pb, rank - 1, s, &ctx->last_error);
+      ok &= comm_recv(ctx->comm, ylo, pb, rank - 1, s, &ctx->last_error);
+    }
+    if (!comm_group_end(&ctx->last_error) || !ok) return comm_err(ctx);
+    int k = 0;
+    if (hlo) { F.xs[k] = xlo; F.ys[k] = ylo; F.zs[k] = z0 - hlo; k++; }
+    F.xs[k] = x; F.ys[k] = y; F.zs[k] = z0; k++;
+    if (hhi) { F.xs[k] = xhi; F.ys[k] = yhi; F.zs[k] = z0 + nzl; k++; }
+    F.nseg = k;
+    F.zs[k] = z0 + nzl + hhi;
+  } else {
+    F.nseg = 1; F.xs[0] = x; F.ys[0] = y; F.zs[0] = 0; F.zs[1] = F.nz;
+  }
+
+  // ---- scratch sizing (partials of the largest launch) ------------------------------------------
+  size_t need = (size_t)ctx->p1_grid_cap * sizeof(P1State);
+  if (P.run_deriv) need = std::max(need, (size_t)deriv_blocks(F, zchunk_d) * kDerivSlots * sizeof(double));
+  if (P.run_ac) need = std::max(need, (size_t)ac_blocks(F, zchunk_ac) * kAcSlots * sizeof(double));
+  SsimParams sp{};
+  if (P.run_ssim) {
+    sp.sz = P.step[0]; sp.sy = P.step[1]; sp.sx = P.step[2];
+    sp.zchunk = zchunk_ss;
+    sp.range_mode = ctx->cfg.ssim_range_mode;
+    sp.nwz = (F.nz - P.win3[0]) / sp.sz + 1;
+    sp.nwy = (F.ny - P.win3[1]) / sp.sy + 1;
+    sp.nwx = (F.nx - P.win3[2]) / sp.sx + 1;
+    int64_t nb = 0;
+    if (launch_ssim(P.kind, P.W, F, sp, nullptr, nullptr, nullptr, nullptr, s, &nb) != cudaSuccess) {
+      ctx->last_error = "unsupported SSIM window";
+      return CZC_ERR_UNSUPPORTED;
+    }
+    need = std::max(need, (size_t)nb * kSsimSlots * sizeof(double));
+  }
+  if ((st = ensure_buf(ctx, &ctx->parts, &ctx->parts_cap, need)) != CZC_OK) return st;
+
+  // ---- launches (coordinator order P1 -> P2 -> P3; AC needs P1's mu_e, sigma_e^2, Alg. 2) --
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
+  if (P.run_p1) {
+    CZC_CUDA(ctx, launch_p1(x, y, P.n, ctx->p1_grid_cap, (P1State*)ctx->parts, ctx->dres, ctx->tickets + TICKET_P1, s));
+    if (slab) {   // one small allgather of the partial moments, merged in rank order on device
+      if (!comm_allgather(ctx->comm, &ctx->dres->p1, ctx->dgather, sizeof(P1State), s, &ctx->last_error)) return comm_err(ctx);
+      CZC_CUDA(ctx, launch_p1_combine((const P1State*)ctx->dgather, nranks, ctx->dres, s));
+    }
+  }
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
+  if (P.run_deriv)
+    CZC_CUDA(ctx, launch_deriv(F, zchunk_d, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_DERIV, s));
+  if (P.run_ac)
+    CZC_CUDA(ctx, launch_ac(F, P.T, zchunk_ac, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_AC, s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
+  if (P.run_ssim)
+    CZC_CUDA(ctx, launch_ssim(P.kind, P.W, F, sp, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_SSIM,
+                              ctx->cfg.debug_wssim, s, nullptr));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));
+  DevResults R;
+  if (slab) {   // second small allgather: the P2 / P3 slot records, combined in rank order
+    if (!comm_allgather(ctx->comm, ctx->dres, ctx->dgather, sizeof(DevResults), s, &ctx->last_error)) return comm_err(ctx);
+    CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hgather, ctx->dgather, nranks * sizeof(DevResults), cudaMemcpyDeviceToHost, s));
+  } else {
+    CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hres, ctx->dres, sizeof(DevResults), cudaMemcpyDeviceToHost, s));
+  }
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
+  CZC_CUDA(ctx, cudaStreamSynchronize(s));
+  if (slab) {
+    const DevResults* G = (const DevResults*)ctx->hgather;
+    R = G[0];
+    for (int r = 1; r < nranks; r++) {
+      for (int k = 0; k < kDerivSlots; k++) {
+        const int op = deriv_op(k);
+        R.deriv[k] = op == OP_SUM ? R.deriv[k] + G[r].deriv[k]
+                   : op == OP_MIN ? std::min(R.deriv[k], G[r].deriv[k]) : std::max(R.deriv[k], G[r].deriv[k]);
+      }
+      for (int k = 0; k < kAcSlots; k++) R.ac[k] += G[r].ac[k];
+      for (int k = 0; k < kSsimSlots; k++) R.ssim[k] += G[r].ssim[k];
+    }
+  } else {
+    R = *ctx->hres;
+  }
+  finish_all(P, R, mask, out);
+  if (timing) {
+    cudaEventElapsedTime(&out->kernel_ms[0], ctx->ev[0], ctx->ev[1]);
+    cudaEventElapsedTime(&out->kernel_ms[1], ctx->ev[1], ctx->ev[2]);
+    cudaEventElapsedTime(&out->kernel_ms[2], ctx->ev[2], ctx->ev[3]);
+    cudaEventElapsedTime(&out->kernel_ms[3], ctx->ev[0], ctx->ev[4]);
+  }
+  return CZC_OK;
+}
+
+static czc_status check_common(czc_ctx* ctx, const void* orig, const void* recon, const czc_shape* shape,
+                               czc_dtype dtype, czc_result* out) {
+  if (!out) return CZC_ERR_INVALID;
+  memset(out, 0, sizeof(*out));
+  if (!ctx || !orig || !recon || !shape) return CZC_ERR_INVALID;
+  if (dtype != CZC_F32) {
+    ctx->last_error = "only float32 fields are supported on the hot path";
+    return CZC_ERR_DTYPE;
+  }
+  return CZC_OK;
+}
+
+extern "C" czc_status czc_assess(czc_ctx* ctx, const void* orig, const void* recon, const czc_shape* shape,
+                                 czc_dtype dtype, uint64_t metric_mask, czc_result* out) {
+  czc_status st = check_common(ctx, orig, recon, shape, dtype, out);
+  if (st != CZC_OK) return st;
+  if (cudaSetDevice(ctx->device) != cudaSuccess) return cuda_fail(ctx, cudaGetLastError(), "cudaSetDevice");
+  st = assess_core(ctx, (const float*)orig, (const float*)recon, shape, metric_mask, out);
+  if (st != CZC_OK) out->computed_mask = 0;
+  return st;
+}
+
+extern "C" czc_status czc_assess_host(czc_ctx* ctx, const void* orig, const void* recon, const czc_shape* shape,
+                                      czc_dtype dtype, uint64_t metric_mask, czc_result* out) {
+  czc_status st = check_common(ctx, orig, recon, shape, dtype, out);
+  if (st != CZC_OK) return st;
+  if (shape->ndim < 1 || shape->ndim > 3) return CZC_ERR_SHAPE;
+  int64_t n = 1;
+  for (int i = 0; i < shape->ndim; i++) {
+    if (shape->dims[i] < 1) return CZC_ERR_SHAPE;
+    n *= (i == 0 && shape->nz_local > 0) ? shape->nz_local : shape->dims[i];
+  }
+  if (cudaSetDevice(ctx->device) != cudaSuccess) return cuda_fail(ctx, cudaGetLastError(), "cudaSetDevice");
+  const size_t bytes = (size_t)n * sizeof(float);
+  if (bytes > ctx->din_cap) {
+    cudaFree(ctx->din[0]);
+    cudaFree(ctx->din[1]);
+    ctx->din[0] = ctx->din[1] = nullptr;
+    ctx->din_cap = 0;
+    CZC_CUDA(ctx, cudaMalloc(&ctx->din[0], bytes));
+    CZC_CUDA(ctx, cudaMalloc(&ctx->din[1], bytes));
+    ctx->din_cap = bytes;
+  }
+  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->din[0], orig, bytes, cudaMemcpyHostToDevice, ctx->stream));
+  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->din[1], recon, bytes, cudaMemcpyHostToDevice, ctx->stream));
+  return czc_assess(ctx, ctx->din[0], ctx->din[1], shape, dtype, metric_mask, out);
+}

@@ -1,0 +1,234 @@
+// czc_internal.cuh — shared device/host definitions of the CUDA path (never used by oracle/).
+//
+// Partial-result records, the order-fixed (deterministic) cross-block finish, and small device
+// helpers.  Citations "Lnnn" are PAPER.md lines; DESIGN.md §5 describes the kernels.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string.h>
+
+#include "../../include/czc.h"
+
+// host/device bit casts
+__host__ __device__ inline double czc_bits_to_double(long long v) {
+#if defined(__CUDA_ARCH__)
+  return __longlong_as_double(v);
+#else
+  double d;
+  memcpy(&d, &v, 8);
+  return d;
+#endif
+}
+__host__ __device__ inline float czc_bits_to_float(int v) {
+#if defined(__CUDA_ARCH__)
+  return __int_as_float(v);
+#else
+  float f;
+  memcpy(&f, &v, 4);
+  return f;
+#endif
+}
+
+namespace czc {
+
+constexpr int kMaxWin = 16;      // largest SSIM window extent per axis on the fast path
+constexpr int kP1Threads = 256;
+constexpr int kFinishThreads = 256;
+
+__host__ __device__ inline double dinf() { return czc_bits_to_double(0x7ff0000000000000ll); }
+__host__ __device__ inline float finf() { return czc_bits_to_float(0x7f800000); }
+
+// ------------------------------------------------------------------------------------------------
+// P1 state in merge ("Chan") form: counts, means and centred co-moments.  Per-thread sums are
+// taken about the thread's first element (so the shifted-sum cancellation is bounded by the
+// thread's element count), converted to centred form once, and then merged pairwise with the
+// numerically stable update  M2 = M2a + M2b + d^2 na nb / n  (no catastrophic cancellation).
+// Fields map to Table I Category I (L107) and the north_star list; see DESIGN.md §5.1.
+// ------------------------------------------------------------------------------------------------
+struct P1State {
+  double n;                   // element count (exact as double below 2^53)
+  double mx, my, me;          // means of x, y, e = y - x
+  double m2x, m2y, cxy, m2e;  // sum (x-mx)^2, sum (y-my)^2, sum (x-mx)(y-my), sum (e-me)^2
+  double sae;                 // sum |e|
+  double emin, emax;          // extrema of e (exact doubles)
+  double pmin, pmax, spwr;    // point-wise relative error |e|/|x| over x != 0
+  double npwr;                // count of x != 0
+  float xmin, xmax;           // extrema of x (exact)
+};
+constexpr int kP1Words = sizeof(P1State) / 4;
+static_assert(sizeof(P1State) % 8 == 0, "P1State must be a whole number of doubles");
+
+__host__ __device__ inline void p1_empty(P1State& s) {
+  s.n = 0; s.mx = s.my = s.me = 0; s.m2x = s.m2y = s.cxy = s.m2e = 0; s.sae = 0;
+  s.emin = dinf(); s.emax = -dinf();
+  s.pmin = dinf(); s.pmax = -dinf(); s.spwr = 0; s.npwr = 0;
+  s.xmin = finf(); s.xmax = -finf();
+}
+
+__host__ __device__ inline void p1_merge(P1State& a, const P1State& b) {
+  a.sae += b.sae; a.spwr += b.spwr; a.npwr += b.npwr;
+  a.emin = b.emin < a.emin ? b.emin : a.emin;
+  a.emax = b.emax > a.emax ? b.emax : a.emax;
+  a.pmin = b.pmin < a.pmin ? b.pmin : a.pmin;
+  a.pmax = b.pmax > a.pmax ? b.pmax : a.pmax;
+  a.xmin = b.xmin < a.xmin ? b.xmin : a.xmin;
+  a.xmax = b.xmax > a.xmax ? b.xmax : a.xmax;
+  if (b.n == 0) return;
+  if (a.n == 0) {
+    a.n = b.n; a.mx = b.mx; a.my = b.my; a.me = b.me;
+    a.m2x = b.m2x; a.m2y = b.m2y; a.cxy = b.cxy; a.m2e = b.m2e;
+    return;
+  }
+  const double n = a.n + b.n, fb = b.n / n, g = a.n * fb;
+  const double dx = b.mx - a.mx, dy = b.my - a.my, de = b.me - a.me;
+  a.mx += dx * fb; a.my += dy * fb; a.me += de * fb;
+  a.m2x += b.m2x + dx * dx * g;
+  a.m2y += b.m2y + dy * dy * g;
+  a.cxy += b.cxy + dx * dy * g;
+  a.m2e += b.m2e + de * de * g;
+  a.n = n;
+}
+
+// ------------------------------------------------------------------------------------------------
+// Slot-wise partial records for P2 / P3: each block writes K doubles; the finish combines slot k
+// with its op (sum / min / max) in a fixed order, independent of block completion order.
+// ------------------------------------------------------------------------------------------------
+enum : int { OP_SUM = 0, OP_MIN = 1, OP_MAX = 2 };
+
+// Derivative record: per field f (5): [max|dF|, sum|dF|, sum dF^2, min F(x), max F(x)]
+constexpr int kDerivStats = 5;
+constexpr int kDerivSlots = kDerivStats * CZC_NDERIV;
+__host__ __device__ constexpr int deriv_op(int slot) {
+  return (slot % kDerivStats) == 0 ? OP_MAX : (slot % kDerivStats) == 3 ? OP_MIN
+       : (slot % kDerivStats) == 4 ? OP_MAX : OP_SUM;
+}
+// Autocorrelation record: S(tau) for tau = 1..CZC_MAX_LAG (index tau-1), all sums
+constexpr int kAcSlots = CZC_MAX_LAG;
+// SSIM record: [sum of local SSIM, number of windows, windows recomputed exactly]
+constexpr int kSsimSlots = 3;
+
+// Device-side results of one czc_assess call (fetched with one D2H copy at the end).
+struct DevResults {
+  P1State p1;
+  double deriv[kDerivSlots];
+  double ac[kAcSlots];
+  double ssim[kSsimSlots];
+};
+
+// A 3-D field view for the stencil / window kernels: global extents, the planes this launch
+// owns (stencil points / window origins), and up to three z-segments of plane storage (in slab
+// mode: the lower halo, the local slab and the upper halo received from the neighbour ranks).
+struct Field3 {
+  int64_t nz, ny, nx;        // GLOBAL extents (3-D view, inactive axes squeezed)
+  int64_t zown0, zown1;      // owned planes [zown0, zown1)
+  int nseg;                  // 1..3
+  const float* xs[3];
+  const float* ys[3];
+  int64_t zs[4];             // segment i holds global planes [zs[i], zs[i+1])
+#if defined(__CUDACC__)
+  __device__ __forceinline__ int seg(int64_t z) const {
+    return (nseg > 1 && z >= zs[1]) ? ((nseg > 2 && z >= zs[2]) ? 2 : 1) : 0;
+  }
+  __device__ __forceinline__ const float* xp(int64_t z) const {
+    const int s = seg(z);
+    return xs[s] + (z - zs[s]) * (ny * nx);
+  }
+  __device__ __forceinline__ const float* yp(int64_t z) const {
+    const int s = seg(z);
+    return ys[s] + (z - zs[s]) * (ny * nx);
+  }
+#endif
+};
+
+struct SsimParams {
+  int sz, sy, sx;            // steps
+  int zchunk;                // origin planes per block
+  int range_mode;            // 0 local L, 1 global L
+  int64_t nwz, nwy, nwx;     // window-grid extents (debug output indexing)
+};
+
+// Ticket counters for the last-block finish (zeroed once; the last block re-arms its counter).
+enum : int { TICKET_P1 = 0, TICKET_DERIV = 1, TICKET_AC = 2, TICKET_SSIM = 3, TICKET_N = 8 };
+
+#if defined(__CUDACC__)
+__device__ __forceinline__ double op_apply(int op, double a, double b) {
+  return op == OP_SUM ? a + b : op == OP_MIN ? fmin(a, b) : fmax(a, b);
+}
+__device__ __forceinline__ double op_identity(int op) {
+  return op == OP_SUM ? 0.0 : op == OP_MIN ? dinf() : -dinf();
+}
+
+// Returns true in exactly one block: the last to arrive.  All threads of every block call it
+// after the block's partial has been written.  Standard threadfence-reduction protocol.
+__device__ __forceinline__ bool last_block_arrive(unsigned int* ticket) {
+  __shared__ bool s_last;
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0 && threadIdx.y == 0 && threadIdx.z == 0) {
+    const unsigned int total = gridDim.x * gridDim.y * gridDim.z;
+    const unsigned int t = atomicAdd(ticket, 1u);
+    s_last = (t == total - 1);
+  }
+  __syncthreads();
+  if (s_last) __threadfence();
+  return s_last;
+}
+
+// Deterministic combine of K-slot records (run by every thread of the last block, 1-D view of
+// the block).  Thread t folds records t, t+T, t+2T, ... in increasing order; then a fixed
+// shuffle + shared-memory tree.  Result depends only on nblocks, never on arrival order.
+template <int K, typename OpOf>
+__device__ void finish_slots(const double* parts, int nblocks, OpOf op_of, double* out) {
+  __shared__ double s_red[32];
+  const int tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  const int nthr = blockDim.x * blockDim.y * blockDim.z;
+  const int lane = tid & 31, warp = tid >> 5, nwarps = (nthr + 31) >> 5;
+  for (int k = 0; k < K; k++) {
+    const int op = op_of(k);
+    double v = op_identity(op);
+    for (int b = tid; b < nblocks; b += nthr) v = op_apply(op, v, __ldcg(parts + (size_t)b * K + k));
+    for (int off = 16; off > 0; off >>= 1) v = op_apply(op, v, __shfl_down_sync(0xffffffffu, v, off));
+    if (lane == 0) s_red[warp] = v;
+    __syncthreads();
+    if (warp == 0) {
+      double w = lane < nwarps ? s_red[lane] : op_identity(op);
+      for (int off = 16; off > 0; off >>= 1) w = op_apply(op, w, __shfl_down_sync(0xffffffffu, w, off));
+      if (lane == 0) out[k] = w;
+    }
+    __syncthreads();
+  }
+}
+
+// Block-level combine of a per-thread K-slot record into slot values held by thread 0.
+template <int K, typename OpOf>
+__device__ void block_reduce_slots(double (&v)[K], OpOf op_of, double* dst_global) {
+  __shared__ double s_red[32];
+  const int tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  const int nthr = blockDim.x * blockDim.y * blockDim.z;
+  const int lane = tid & 31, warp = tid >> 5, nwarps = (nthr + 31) >> 5;
+#pragma unroll 1
+  for (int k = 0; k < K; k++) {
+    const int op = op_of(k);
+    double w = v[k];
+    for (int off = 16; off > 0; off >>= 1) w = op_apply(op, w, __shfl_down_sync(0xffffffffu, w, off));
+    if (lane == 0) s_red[warp] = w;
+    __syncthreads();
+    if (warp == 0) {
+      double u = lane < nwarps ? s_red[lane] : op_identity(op);
+      for (int off = 16; off > 0; off >>= 1) u = op_apply(op, u, __shfl_down_sync(0xffffffffu, u, off));
+      if (lane == 0) dst_global[k] = u;
+    }
+    __syncthreads();
+  }
+}
+
+__device__ __forceinline__ float4 ld_stream_f4(const float4* p) {
+  float4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(p));
+  return r;
+}
+#endif
+
+}  // namespace czc

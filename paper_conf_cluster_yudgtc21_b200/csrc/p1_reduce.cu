@@ -1,0 +1,217 @@
+// p1_reduce.cu — Pattern 1: fused global reduction over the (orig, recon) pair.
+//
+// Paper: Table I Category I (L107) — min/max/avg error, pwr error, MSE, RMSE, NRMSE, SNR, PSNR;
+// "one data read from global memory to registers can feed two reductions" (L118); Alg. 1
+// (L173-L203): per-thread strided reduce -> warp shuffles -> shared memory -> per-block partial
+// -> grid-level reduction.  B200 design: a persistent grid of 148 x k blocks
+// streams both arrays with 128-bit L1-bypassing loads; every element feeds all P1 statistics at
+// once; the per-block partials are combined by the last block to finish, in block-index order
+// (deterministic, no float atomics, no cooperative grid sync — reading R18).
+#include "czc_internal.cuh"
+
+namespace czc {
+
+// Per-thread accumulator: sums about the thread's first element (kx, ky, ke).
+struct P1Acc {
+  double n, kx, ky, ke;
+  double sa, sb, sc, saa, sbb, sab, scc, sae;
+  double emin, emax, pmin, pmax, spwr, npwr;
+  float xmin, xmax;
+};
+
+__device__ __forceinline__ void acc_init(P1Acc& a, float kxf, float kyf) {
+  a.n = 0;
+  a.kx = kxf; a.ky = kyf; a.ke = (double)kyf - (double)kxf;
+  a.sa = a.sb = a.sc = a.saa = a.sbb = a.sab = a.scc = a.sae = 0;
+  a.emin = dinf(); a.emax = -dinf(); a.pmin = dinf(); a.pmax = -dinf(); a.spwr = 0; a.npwr = 0;
+  a.xmin = finf(); a.xmax = -finf();
+}
+
+// One element: e = recon - orig in double (reading R1, exact rounding identical to the oracle);
+// the point-wise relative error |e|/|x| uses IEEE double division (bit-identical, reading R3).
+__device__ __forceinline__ void acc_elem(P1Acc& a, float xf, float yf) {
+  const double x = xf, y = yf;
+  const double e = y - x;
+  const double da = x - a.kx, db = y - a.ky, dc = e - a.ke;
+  a.n += 1.0;
+  a.sa += da; a.sb += db; a.sc += dc;
+  a.saa = fma(da, da, a.saa);
+  a.sbb = fma(db, db, a.sbb);
+  a.sab = fma(da, db, a.sab);
+  a.scc = fma(dc, dc, a.scc);
+  const double ae = fabs(e);
+  a.sae += ae;
+  a.emin = e < a.emin ? e : a.emin;
+  a.emax = e > a.emax ? e : a.emax;
+  a.xmin = fminf(a.xmin, xf);
+  a.xmax = fmaxf(a.xmax, xf);
+  const bool nz = xf != 0.0f;
+  const double q = ae / fabs(x);
+  a.spwr += nz ? q : 0.0;
+  a.npwr += nz ? 1.0 : 0.0;
+  a.pmin = (nz && q < a.pmin) ? q : a.pmin;
+  a.pmax = (nz && q > a.pmax) ? q : a.pmax;
+}
+
+__device__ __forceinline__ void acc_vec(P1Acc& a, float4 xv, float4 yv) {
+  acc_elem(a, xv.x, yv.x);
+  acc_elem(a, xv.y, yv.y);
+  acc_elem(a, xv.z, yv.z);
+  acc_elem(a, xv.w, yv.w);
+}
+
+__device__ __forceinline__ P1State acc_to_state(const P1Acc& a) {
+  P1State s;
+  p1_empty(s);
+  s.sae = a.sae; s.spwr = a.spwr; s.npwr = a.npwr;
+  s.emin = a.emin; s.emax = a.emax; s.pmin = a.pmin; s.pmax = a.pmax;
+  s.xmin = a.xmin; s.xmax = a.xmax;
+  if (a.n > 0) {
+    const double n = a.n;
+    s.n = n;
+    s.mx = a.kx + a.sa / n;
+    s.my = a.ky + a.sb / n;
+    s.me = a.ke + a.sc / n;
+    s.m2x = a.saa - a.sa * (a.sa / n);
+    s.m2y = a.sbb - a.sb * (a.sb / n);
+    s.cxy = a.sab - a.sa * (a.sb / n);
+    s.m2e = a.scc - a.sc * (a.sc / n);
+  }
+  return s;
+}
+
+__device__ __forceinline__ P1State shfl_down_state(const P1State& s, int off) {
+  P1State r;
+  const int* src = reinterpret_cast<const int*>(&s);
+  int* dst = reinterpret_cast<int*>(&r);
+#pragma unroll
+  for (int i = 0; i < kP1Words; i++) dst[i] = __shfl_down_sync(0xffffffffu, src[i], off);
+  return r;
+}
+
+// Merge the block's per-thread states in a fixed tree; result valid in thread 0.
+__device__ __forceinline__ P1State block_merge(P1State s) {
+  __shared__ P1State s_w[32];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+  for (int off = 16; off > 0; off >>= 1) {
+    P1State o = shfl_down_state(s, off);
+    if (lane + off < 32) p1_merge(s, o);
+  }
+  if (lane == 0) s_w[warp] = s;
+  __syncthreads();
+  if (warp == 0) {
+    if (lane < nw) s = s_w[lane]; else p1_empty(s);
+    for (int off = 16; off > 0; off >>= 1) {
+      P1State o = shfl_down_state(s, off);
+      if (lane + off < 32) p1_merge(s, o);
+    }
+  }
+  __syncthreads();
+  return s;
+}
+
+// VEC: x and y share the same 16-byte misalignment; elements [head, head + 4*nvec) are read as
+// float4, the <= 6 leftovers (prologue [0, head) and tail) by threads 0..nleft-1.
+template <bool VEC>
+__global__ void __launch_bounds__(kP1Threads)
+p1_kernel(const float* __restrict__ x, const float* __restrict__ y, int64_t n, int64_t head,
+          P1State* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket) {
+  const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
+  const int64_t nvec = VEC ? (n - head) / 4 : 0;
+  const int64_t tail0 = head + 4 * nvec;
+  const int64_t nleft = VEC ? head + (n - tail0) : n;   // scalar elements
+  auto left_index = [&](int64_t k) -> int64_t { return VEC ? (k < head ? k : tail0 + (k - head)) : k; };
+
+  P1Acc a;
+  int64_t first = -1;
+  if (VEC && gtid < nvec) first = head + 4 * gtid;
+  else if (gtid < nleft) first = left_index(gtid);
+  acc_init(a, first >= 0 ? x[first] : 0.0f, first >= 0 ? y[first] : 0.0f);
+
+  if (VEC) {
+    const float4* x4 = reinterpret_cast<const float4*>(x + head);
+    const float4* y4 = reinterpret_cast<const float4*>(y + head);
+    int64_t v = gtid;
+    for (; v + 3 * gsz < nvec; v += 4 * gsz) {   // 4 independent 2x16-byte loads in flight
+      const float4 xa = ld_stream_f4(x4 + v), ya = ld_stream_f4(y4 + v);
+      const float4 xb = ld_stream_f4(x4 + v + gsz), yb = ld_stream_f4(y4 + v + gsz);
+      const float4 xc = ld_stream_f4(x4 + v + 2 * gsz), yc = ld_stream_f4(y4 + v + 2 * gsz);
+      const float4 xd = ld_stream_f4(x4 + v + 3 * gsz), yd = ld_stream_f4(y4 + v + 3 * gsz);
+      acc_vec(a, xa, ya);
+      acc_vec(a, xb, yb);
+      acc_vec(a, xc, yc);
+      acc_vec(a, xd, yd);
+    }
+    for (; v < nvec; v += gsz) acc_vec(a, ld_stream_f4(x4 + v), ld_stream_f4(y4 + v));
+    if (gtid < nleft) {
+      const int64_t i = left_index(gtid);
+      acc_elem(a, x[i], y[i]);
+    }
+  } else {
+    for (int64_t i = gtid; i < n; i += gsz) acc_elem(a, x[i], y[i]);
+  }
+
+  P1State s = block_merge(acc_to_state(a));
+  if (threadIdx.x == 0) parts[blockIdx.x] = s;
+  if (!last_block_arrive(ticket)) return;
+
+  // Last block: fold the partials in block-index order (thread t: t, t+T, ...), fixed tree.
+  P1State f;
+  p1_empty(f);
+  for (int b = threadIdx.x; b < (int)gridDim.x; b += blockDim.x) {
+    P1State pb;
+    const double* src = reinterpret_cast<const double*>(parts + b);
+    double* dst = reinterpret_cast<double*>(&pb);
+#pragma unroll
+    for (int i = 0; i < (int)(sizeof(P1State) / 8); i++) dst[i] = __ldcg(src + i);
+    p1_merge(f, pb);
+  }
+  f = block_merge(f);
+  if (threadIdx.x == 0) {
+    res->p1 = f;
+    *ticket = 0;   // re-arm for the next launch
+  }
+}
+
+// Host launcher.  Returns the cuda error of the launch.
+cudaError_t launch_p1(const float* x, const float* y, int64_t n, int grid_cap, P1State* parts,
+                      DevResults* res, unsigned int* ticket, cudaStream_t st) {
+  const uintptr_t ax = reinterpret_cast<uintptr_t>(x), ay = reinterpret_cast<uintptr_t>(y);
+  const bool vec = (ax % 16) == (ay % 16) && (ax % 4) == 0;
+  int64_t head = 0;
+  if (vec) head = (int64_t)(((16 - ax % 16) % 16) / 4);
+  if (head > n) head = n;
+  const int64_t work = vec ? ((n - head) / 4 + 8) : n;
+  int64_t blocks = (work + kP1Threads - 1) / kP1Threads;
+  if (blocks > grid_cap) blocks = grid_cap;
+  if (blocks < 1) blocks = 1;
+  if (vec)
+    p1_kernel<true><<<(unsigned)blocks, kP1Threads, 0, st>>>(x, y, n, head, parts, res, ticket);
+  else
+    p1_kernel<false><<<(unsigned)blocks, kP1Threads, 0, st>>>(x, y, n, head, parts, res, ticket);
+  return cudaGetLastError();
+}
+
+// Slab mode: merge the allgathered per-rank states in rank order (every rank runs the same code
+// on the same bytes, so all ranks hold identical results).
+__global__ void p1_combine_kernel(const P1State* __restrict__ states, int count, DevResults* __restrict__ res) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  P1State f;
+  p1_empty(f);
+  for (int r = 0; r < count; r++) p1_merge(f, states[r]);
+  res->p1 = f;
+}
+
+cudaError_t launch_p1_combine(const P1State* states, int count, DevResults* res, cudaStream_t st) {
+  p1_combine_kernel<<<1, 32, 0, st>>>(states, count, res);
+  return cudaGetLastError();
+}
+
+int p1_max_blocks_per_sm() {
+  int nb = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, p1_kernel<true>, kP1Threads, 0);
+  return nb > 0 ? nb : 1;
+}
+
+}  // namespace czc

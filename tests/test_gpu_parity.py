@@ -1,0 +1,208 @@
+"""CUDA path vs CPU oracle, element by element on the same seeded inputs, through the C ABI.
+
+Sizes span several tiles with ragged tails; edge cases cover 1-D/2-D, inactive axes, misaligned
+pointers, steps, global-range SSIM, zero error, sparse fields and an adversarial step field.
+Full-size (BASELINE configs[1]) checks compare all of P1/P2 and sampled SSIM windows."""
+import math
+
+import numpy as np
+import pytest
+import torch
+
+import synth
+from parity_util import check_ac, check_deriv, check_p1, check_ssim, report
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def czc():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_cluster_yudgtc21_b200 as m
+    m.get_lib()
+    return m
+
+
+def run_both(czc, orc, x, y, window=8, step=1, lag=10, range_mode=0, mask=None):
+    """GPU (through czc_assess) and oracle on the same host arrays."""
+    xn, yn = np.ascontiguousarray(x), np.ascontiguousarray(y)
+    xd, yd = torch.from_numpy(xn).cuda(), torch.from_numpy(yn).cuda()
+    nd = xn.ndim
+    with czc.Assessor(ndim=nd, ssim_window=window, ssim_step=step, ac_max_lag=lag,
+                      ssim_range_mode=range_mode) as a:
+        g = a.assess(xd, yd, czc.M_ALL if mask is None else mask)
+    o = {}
+    o.update(orc.p1(xn, yn))
+    o.update(orc.deriv(xn, yn))
+    o["ac"], o["ac_count"] = orc.autocorr(xn, yn, lag)
+    w = [window] * nd if isinstance(window, int) else list(window)
+    s = [step] * nd if isinstance(step, int) else list(step)
+    o["ssim"], o["n_windows"] = orc.ssim(xn, yn, w, s, range_mode)
+    return g, o
+
+
+def full_check(g, o, ssim_tol=1e-6):
+    errors = []
+    check_p1(g, o, errors)
+    check_deriv(g, o, errors)
+    check_ac(g["ac"], g["ac_count"], o["ac"], o["ac_count"], errors)
+    check_ssim(g["ssim"], g["n_windows"], o["ssim"], o["n_windows"], errors, ssim_tol)
+    report(errors)
+
+
+CASES = [
+    ("C1", (64, 64, 64), 7),
+    ("C1", (13, 17, 35), 5),
+    ("C2", (40, 70, 90), 8),
+    ("C2q", (36, 66, 75), 8),
+    ("C3", (33, 45, 61), 8),
+    ("C4", (180, 360), 8),
+    ("C4", (77, 1000), 16),
+    ("C1", (20, 33, 40), 2),
+    ("C2", (9, 300, 41), 3),
+]
+
+
+@pytest.mark.parametrize("cfg,dims,w", CASES)
+def test_parity_configs(czc, orc, cfg, dims, w):
+    x, y = synth.make_pair(synth.config(cfg, dims=dims))
+    g, o = run_both(czc, orc, x.numpy(), y.numpy(), window=w)
+    assert g["computed_mask"] == czc.M_ALL
+    full_check(g, o)
+
+
+@pytest.mark.parametrize("lag", [1, 4, 16])
+def test_lags(czc, orc, lag):
+    x, y = synth.make_pair(synth.config("C1", dims=(24, 28, 40)))
+    g, o = run_both(czc, orc, x.numpy(), y.numpy(), window=4, lag=lag)
+    errors = []
+    check_ac(g["ac"], g["ac_count"], o["ac"], o["ac_count"], errors)
+    report(errors)
+
+
+@pytest.mark.parametrize("step", [2, 3, (1, 2, 3)])
+def test_steps(czc, orc, step):
+    x, y = synth.make_pair(synth.config("C1", dims=(21, 34, 47)))
+    g, o = run_both(czc, orc, x.numpy(), y.numpy(), window=5, step=step)
+    full_check(g, o)
+
+
+def test_global_range_mode(czc, orc):
+    x, y = synth.make_pair(synth.config("C1", dims=(22, 40, 50)))
+    g, o = run_both(czc, orc, x.numpy(), y.numpy(), window=7, range_mode=1)
+    full_check(g, o)
+
+
+def test_one_dimensional_and_inactive_axes(czc, orc):
+    x, y = synth.make_pair(synth.config("C4", dims=(7, 1000)))
+    xn, yn = x.numpy()[3].copy(), y.numpy()[3].copy()            # 1-D
+    g, o = run_both(czc, orc, xn, yn, window=9)
+    full_check(g, o)
+    x3, y3 = x.numpy()[:, None, :].copy(), y.numpy()[:, None, :].copy()   # (7, 1, 1000)
+    g, o = run_both(czc, orc, x3, y3, window=(5, 1, 5))
+    full_check(g, o)
+
+
+def test_zero_error(czc, orc):
+    x, _ = synth.make_pair(synth.config("C2q", dims=(20, 30, 40)))
+    xn = x.numpy()
+    g, o = run_both(czc, orc, xn, xn.copy(), window=6)
+    full_check(g, o)
+    assert g["psnr"] == math.inf and g["mse"] == 0 and g["ssim"] == 1.0
+    assert all(math.isnan(v) for v in g["ac"][1:])
+
+
+def test_adversarial_step_field(czc, orc):
+    x, y = synth.make_pair(synth.config("C1", dims=(18, 20, 64), kind="step", recon="quant", eb=0.1))
+    g, o = run_both(czc, orc, x.numpy(), y.numpy(), window=8)
+    full_check(g, o)
+
+
+def test_misaligned_pointers(czc, orc):
+    """Same 4-byte offset on both arrays (vector path with prologue) and different offsets
+    (scalar path): P1 is flat, so views of a larger buffer exercise both."""
+    base_x, base_y = synth.make_pair(synth.config("C1", dims=(5, 77, 131)))
+    bx, by = base_x.numpy().ravel(), base_y.numpy().ravel()
+    n = 50000
+    for ox, oy in ((1, 1), (3, 3), (1, 2), (0, 3)):
+        xs = torch.from_numpy(bx).cuda()[ox:ox + n]
+        ys = torch.from_numpy(by).cuda()[oy:oy + n]
+        with czc.Assessor(ndim=1) as a:
+            g = a.assess(xs, ys, czc.M_P1)
+        o = orc.p1(bx[ox:ox + n], by[oy:oy + n])
+        errors = []
+        check_p1(g, o, errors)
+        report(errors)
+
+
+def test_determinism(czc):
+    x, y = synth.make_pair(synth.config("C3", dims=(40, 64, 96)))
+    xd, yd = x.cuda(), y.cuda()
+    outs = []
+    with czc.Assessor(ssim_window=8) as a:
+        for _ in range(5):
+            r = a.assess(xd, yd)
+            outs.append({k: (v.tobytes() if isinstance(v, np.ndarray) else v) for k, v in r.items() if k != "kernel_ms"})
+    for r in outs[1:]:
+        for k in r:
+            a_, b_ = r[k], outs[0][k]
+            assert a_ == b_ or (isinstance(a_, float) and math.isnan(a_) and math.isnan(b_)), k
+
+
+def test_errors(czc):
+    x = torch.zeros((5, 6, 7), device="cuda")
+    with czc.Assessor(ssim_window=8) as a:
+        with pytest.raises(czc.CzcError) as ei:
+            a.assess(x, x, czc.M_SSIM)               # window larger than the field
+        assert ei.value.status == 2
+        r = a.assess(x, x, czc.M_P1)                   # the context stays usable
+        assert r["computed_mask"] == czc.M_P1
+    with czc.Assessor(ssim_window=(8, 4, 8)) as a:
+        with pytest.raises(czc.CzcError) as ei:
+            a.assess(torch.zeros((20, 20, 20), device="cuda"), torch.zeros((20, 20, 20), device="cuda"), czc.M_SSIM)
+        assert ei.value.status == 7
+
+
+def test_debug_windows_match_oracle(czc, orc):
+    x, y = synth.make_pair(synth.config("C2q", dims=(30, 50, 70)))
+    xn, yn = x.numpy(), y.numpy()
+    w = 8
+    nw = [n - w + 1 for n in xn.shape]
+    dbg = torch.full(nw, float("nan"), dtype=torch.float64, device="cuda")
+    with czc.Assessor(ssim_window=w, debug_wssim=dbg.data_ptr()) as a:
+        g = a.assess(x.cuda(), y.cuda(), czc.M_SSIM)
+    d = dbg.cpu().numpy()
+    assert not np.isnan(d).any()
+    assert abs(d.mean() - g["ssim"]) < 1e-12
+    rng = np.random.default_rng(7)
+    for _ in range(300):
+        o = [int(rng.integers(0, k)) for k in nw]
+        ref = orc.ssim_window(xn, yn, o, [w] * 3)
+        assert abs(d[tuple(o)] - ref) < 1e-6, (o, d[tuple(o)], ref)
+
+
+@pytest.mark.slow
+def test_full_size_hurricane(czc, orc):
+    """BASELINE configs[1]: 100 x 500 x 500 pair, full metric set, bench launch configuration."""
+    spec = synth.CONFIGS["C2"]
+    x, y = synth.make_pair(spec)
+    xn, yn = x.numpy(), y.numpy()
+    nw = [n - 8 + 1 for n in xn.shape]
+    dbg = torch.empty(nw, dtype=torch.float64, device="cuda")
+    with czc.Assessor(ssim_window=8, debug_wssim=dbg.data_ptr()) as a:
+        g = a.assess(x.cuda(), y.cuda())
+    errors = []
+    check_p1(g, orc.p1(xn, yn), errors)
+    check_deriv(g, orc.deriv(xn, yn), errors)
+    ac, cnt = orc.autocorr(xn, yn, 10)
+    check_ac(g["ac"], g["ac_count"], ac, cnt, errors)
+    report(errors)
+    d = dbg.cpu().numpy()
+    assert g["n_windows"] == np.prod(nw)
+    assert abs(d.mean() - g["ssim"]) < 1e-12
+    rng = np.random.default_rng(11)
+    for _ in range(400):
+        o = [int(rng.integers(0, k)) for k in nw]
+        ref = orc.ssim_window(xn, yn, o, [8, 8, 8])
+        assert abs(d[tuple(o)] - ref) < 1e-6, (o, d[tuple(o)], ref)
