@@ -305,7 +305,8 @@ void finish_all(const Plan& P, const DevResults& R, uint64_t mask, czc_result* o
       int64_t ne = 1;
       for (int a = 0; a < 3; a++) ne *= P.g3[a] > 1 ? P.g3[a] - t : 1;
       out->ac_count[t] = (uint64_t)ne;
-      out->ac[t] = var > 0 ? R.ac[t - 1] / (double)P.D / (double)ne / var : NAN;
+      const double S = R.ac[0][t - 1] + R.ac[1][t - 1] + R.ac[2][t - 1];   // z, y, x walks
+      out->ac[t] = var > 0 ? S / (double)P.D / (double)ne / var : NAN;
     }
     done |= CZC_M_AUTOCORR;
   }
@@ -449,7 +450,7 @@ static czc_status assess_core(czc_ctx* ctx, const float* x, const float* y, cons
   if (P.run_deriv)
     CZC_CUDA(ctx, launch_deriv(F, zchunk_d, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_DERIV, s));
   if (P.run_ac)
-    CZC_CUDA(ctx, launch_ac(F, P.T, zchunk_ac, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_AC, s));
+    CZC_CUDA(ctx, launch_ac(F, P.T, zchunk_ac, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_ACZ, s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
   if (P.run_ssim)
     CZC_CUDA(ctx, launch_ssim(P.kind, P.W, F, sp, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_SSIM,
@@ -473,7 +474,8 @@ static czc_status assess_core(czc_ctx* ctx, const float* x, const float* y, cons
         R.deriv[k] = op == OP_SUM ? R.deriv[k] + G[r].deriv[k]
                    : op == OP_MIN ? std::min(R.deriv[k], G[r].deriv[k]) : std::max(R.deriv[k], G[r].deriv[k]);
       }
-      for (int k = 0; k < kAcSlots; k++) R.ac[k] += G[r].ac[k];
+      for (int w = 0; w < kAcWalks; w++)
+        for (int k = 0; k < kAcSlots; k++) R.ac[w][k] += G[r].ac[w][k];
       for (int k = 0; k < kSsimSlots; k++) R.ssim[k] += G[r].ssim[k];
     }
   } else {

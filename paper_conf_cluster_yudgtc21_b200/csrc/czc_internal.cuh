@@ -103,8 +103,10 @@ __host__ __device__ constexpr int deriv_op(int slot) {
   return (slot % kDerivStats) == 0 ? OP_MAX : (slot % kDerivStats) == 3 ? OP_MIN
        : (slot % kDerivStats) == 4 ? OP_MAX : OP_SUM;
 }
-// Autocorrelation record: S(tau) for tau = 1..CZC_MAX_LAG (index tau-1), all sums
+// Autocorrelation record: S(tau) for tau = 1..CZC_MAX_LAG (index tau-1), all sums; one record
+// per walk axis (z, y, x), summed at the finish.
 constexpr int kAcSlots = CZC_MAX_LAG;
+constexpr int kAcWalks = 3;
 // SSIM record: [sum of local SSIM, number of windows, windows recomputed exactly]
 constexpr int kSsimSlots = 3;
 
@@ -112,7 +114,7 @@ constexpr int kSsimSlots = 3;
 struct DevResults {
   P1State p1;
   double deriv[kDerivSlots];
-  double ac[kAcSlots];
+  double ac[kAcWalks][kAcSlots];
   double ssim[kSsimSlots];
 };
 
@@ -127,16 +129,19 @@ struct Field3 {
   const float* ys[3];
   int64_t zs[4];             // segment i holds global planes [zs[i], zs[i+1])
 #if defined(__CUDACC__)
-  __device__ __forceinline__ int seg(int64_t z) const {
-    return (nseg > 1 && z >= zs[1]) ? ((nseg > 2 && z >= zs[2]) ? 2 : 1) : 0;
-  }
+  // Plane pointers.  Segment selection uses static indices only (a dynamic index into the
+  // by-value kernel parameter would force a local-memory copy of the struct).
   __device__ __forceinline__ const float* xp(int64_t z) const {
-    const int s = seg(z);
-    return xs[s] + (z - zs[s]) * (ny * nx);
+    const bool s1 = nseg > 1 && z >= zs[1], s2 = nseg > 2 && z >= zs[2];
+    const float* b = s2 ? xs[2] : (s1 ? xs[1] : xs[0]);
+    const int64_t z0 = s2 ? zs[2] : (s1 ? zs[1] : zs[0]);
+    return b + (z - z0) * (ny * nx);
   }
   __device__ __forceinline__ const float* yp(int64_t z) const {
-    const int s = seg(z);
-    return ys[s] + (z - zs[s]) * (ny * nx);
+    const bool s1 = nseg > 1 && z >= zs[1], s2 = nseg > 2 && z >= zs[2];
+    const float* b = s2 ? ys[2] : (s1 ? ys[1] : ys[0]);
+    const int64_t z0 = s2 ? zs[2] : (s1 ? zs[1] : zs[0]);
+    return b + (z - z0) * (ny * nx);
   }
 #endif
 };
@@ -149,7 +154,7 @@ struct SsimParams {
 };
 
 // Ticket counters for the last-block finish (zeroed once; the last block re-arms its counter).
-enum : int { TICKET_P1 = 0, TICKET_DERIV = 1, TICKET_AC = 2, TICKET_SSIM = 3, TICKET_N = 8 };
+enum : int { TICKET_P1 = 0, TICKET_DERIV = 1, TICKET_SSIM = 2, TICKET_ACZ = 3, TICKET_ACY = 4, TICKET_ACX = 5, TICKET_N = 8 };
 
 #if defined(__CUDACC__)
 __device__ __forceinline__ double op_apply(int op, double a, double b) {
@@ -207,7 +212,7 @@ __device__ void block_reduce_slots(double (&v)[K], OpOf op_of, double* dst_globa
   const int tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
   const int nthr = blockDim.x * blockDim.y * blockDim.z;
   const int lane = tid & 31, warp = tid >> 5, nwarps = (nthr + 31) >> 5;
-#pragma unroll 1
+#pragma unroll
   for (int k = 0; k < K; k++) {
     const int op = op_of(k);
     double w = v[k];

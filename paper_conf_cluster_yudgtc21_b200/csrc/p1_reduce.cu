@@ -11,29 +11,47 @@
 
 namespace czc {
 
-// Per-thread accumulator: sums about the thread's first element (kx, ky, ke).
+// Per-thread accumulator: sums about the thread's first element (kx, ky, ke).  The element count
+// is implicit (counted per vector), so no per-element work is spent on it.
 struct P1Acc {
-  double n, kx, ky, ke;
+  double kx, ky, ke;
   double sa, sb, sc, saa, sbb, sab, scc, sae;
-  double emin, emax, pmin, pmax, spwr, npwr;
+  double emin, emax, pmin, pmax, spwr;
+  double pthr_hi, pthr_lo;          // candidate thresholds for the exact pwr extrema
+  unsigned npwr;                    // count of x != 0 (per thread, < 2^32)
   float xmin, xmax;
 };
 
 __device__ __forceinline__ void acc_init(P1Acc& a, float kxf, float kyf) {
-  a.n = 0;
   a.kx = kxf; a.ky = kyf; a.ke = (double)kyf - (double)kxf;
   a.sa = a.sb = a.sc = a.saa = a.sbb = a.sab = a.scc = a.sae = 0;
-  a.emin = dinf(); a.emax = -dinf(); a.pmin = dinf(); a.pmax = -dinf(); a.spwr = 0; a.npwr = 0;
+  a.emin = dinf(); a.emax = -dinf(); a.pmin = dinf(); a.pmax = -dinf(); a.spwr = 0;
+  a.pthr_hi = -dinf(); a.pthr_lo = dinf();
+  a.npwr = 0;
   a.xmin = finf(); a.xmax = -finf();
 }
 
-// One element: e = recon - orig in double (reading R1, exact rounding identical to the oracle);
-// the point-wise relative error |e|/|x| uses IEEE double division (bit-identical, reading R3).
+// 1/v for v > 0 (finite, normal): rcp.approx (MUFU.RCP64H) + two Newton steps -> |rel err| <= 2u.
+__device__ __forceinline__ double fast_rcp(double v) {
+  double r;
+  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(v));
+  double e = fma(-v, r, 1.0);
+  r = fma(r, e, r);
+  e = fma(-v, r, 1.0);
+  return fma(r, e, r);
+}
+
+// One element: e = recon - orig in double (reading R1; same rounding as the oracle).  Point-wise
+// relative error |e|/|x| (reading R3): its SUM uses q~ = |e| * rcp(|x|) (relative error <= 4u,
+// far inside the 1e-9 tolerance of pwr_mean); its extrema must be the IEEE quotient, bit-exact
+// with the oracle, so the correctly rounded division runs only for candidates: an element can be
+// the maximum only if q~ >= pmax (1 - 1e-12) (q~ >= Q (1 - 4u) and pmax <= RN(Q) for the true
+// maximum Q), and symmetrically for the minimum.  After the first few elements of a thread
+// candidates are rare, so the division is off the hot path.
 __device__ __forceinline__ void acc_elem(P1Acc& a, float xf, float yf) {
   const double x = xf, y = yf;
   const double e = y - x;
   const double da = x - a.kx, db = y - a.ky, dc = e - a.ke;
-  a.n += 1.0;
   a.sa += da; a.sb += db; a.sc += dc;
   a.saa = fma(da, da, a.saa);
   a.sbb = fma(db, db, a.sbb);
@@ -46,11 +64,15 @@ __device__ __forceinline__ void acc_elem(P1Acc& a, float xf, float yf) {
   a.xmin = fminf(a.xmin, xf);
   a.xmax = fmaxf(a.xmax, xf);
   const bool nz = xf != 0.0f;
-  const double q = ae / fabs(x);
-  a.spwr += nz ? q : 0.0;
-  a.npwr += nz ? 1.0 : 0.0;
-  a.pmin = (nz && q < a.pmin) ? q : a.pmin;
-  a.pmax = (nz && q > a.pmax) ? q : a.pmax;
+  const double ax = nz ? fabs(x) : 1.0;
+  const double qa = nz ? ae * fast_rcp(ax) : 0.0;
+  a.spwr += qa;
+  a.npwr += nz ? 1u : 0u;
+  if (nz && (qa >= a.pthr_hi || qa <= a.pthr_lo)) {
+    const double q = ae / ax;                        // IEEE, correctly rounded
+    if (q > a.pmax) { a.pmax = q; a.pthr_hi = q * (1.0 - 1e-12); }
+    if (q < a.pmin) { a.pmin = q; a.pthr_lo = q * (1.0 + 1e-12); }
+  }
 }
 
 __device__ __forceinline__ void acc_vec(P1Acc& a, float4 xv, float4 yv) {
@@ -60,14 +82,13 @@ __device__ __forceinline__ void acc_vec(P1Acc& a, float4 xv, float4 yv) {
   acc_elem(a, xv.w, yv.w);
 }
 
-__device__ __forceinline__ P1State acc_to_state(const P1Acc& a) {
+__device__ __forceinline__ P1State acc_to_state(const P1Acc& a, double n) {
   P1State s;
   p1_empty(s);
-  s.sae = a.sae; s.spwr = a.spwr; s.npwr = a.npwr;
+  s.sae = a.sae; s.spwr = a.spwr; s.npwr = (double)a.npwr;
   s.emin = a.emin; s.emax = a.emax; s.pmin = a.pmin; s.pmax = a.pmax;
   s.xmin = a.xmin; s.xmax = a.xmax;
-  if (a.n > 0) {
-    const double n = a.n;
+  if (n > 0) {
     s.n = n;
     s.mx = a.kx + a.sa / n;
     s.my = a.ky + a.sb / n;
@@ -124,15 +145,17 @@ p1_kernel(const float* __restrict__ x, const float* __restrict__ y, int64_t n, i
   auto left_index = [&](int64_t k) -> int64_t { return VEC ? (k < head ? k : tail0 + (k - head)) : k; };
 
   P1Acc a;
-  int64_t first = -1;
+  int64_t first = -1;   // anchor = the thread's first element
   if (VEC && gtid < nvec) first = head + 4 * gtid;
   else if (gtid < nleft) first = left_index(gtid);
   acc_init(a, first >= 0 ? x[first] : 0.0f, first >= 0 ? y[first] : 0.0f);
 
+  int64_t cnt = 0;                                 // elements processed by this thread
   if (VEC) {
     const float4* x4 = reinterpret_cast<const float4*>(x + head);
     const float4* y4 = reinterpret_cast<const float4*>(y + head);
     int64_t v = gtid;
+    if (gtid < nvec) cnt = 4 * ((nvec - 1 - gtid) / gsz + 1);
     for (; v + 3 * gsz < nvec; v += 4 * gsz) {   // 4 independent 2x16-byte loads in flight
       const float4 xa = ld_stream_f4(x4 + v), ya = ld_stream_f4(y4 + v);
       const float4 xb = ld_stream_f4(x4 + v + gsz), yb = ld_stream_f4(y4 + v + gsz);
@@ -147,12 +170,14 @@ p1_kernel(const float* __restrict__ x, const float* __restrict__ y, int64_t n, i
     if (gtid < nleft) {
       const int64_t i = left_index(gtid);
       acc_elem(a, x[i], y[i]);
+      cnt += 1;
     }
   } else {
+    if (gtid < n) cnt = (n - 1 - gtid) / gsz + 1;
     for (int64_t i = gtid; i < n; i += gsz) acc_elem(a, x[i], y[i]);
   }
 
-  P1State s = block_merge(acc_to_state(a));
+  P1State s = block_merge(acc_to_state(a, (double)cnt));
   if (threadIdx.x == 0) parts[blockIdx.x] = s;
   if (!last_block_arrive(ticket)) return;
 

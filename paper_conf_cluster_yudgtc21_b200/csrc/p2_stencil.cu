@@ -8,39 +8,66 @@
 // Readings R7, R9, R11, R12, R13.  AC needs P1's mean / variance of the error
 // (Alg. 2 takes mu as input, L226): it is read from the device result of P1, no host round trip.
 //
-// B200 design: blocks own a 32 x 8 (x, y) column tile and stream along z; the
-// z-neighbours live in registers, the in-plane neighbours in a shared-memory plane with halo;
-// per-thread FP64 accumulators; block partials combined by the last block in index order.
+// B200 design.
+//  * Derivatives: a block owns a 32 x 8 column tile and streams z; the z-neighbours live in
+//    registers (prefetched one plane ahead), the in-plane neighbours come from a double-buffered
+//    shared-memory plane with a 1-cell halo (one __syncthreads per plane).
+//  * Autocorrelation: Eq. 2's sum splits into one lag-product sum per axis,
+//      S(tau) = sum_a sum_{p in R_tau} eps_p eps_{p + tau e_a},
+//    each computed by a "line walk" along that axis: a thread walks a line, keeps the last TM
+//    values of eps in a register ring (static rotation: the walk is unrolled by TM) and adds
+//    eps_{i-tau} * eps_i for tau <= min(T, m_line), where m_line is the R_tau bound of the
+//    line's other coordinates.  z- and y-walks read coalesced rows directly; the x-walk goes
+//    through a warp-private shared-memory transpose.  Every product is formed exactly once.
+// FP64 accumulators per thread; block partials combined by the last block in index order.
 #include "czc_internal.cuh"
 
 namespace czc {
 
 constexpr int kTX = 32, kTY = 8;
 
+// ================================================================================================
+// Derivatives
+// ================================================================================================
+// sqrt for FP64 without the correctly-rounded slow path: rsqrt.approx + two Newton steps,
+// relative error ~2^-52 (the oracle's sqrt differs by at most ~1 ulp; metrics are compared with
+// a 1e-9 relative tolerance).  sqrt(0) = 0.
+__device__ __forceinline__ double fast_sqrt(double a) {
+  double r;
+  asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(a));
+  r = r * fma(-0.5 * a, r * r, 1.5);
+  r = r * fma(-0.5 * a, r * r, 1.5);
+  const double g = a * r;
+  return a > 0.0 ? g : 0.0;
+}
+__device__ __forceinline__ double dmax(double a, double b) { return a > b ? a : b; }
+__device__ __forceinline__ double dmin(double a, double b) { return a < b ? a : b; }
+
+// Derived fields of one point.  AXES is compile-time: 3 -> (z, y, x), 2 -> (y, x), 1 -> (x).
+// Axis order z, y, x (slowest first) as in the oracle.
+template <int AXES>
 __device__ __forceinline__ void deriv_fields(const double c, const double zp, const double zm,
                                              const double yp, const double ym, const double xp,
-                                             const double xm, bool az, bool ay, bool ax,
-                                             double F[CZC_NDERIV]) {
+                                             const double xm, double F[CZC_NDERIV]) {
   double der1 = 0, der2 = 0, g2 = 0, div = 0, lap = 0;
-  // axis order z, y, x (slowest first) — same as the oracle
-#define CZC_AXIS(ACT, P, M)                     \
-  if (ACT) {                                    \
+#define CZC_AXIS(P, M)                          \
+  {                                             \
     const double delta = (P) - (M);             \
-    const double D = delta / 2.0;               \
+    const double D = delta * 0.5;               \
     const double l = (P) - 2.0 * c + (M);       \
     der1 += fabs(delta);                        \
     der2 += fabs(l);                            \
-    g2 += D * D;                                \
+    g2 = fma(D, D, g2);                         \
     div += D;                                   \
     lap += l;                                   \
   }
-  CZC_AXIS(az, zp, zm)
-  CZC_AXIS(ay, yp, ym)
-  CZC_AXIS(ax, xp, xm)
+  if (AXES >= 3) CZC_AXIS(zp, zm)
+  if (AXES >= 2) CZC_AXIS(yp, ym)
+  CZC_AXIS(xp, xm)
 #undef CZC_AXIS
   F[CZC_DER1] = der1;
   F[CZC_DER2] = der2;
-  F[CZC_GRAD] = sqrt(g2);
+  F[CZC_GRAD] = fast_sqrt(g2);
   F[CZC_DIV] = div;
   F[CZC_LAP] = lap;
 }
@@ -52,22 +79,24 @@ struct SumOp {
   __device__ int operator()(int) const { return OP_SUM; }
 };
 
-// grid: (ceil(nx/32), ceil(ny/8), nzchunks); block (32, 8)
-__global__ void __launch_bounds__(kTX * kTY)
-deriv_kernel(Field3 s, int zchunk,
-             double* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket) {
-  __shared__ double sx[kTY + 2][kTX + 2];
-  __shared__ double sy[kTY + 2][kTX + 2];
+constexpr int kHalo = 2 * (kTX + 2) + 2 * kTY;   // halo cells of one plane tile
+
+// grid: (ceil(nx/32), ceil(ny/8), zchunks); block (32, 8).  AXES: active axes (3, 2 or 1).
+template <int AXES>
+__global__ void __launch_bounds__(kTX * kTY, 2)
+deriv_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+             unsigned int* __restrict__ ticket) {
+  __shared__ double2 pl[2][kTY + 2][kTX + 2];     // (x, y) of the current plane, double-buffered
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * kTX + tx;
   const int64_t gx = (int64_t)blockIdx.x * kTX + tx, gy = (int64_t)blockIdx.y * kTY + ty;
-  const bool az = s.nz > 1, ay = s.ny > 1, ax = s.nx > 1;
-  const int64_t plane = s.ny * s.nx;
-  // interior ranges (reading R11)
+  constexpr bool az = AXES >= 3, ay = AXES >= 2;
+  // interior ranges (reading R11), restricted to the owned planes
   int64_t zlo = az ? 1 : 0, zhi = az ? s.nz - 1 : 1;
   if (zlo < s.zown0) zlo = s.zown0;
   if (zhi > s.zown1) zhi = s.zown1;
-  const bool inxy = (ay ? (gy >= 1 && gy < s.ny - 1) : gy == 0) && (ax ? (gx >= 1 && gx < s.nx - 1) : gx == 0);
-  int64_t zb = zlo + (int64_t)blockIdx.z * zchunk, ze = zb + zchunk;
+  const bool inxy = (ay ? (gy >= 1 && gy < s.ny - 1) : gy == 0) && (gx >= 1 && gx < s.nx - 1);
+  const int64_t zb = zlo + (int64_t)blockIdx.z * zchunk;
+  int64_t ze = zb + zchunk;
   if (ze > zhi) ze = zhi;
 
   double acc[kDerivSlots];
@@ -75,48 +104,53 @@ deriv_kernel(Field3 s, int zchunk,
   for (int k = 0; k < kDerivSlots; k++) acc[k] = op_identity(deriv_op(k));
 
   const bool own = gx < s.nx && gy < s.ny;
-  const int64_t col = gy * s.nx + gx;
-  double xm = 0, x0 = 0, xp = 0, ym = 0, y0 = 0, yp = 0;
-  if (own && zb < ze) {
-    x0 = s.xp(zb)[col]; y0 = s.yp(zb)[col];
-    if (az) { xm = s.xp(zb - 1)[col]; ym = s.yp(zb - 1)[col]; }
+  const int64_t col = own ? gy * s.nx + gx : 0;
+  // halo cell of this thread (tid < kHalo): row hr, column hc of the padded tile
+  int hr = 0, hc = 0;
+  if (tid < 2 * (kTX + 2)) { hr = tid < kTX + 2 ? 0 : kTY + 1; hc = tid % (kTX + 2); }
+  else if (tid < kHalo) { const int t = tid - 2 * (kTX + 2); hr = 1 + t % kTY; hc = t < kTY ? 0 : kTX + 1; }
+  const int64_t hy = (int64_t)blockIdx.y * kTY + hr - 1, hx = (int64_t)blockIdx.x * kTX + hc - 1;
+  const bool hown = tid < kHalo && hy >= 0 && hy < s.ny && hx >= 0 && hx < s.nx;
+  const int64_t hcol = hown ? hy * s.nx + hx : 0;
+
+  double xm = 0, x0 = 0, ym = 0, y0 = 0;
+  float nxv = 0.f, nyv = 0.f, nhx = 0.f, nhy = 0.f;   // prefetched: own at z+1, halo at z
+  if (zb < ze) {
+    if (own) {
+      x0 = s.xp(zb)[col]; y0 = s.yp(zb)[col];
+      if (az) { xm = s.xp(zb - 1)[col]; ym = s.yp(zb - 1)[col]; nxv = s.xp(zb + 1)[col]; nyv = s.yp(zb + 1)[col]; }
+    }
+    if (hown) { nhx = s.xp(zb)[hcol]; nhy = s.yp(zb)[hcol]; }
   }
   for (int64_t z = zb; z < ze; z++) {
-    if (own && az) { xp = s.xp(z + 1)[col]; yp = s.yp(z + 1)[col]; }
-    const float* Xz = s.xp(z);
-    const float* Yz = s.yp(z);
-    // stage plane z (own + 1-cell halo) as doubles
-    for (int i = tid; i < (kTY + 2) * (kTX + 2); i += kTX * kTY) {
-      const int r = i / (kTX + 2), c = i % (kTX + 2);
-      const int64_t yy = (int64_t)blockIdx.y * kTY + r - 1, xx = (int64_t)blockIdx.x * kTX + c - 1;
-      double vx = 0, vy = 0;
-      if (yy >= 0 && yy < s.ny && xx >= 0 && xx < s.nx) {
-        vx = Xz[yy * s.nx + xx];
-        vy = Yz[yy * s.nx + xx];
-      }
-      sx[r][c] = vx;
-      sy[r][c] = vy;
-    }
+    const int buf = (int)((z - zb) & 1);
+    const double xp = az ? (double)nxv : 0.0, yp = az ? (double)nyv : 0.0;
+    const float hxv = nhx, hyv = nhy;
+    // prefetch: own column at z+2, halo at z+1
+    if (own && az && z + 2 <= s.nz - 1 && z + 1 < ze) { nxv = __ldg(s.xp(z + 2) + col); nyv = __ldg(s.yp(z + 2) + col); }
+    if (hown && z + 1 < ze) { nhx = __ldg(s.xp(z + 1) + hcol); nhy = __ldg(s.yp(z + 1) + hcol); }
+    pl[buf][ty + 1][tx + 1] = make_double2(x0, y0);
+    if (tid < kHalo) pl[buf][hr][hc] = make_double2(hxv, hyv);
     __syncthreads();
     if (own && inxy) {
+      const double2 yn = pl[buf][ty + 2][tx + 1], ys = pl[buf][ty][tx + 1];
+      const double2 xe = pl[buf][ty + 1][tx + 2], xw = pl[buf][ty + 1][tx];
       double Fx[CZC_NDERIV], Fy[CZC_NDERIV];
-      deriv_fields(x0, xp, xm, sx[ty + 2][tx + 1], sx[ty][tx + 1], sx[ty + 1][tx + 2], sx[ty + 1][tx], az, ay, ax, Fx);
-      deriv_fields(y0, yp, ym, sy[ty + 2][tx + 1], sy[ty][tx + 1], sy[ty + 1][tx + 2], sy[ty + 1][tx], az, ay, ax, Fy);
+      deriv_fields<AXES>(x0, xp, xm, yn.x, ys.x, xe.x, xw.x, Fx);
+      deriv_fields<AXES>(y0, yp, ym, yn.y, ys.y, xe.y, xw.y, Fy);
 #pragma unroll
-      for (int f = 0; f < CZC_NDERIV; f++) {
-        const double d = Fy[f] - Fx[f];
-        double* a = acc + f * kDerivStats;
-        a[0] = fmax(a[0], fabs(d));
-        a[1] += fabs(d);
-        a[2] = fma(d, d, a[2]);
-        a[3] = fmin(a[3], Fx[f]);
-        a[4] = fmax(a[4], Fx[f]);
+      for (int fi = 0; fi < CZC_NDERIV; fi++) {
+        const double d = Fy[fi] - Fx[fi];
+        acc[fi * kDerivStats + 0] = dmax(acc[fi * kDerivStats + 0], fabs(d));
+        acc[fi * kDerivStats + 1] += fabs(d);
+        acc[fi * kDerivStats + 2] = fma(d, d, acc[fi * kDerivStats + 2]);
+        acc[fi * kDerivStats + 3] = dmin(acc[fi * kDerivStats + 3], Fx[fi]);
+        acc[fi * kDerivStats + 4] = dmax(acc[fi * kDerivStats + 4], Fx[fi]);
       }
     }
-    __syncthreads();
     xm = x0; x0 = xp; ym = y0; y0 = yp;
   }
-
+  __syncthreads();
   const unsigned bid = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
   block_reduce_slots<kDerivSlots>(acc, DerivOp{}, parts + (size_t)bid * kDerivSlots);
   if (!last_block_arrive(ticket)) return;
@@ -124,88 +158,188 @@ deriv_kernel(Field3 s, int zchunk,
   if (tid == 0) *ticket = 0;
 }
 
-// ------------------------------------------------------------------------------------------------
-// Autocorrelation (Eq. 2).  Ring of T+1 planes of eps = e - mu (FP64) in shared memory, tile of
-// 32 x 8 points plus a +T halo in x and y.  Point p of plane zp is processed once planes
-// zp..zp+T are resident; lag tau contributes iff p in R_tau, i.e. tau <= m(p) = min over active
-// axes of (n_a - 1 - p_a).  S(tau) accumulates eps_p * sum_a eps_{p + tau e_a}.
-// ------------------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kTX * kTY)
-ac_kernel(Field3 s, int T, int zchunk,
-          double* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket) {
-  extern __shared__ double ring[];   // [(T+1)][kTY+T][kTX+T]
-  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * kTX + tx;
-  const int FY = kTY + T, FX = kTX + T, R = T + 1;
-  const int64_t gx = (int64_t)blockIdx.x * kTX + tx, gy = (int64_t)blockIdx.y * kTY + ty;
-  const bool az = s.nz > 1, ay = s.ny > 1, ax = s.nx > 1;
-  const int64_t plane = s.ny * s.nx;
-  const double mu = res->p1.me;
-  const int64_t zb = s.zown0 + (int64_t)blockIdx.z * zchunk;
-  int64_t ze = zb + zchunk;
-  if (ze > s.zown1) ze = s.zown1;
-
-  double acc[kAcSlots];
+// ================================================================================================
+// Autocorrelation line walks
+// ================================================================================================
+// One walk step at ring slot S (S is a constant once the caller's loop is unrolled, so the ring
+// indexing is static).  The ring holds eps of the last TM positions of the walk, zero-filled for
+// positions before the owned range [lo, hi) and for positions >= hi (those points belong to the
+// next chunk), so every product eps_{i-t} * eps_i that should not count is exactly 0 * eps_i and
+// no per-lag predicate is needed.  The R_tau bound of the line (t <= lim) is applied once, at the
+// end (`walk_mask`).
+template <int TM>
+__device__ __forceinline__ void walk_step(double (&ring)[TM], double (&acc)[TM], double eps, bool keep, int S) {
 #pragma unroll
-  for (int k = 0; k < kAcSlots; k++) acc[k] = 0;
+  for (int t = 1; t <= TM; t++) acc[t - 1] = fma(ring[(S - t + 2 * TM) % TM], eps, acc[t - 1]);
+  ring[S] = keep ? eps : 0.0;
+}
 
-  auto load_plane = [&](int64_t zl) {
-    double* dst = ring + (size_t)(zl % R) * FY * FX;
-    const float* Xz = s.xp(zl);
-    const float* Yz = s.yp(zl);
-    for (int i = tid; i < FY * FX; i += kTX * kTY) {
-      const int r = i / FX, c = i % FX;
-      const int64_t yy = (int64_t)blockIdx.y * kTY + r, xx = (int64_t)blockIdx.x * kTX + c;
-      double v = 0;
-      if (yy < s.ny && xx < s.nx) {
-        const int64_t idx = yy * s.nx + xx;
-        v = ((double)Yz[idx] - (double)Xz[idx]) - mu;
-      }
-      dst[i] = v;
-    }
-  };
-  // m(p) over the in-plane axes (z handled per plane)
-  int64_t mxy = INT64_MAX;
-  if (ay) mxy = min(mxy, s.ny - 1 - gy);
-  if (ax) mxy = min(mxy, s.nx - 1 - gx);
-  const bool own = gx < s.nx && gy < s.ny;
-
-  if (zb < ze) {
-    const int64_t pre_end = (zb + (int64_t)T < s.nz) ? zb + (int64_t)T : s.nz;   // planes zb .. zb+T-1
-    for (int64_t zl = zb; zl < pre_end; zl++) load_plane(zl);
-  }
-  for (int64_t zp = zb; zp < ze; zp++) {
-    if (zp + T < s.nz) load_plane(zp + T);
-    __syncthreads();
-    if (own) {
-      int64_t m = mxy;
-      if (az) m = min(m, s.nz - 1 - zp);
-      const int mlim = (int)(m < (int64_t)T ? m : (int64_t)T);
-      const int sp = (int)(zp % R);
-      const double* P0 = ring + (size_t)sp * FY * FX;
-      const double ep = P0[ty * FX + tx];
+template <int TM>
+__device__ __forceinline__ void walk_mask(double (&acc)[TM], int lim) {
 #pragma unroll
-      for (int tau = 1; tau <= CZC_MAX_LAG; tau++) {
-        if (tau <= mlim) {
-          double nb = 0;
-          if (az) {
-            int sl = sp + tau;
-            if (sl >= R) sl -= R;
-            nb += ring[(size_t)sl * FY * FX + ty * FX + tx];
-          }
-          if (ay) nb += P0[(ty + tau) * FX + tx];
-          if (ax) nb += P0[ty * FX + tx + tau];
-          acc[tau - 1] = fma(ep, nb, acc[tau - 1]);
-        }
-      }
-    }
-    __syncthreads();
-  }
+  for (int t = 1; t <= TM; t++)
+    if (t > lim) acc[t - 1] = 0.0;
+}
 
+template <int TM>
+__device__ __forceinline__ void ac_finish(double (&acc)[TM], double* parts, double* out, unsigned int* ticket) {
+  double rec[kAcSlots];
+#pragma unroll
+  for (int t = 0; t < kAcSlots; t++) rec[t] = 0.0;
+#pragma unroll
+  for (int t = 0; t < TM; t++) rec[t] = acc[t];
   const unsigned bid = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
-  block_reduce_slots<kAcSlots>(acc, SumOp{}, parts + (size_t)bid * kAcSlots);
+  __syncthreads();
+  block_reduce_slots<kAcSlots>(rec, SumOp{}, parts + (size_t)bid * kAcSlots);
   if (!last_block_arrive(ticket)) return;
-  finish_slots<kAcSlots>(parts, gridDim.x * gridDim.y * gridDim.z, SumOp{}, res->ac);
-  if (tid == 0) *ticket = 0;
+  finish_slots<kAcSlots>(parts, gridDim.x * gridDim.y * gridDim.z, SumOp{}, out);
+  if (threadIdx.x + threadIdx.y == 0) *ticket = 0;
+}
+
+// Walk of one line with element stride `stride` through up to three plane segments (z-walk) or a
+// single row (y-walk: stride nx within one plane).  Positions [lo, end) are visited; points p in
+// [lo, hi) own their products.  TM loads are kept in flight in a register queue (slot u of the
+// TM-unrolled loop holds position i0 + u), so the queue also rotates statically.
+template <int TM, typename PtrOf>
+__device__ __forceinline__ void walk_line(PtrOf ptr_of, int64_t lo, int64_t hi, int64_t end, double mu,
+                                          bool own, double (&ring)[TM], double (&acc)[TM]) {
+  float qx[TM], qy[TM];
+#pragma unroll
+  for (int u = 0; u < TM; u++) {
+    qx[u] = 0.f; qy[u] = 0.f;
+    if (own && lo + u < end) { const float2 v = ptr_of(lo + u); qx[u] = v.x; qy[u] = v.y; }
+  }
+  for (int64_t i0 = lo; i0 < end; i0 += TM) {
+#pragma unroll
+    for (int u = 0; u < TM; u++) {
+      const int64_t i = i0 + u;
+      if (i < end) {
+        const double eps = ((double)qy[u] - (double)qx[u]) - mu;
+        if (own && i + TM < end) { const float2 v = ptr_of(i + TM); qx[u] = v.x; qy[u] = v.y; }
+        walk_step<TM>(ring, acc, eps, i < hi, u);
+      }
+    }
+  }
+}
+
+// z-walk: thread <-> column (y, x); block 32 x 8 columns; grid.z chunks of owned planes.
+template <int TM>
+__global__ void __launch_bounds__(256)
+ac_zwalk(Field3 s, int T, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+         unsigned int* __restrict__ ticket) {
+  const int64_t gx = (int64_t)blockIdx.x * kTX + threadIdx.x, gy = (int64_t)blockIdx.y * kTY + threadIdx.y;
+  const double mu = res->p1.me;
+  const bool own = gx < s.nx && gy < s.ny;
+  int64_t m = T;
+  if (s.ny > 1 && s.ny - 1 - gy < m) m = s.ny - 1 - gy;
+  if (s.nx > 1 && s.nx - 1 - gx < m) m = s.nx - 1 - gx;
+  const int64_t lo = s.zown0 + (int64_t)blockIdx.z * zchunk;
+  int64_t hi = lo + zchunk;
+  if (hi > s.zown1) hi = s.zown1;
+  int64_t end = hi + T;
+  if (end > s.nz) end = s.nz;
+  const int64_t col = own ? gy * s.nx + gx : 0;
+  double ring[TM], acc[TM];
+#pragma unroll
+  for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
+  walk_line<TM>([&](int64_t z) { return make_float2(__ldg(s.xp(z) + col), __ldg(s.yp(z) + col)); }, lo, hi, end, mu, own, ring, acc);
+  walk_mask<TM>(acc, own ? (int)m : 0);
+  ac_finish<TM>(acc, parts, res->ac[0], ticket);
+}
+
+// y-walk: thread <-> line (z, x); block 32 (x) x 8 (z); grid.z chunks of y.
+template <int TM>
+__global__ void __launch_bounds__(256)
+ac_ywalk(Field3 s, int T, int ychunk, double* __restrict__ parts, DevResults* __restrict__ res,
+         unsigned int* __restrict__ ticket) {
+  const int64_t gx = (int64_t)blockIdx.x * kTX + threadIdx.x;
+  const int64_t z = s.zown0 + (int64_t)blockIdx.y * kTY + threadIdx.y;
+  const double mu = res->p1.me;
+  const bool own = gx < s.nx && z < s.zown1;
+  int64_t m = T;
+  if (s.nz > 1 && s.nz - 1 - z < m) m = s.nz - 1 - z;
+  if (s.nx > 1 && s.nx - 1 - gx < m) m = s.nx - 1 - gx;
+  const int64_t lo = (int64_t)blockIdx.z * ychunk;
+  int64_t hi = lo + ychunk;
+  if (hi > s.ny) hi = s.ny;
+  int64_t end = hi + T;
+  if (end > s.ny) end = s.ny;
+  const float* X = own ? s.xp(z) + gx : nullptr;
+  const float* Y = own ? s.yp(z) + gx : nullptr;
+  const int64_t nx = s.nx;
+  double ring[TM], acc[TM];
+#pragma unroll
+  for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
+  walk_line<TM>([&](int64_t y) { return make_float2(__ldg(X + y * nx), __ldg(Y + y * nx)); }, lo, hi, end, mu, own, ring, acc);
+  walk_mask<TM>(acc, own ? (int)m : 0);
+  ac_finish<TM>(acc, parts, res->ac[1], ticket);
+}
+
+// x-walk: each warp owns 32 consecutive rows (z, y); per segment of SEG columns (a multiple of
+// TM, so the ring slot of column c is (c - lo) mod TM, static under unrolling) it stages the rows
+// coalesced into a warp-private shared-memory tile (transpose), then lane l walks row l.  The
+// staged row's (z, y) advance incrementally (no divisions in the loop).
+constexpr int kXWarps = 4;   // 4 warps x 32 rows per block (tile: 4 x 32 x <=33 doubles <= 34 KB)
+template <int TM>
+__global__ void __launch_bounds__(kXWarps * 32)
+ac_xwalk(Field3 s, int T, int xchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+         unsigned int* __restrict__ ticket) {
+  constexpr int SEG = (32 / TM) * TM;
+  __shared__ double tile[kXWarps][32][SEG + 1];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const double mu = res->p1.me;
+  const int64_t nrows = (s.zown1 - s.zown0) * s.ny;
+  const int64_t row0 = ((int64_t)blockIdx.x * kXWarps + warp) * 32;   // first row of this warp
+  const int64_t myrow = row0 + lane;
+  const bool own = myrow < nrows;
+  const int64_t z = own ? s.zown0 + myrow / s.ny : 0, y = own ? myrow % s.ny : 0;
+  int64_t m = T;
+  if (s.nz > 1 && s.nz - 1 - z < m) m = s.nz - 1 - z;
+  if (s.ny > 1 && s.ny - 1 - y < m) m = s.ny - 1 - y;
+  const int64_t lo = (int64_t)blockIdx.y * xchunk;
+  int64_t hi = lo + xchunk;
+  if (hi > s.nx) hi = s.nx;
+  int64_t end = hi + T;
+  if (end > s.nx) end = s.nx;
+  const int64_t zr0 = s.zown0 + (row0 < nrows ? row0 : 0) / s.ny, yr0 = (row0 < nrows ? row0 : 0) % s.ny;
+  double ring[TM], acc[TM];
+#pragma unroll
+  for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
+  double (*tl)[SEG + 1] = tile[warp];
+  for (int64_t c0 = lo; c0 < end; c0 += SEG) {
+    // stage 32 rows x SEG columns of eps, coalesced per row; rows advance (y, z) incrementally
+    int64_t zr = zr0, yr = yr0;
+    const float* X = s.xp(zr) + yr * s.nx;
+    const float* Y = s.yp(zr) + yr * s.nx;
+    const int64_t c = c0 + lane;
+    const bool cin = lane < SEG && c < end;
+#pragma unroll 4
+    for (int i = 0; i < 32; i++) {
+      double v = 0;
+      if (cin && row0 + i < nrows) v = ((double)__ldg(Y + c) - (double)__ldg(X + c)) - mu;
+      if (lane < SEG) tl[i][lane] = v;
+      if (++yr == s.ny) {
+        yr = 0;
+        ++zr;
+        if (row0 + i + 1 < nrows) { X = s.xp(zr); Y = s.yp(zr); }
+      } else {
+        X += s.nx;
+        Y += s.nx;
+      }
+    }
+    __syncwarp();
+    const int64_t ncol = (end - c0) < SEG ? (end - c0) : SEG;
+    for (int j0 = 0; j0 < SEG; j0 += TM) {
+#pragma unroll
+      for (int u = 0; u < TM; u++) {
+        const int j = j0 + u;
+        if (j < ncol) walk_step<TM>(ring, acc, tl[lane][j], c0 + j < hi, u);
+      }
+    }
+    __syncwarp();
+  }
+  walk_mask<TM>(acc, own ? (int)m : 0);
+  ac_finish<TM>(acc, parts, res->ac[2], ticket);
 }
 
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
@@ -219,28 +353,64 @@ static int64_t deriv_zplanes(const Field3& s) {
 int64_t deriv_blocks(const Field3& s, int zchunk) {
   return cdiv(s.nx, kTX) * cdiv(s.ny, kTY) * cdiv(deriv_zplanes(s), zchunk);
 }
-int64_t ac_blocks(const Field3& s, int zchunk) {
-  const int64_t nzo = s.zown1 > s.zown0 ? s.zown1 - s.zown0 : 1;
-  return cdiv(s.nx, kTX) * cdiv(s.ny, kTY) * cdiv(nzo, zchunk);
-}
-size_t ac_smem_bytes(int T) { return (size_t)(T + 1) * (kTY + T) * (kTX + T) * sizeof(double); }
 
 cudaError_t launch_deriv(const Field3& s, int zchunk, double* parts, DevResults* res,
                          unsigned int* ticket, cudaStream_t st) {
   dim3 grid((unsigned)cdiv(s.nx, kTX), (unsigned)cdiv(s.ny, kTY), (unsigned)cdiv(deriv_zplanes(s), zchunk));
-  deriv_kernel<<<grid, dim3(kTX, kTY), 0, st>>>(s, zchunk, parts, res, ticket);
+  if (s.nz > 1) deriv_kernel<3><<<grid, dim3(kTX, kTY), 0, st>>>(s, zchunk, parts, res, ticket);
+  else if (s.ny > 1) deriv_kernel<2><<<grid, dim3(kTX, kTY), 0, st>>>(s, zchunk, parts, res, ticket);
+  else deriv_kernel<1><<<grid, dim3(kTX, kTY), 0, st>>>(s, zchunk, parts, res, ticket);
   return cudaGetLastError();
 }
 
-cudaError_t launch_ac(const Field3& s, int T, int zchunk, double* parts, DevResults* res,
-                      unsigned int* ticket, cudaStream_t st) {
-  const size_t smem = ac_smem_bytes(T);
-  cudaError_t e = cudaFuncSetAttribute(ac_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+// Autocorrelation: one launch per active walk axis, each with its own partial-buffer slice and
+// ticket; the three records are summed at the finish.
+struct AcGrids {
+  dim3 z, y, x;
+  bool rz, ry, rx;
+  int zc, yc, xc;
+};
+static AcGrids ac_grids(const Field3& s) {
+  AcGrids g{};
+  const int64_t nzo = s.zown1 - s.zown0;
+  g.zc = 50; g.yc = 125; g.xc = 125;
+  g.rz = s.nz > 1; g.ry = s.ny > 1; g.rx = s.nx > 1;
+  g.z = dim3((unsigned)cdiv(s.nx, kTX), (unsigned)cdiv(s.ny, kTY), (unsigned)cdiv(nzo, g.zc));
+  g.y = dim3((unsigned)cdiv(s.nx, kTX), (unsigned)cdiv(nzo, kTY), (unsigned)cdiv(s.ny, g.yc));
+  g.x = dim3((unsigned)cdiv(nzo * s.ny, kXWarps * 32), (unsigned)cdiv(s.nx, g.xc), 1);
+  return g;
+}
+int64_t ac_blocks(const Field3& s, int) {
+  const AcGrids g = ac_grids(s);
+  auto n = [](dim3 d) { return (int64_t)d.x * d.y * d.z; };
+  return n(g.z) + n(g.y) + n(g.x);
+}
+
+template <int TM>
+static cudaError_t launch_ac_t(const Field3& s, int T, double* parts, DevResults* res,
+                               unsigned int* tickets, cudaStream_t st) {
+  const AcGrids g = ac_grids(s);
+  double* pz = parts;
+  double* py = pz + (size_t)g.z.x * g.z.y * g.z.z * kAcSlots;
+  double* px = py + (size_t)g.y.x * g.y.y * g.y.z * kAcSlots;
+  cudaError_t e = cudaMemsetAsync(res->ac, 0, sizeof(res->ac), st);
   if (e != cudaSuccess) return e;
-  const int64_t nzo = s.zown1 > s.zown0 ? s.zown1 - s.zown0 : 1;
-  dim3 grid((unsigned)cdiv(s.nx, kTX), (unsigned)cdiv(s.ny, kTY), (unsigned)cdiv(nzo, zchunk));
-  ac_kernel<<<grid, dim3(kTX, kTY), smem, st>>>(s, T, zchunk, parts, res, ticket);
+  if (g.rz) ac_zwalk<TM><<<g.z, dim3(kTX, kTY), 0, st>>>(s, T, g.zc, pz, res, tickets + 0);
+  if (g.ry) ac_ywalk<TM><<<g.y, dim3(kTX, kTY), 0, st>>>(s, T, g.yc, py, res, tickets + 1);
+  if (g.rx) ac_xwalk<TM><<<g.x, kXWarps * 32, 0, st>>>(s, T, g.xc, px, res, tickets + 2);
   return cudaGetLastError();
+}
+
+// tickets: three consecutive counters (z, y, x walks)
+cudaError_t launch_ac(const Field3& s, int T, int, double* parts, DevResults* res,
+                      unsigned int* tickets, cudaStream_t st) {
+  if (T <= 2) return launch_ac_t<2>(s, T, parts, res, tickets, st);
+  if (T <= 4) return launch_ac_t<4>(s, T, parts, res, tickets, st);
+  if (T <= 6) return launch_ac_t<6>(s, T, parts, res, tickets, st);
+  if (T <= 8) return launch_ac_t<8>(s, T, parts, res, tickets, st);
+  if (T <= 10) return launch_ac_t<10>(s, T, parts, res, tickets, st);
+  if (T <= 12) return launch_ac_t<12>(s, T, parts, res, tickets, st);
+  return launch_ac_t<16>(s, T, parts, res, tickets, st);
 }
 
 }  // namespace czc

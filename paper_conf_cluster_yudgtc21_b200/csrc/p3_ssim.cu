@@ -4,219 +4,255 @@
 // fields; at each position the window's min, max, sum and power sums are reduced, "mixed (by some
 // simple sums and multiplications) to generate the local SSIM", and a global reduction averages
 // the local SSIMs.  The paper's kernel keeps per-slice window partials in a shared-memory FIFO of
-// depth w along z so each slice is "read and processed only once" (L270, L318).
+// depth w along z so each slice is "read and processed only once" (L270, L318), shares the
+// x-direction through warp shuffles and the y-direction through shared memory (L270, L320).
 //
-// B200 design.  A block owns a tile of 32 (x) x 8 (y) window origins and a chunk
-// of origin planes, and streams z:
-//   (a) z-walk: every thread owns footprint columns (y, x) of the tile + halo and keeps FP64
-//       running sums over the last WZ planes of the four anchored moments
+// B200 design.  A block = 8 warps owns a tile of (32 - WX + 1) x (8 G) window
+// origins and a chunk of origin planes, and streams z.  Lane l of warp w owns the footprint
+// columns (rows w, w+8, ...; column l) of the tile and, per plane:
+//   (a) z-walk — keeps FP64 running sums over the last WZ planes of four anchored moments
 //         a = x - K,  e = y - x,  a*b (b = y - K),  e*e
-//       (the leaving plane comes from a shared-memory ring of raw (x, y) — the paper's FIFO moved
-//       from window partials to raw samples), plus the z-window min / max of x from the ring;
-//   (b) y-pass: running sums over WY rows, segments of 4 origins per thread;
-//   (c) x-pass: running sums over WX columns, then the per-window mix in the cancellation-free
-//       two-factor form  ssim = A/(A + mu_e^2) * B/(B + s_e^2),  A = 2 mu_x mu_y + C1,
-//       B = 2 s_xy + C2  (identical to Wang et al.'s formula with C3 = C2/2, reading R14), with
-//       L = max - min of the original window (reading R15) or the global range.
+//       in registers; the leaving plane's x sits in a per-thread register ring (the paper's
+//       FIFO, moved from window partials to raw samples; the ring rotates statically because
+//       the plane loop is unrolled by WZ), which also gives the z-window min/max of x, and its
+//       y is re-read from L2; the next plane is prefetched into registers one plane ahead;
+//   (b) y-pass — after ONE __syncthreads on a double-buffered shared-memory exchange of the
+//       z-sums, each warp forms running sums over WY rows for its G origin rows;
+//   (c) x-pass — power-of-two doubling with warp shuffles across the 32 lanes (the paper's
+//       shfl_down x-reduction, L270), then the per-window mix in the cancellation-free form
+//         ssim = A/(A + mu_e^2) * B/(B + s_e^2),  A = 2 mu_x mu_y + C1,  B = 2 s_xy + C2
+//       (identical to Wang et al.'s formula with C3 = C2/2, reading R14), with L = max - min of
+//       the original window (reading R15) or the global range.
 // K is one anchor per block (the tile-centre sample of its first plane) so the moment sums stay
-// small; all sums are FP64.  Window extents are compile-time (cubic 3-D, square 2-D, or 1-D).
+// small; every sum is FP64.  Window extents are compile-time (cubic 3-D, square 2-D, 1-D).
 #include "czc_internal.cuh"
 
 namespace czc {
 
-constexpr int kOX = 32;     // origins per tile along x
-constexpr int kOY = 8;      // origins per tile along y
-constexpr int kSeg = 4;     // origins per thread in the running-sum passes
 constexpr int kP3Threads = 256;
+constexpr int kP3Warps = 8;
 
-template <int WY, int WX, int WZ>
+template <int WX, int WY, int WZ, int G>
 struct SsimGeom {
-  static constexpr int FX = kOX + WX - 1;
-  static constexpr int FY = kOY + WY - 1;
-  static constexpr int NCOL = FX * FY;
-  static constexpr int KC = (NCOL + kP3Threads - 1) / kP3Threads;
-  static constexpr size_t ring_bytes = (size_t)WZ * NCOL * sizeof(float2);
-  static constexpr size_t z_bytes = (size_t)NCOL * (4 * sizeof(double) + 2 * sizeof(float));
-  static constexpr size_t h_bytes = (size_t)kOY * FX * (4 * sizeof(double) + 2 * sizeof(float));
-  static constexpr size_t smem = ring_bytes + z_bytes + h_bytes;
+  static constexpr int TX = 32 - WX + 1;                 // origins per tile along x
+  static constexpr int TY = kP3Warps * G;                // origins per tile along y
+  static constexpr int FY = TY + WY - 1;                 // footprint rows
+  static constexpr int KC = (FY + kP3Warps - 1) / kP3Warps;   // z-walk rows per thread
+  static constexpr int ZSTRIDE = FY * 32;                // one component plane of the exchange
+  // exchange buffer: { 4 double comps, 2 float comps } x FY x 32, double-buffered
+  static constexpr size_t buf_bytes = (size_t)ZSTRIDE * (4 * sizeof(double) + 2 * sizeof(float));
+  static constexpr size_t smem = 2 * buf_bytes;
 };
 
-template <int WY, int WX, int WZ>
-__global__ void __launch_bounds__(kP3Threads)
-p3_kernel(Field3 f, SsimParams p,
-          double* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket,
-          double* __restrict__ dbg) {
-  using G = SsimGeom<WY, WX, WZ>;
-  constexpr int FX = G::FX, FY = G::FY, NCOL = G::NCOL, KC = G::KC;
+__device__ __forceinline__ double shd(double v, int d) { return __shfl_down_sync(0xffffffffu, v, d); }
+__device__ __forceinline__ float shf(float v, int d) { return __shfl_down_sync(0xffffffffu, v, d); }
+
+// Sum over lanes [l, l+W) of v (W compile-time): power-of-two doubling + binary decomposition.
+// Lanes whose window leaves the warp return garbage (their origins are outside the tile).
+template <int W>
+__device__ __forceinline__ double lane_window_sum(double v) {
+  double p[5];
+  p[0] = v;
+#pragma unroll
+  for (int k = 1; k < 5; k++)
+    if ((1 << k) <= W) p[k] = p[k - 1] + shd(p[k - 1], 1 << (k - 1));
+  double r = 0;
+  int off = 0;
+#pragma unroll
+  for (int k = 4; k >= 0; k--) {
+    if (W & (1 << k)) {
+      r += off == 0 ? p[k] : shd(p[k], off);
+      off += 1 << k;
+    }
+  }
+  return r;
+}
+
+// min / max over lanes [l, l+W): doubling to the largest power of two <= W, then one
+// overlapping combine (max and min are idempotent).
+template <int W, bool IS_MAX>
+__device__ __forceinline__ float lane_window_ext(float v) {
+  float q = v;
+  int k = 0;
+#pragma unroll
+  for (int j = 1; j < 5; j++)
+    if ((1 << j) <= W) {
+      const float o = shf(q, 1 << (j - 1));
+      q = IS_MAX ? fmaxf(q, o) : fminf(q, o);
+      k = j;
+    }
+  if ((1 << k) != W) {
+    const float o = shf(q, W - (1 << k));
+    q = IS_MAX ? fmaxf(q, o) : fminf(q, o);
+  }
+  return q;
+}
+
+template <int WX, int WY, int WZ, int G>
+__global__ void __launch_bounds__(kP3Threads, (SsimGeom<WX, WY, WZ, G>::KC * WZ <= 24) ? 2 : 1)
+p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __restrict__ res,
+          unsigned int* __restrict__ ticket, double* __restrict__ dbg) {
+  using Gm = SsimGeom<WX, WY, WZ, G>;
+  constexpr int TX = Gm::TX, FY = Gm::FY, KC = Gm::KC, ZS = Gm::ZSTRIDE;
   constexpr double invM = 1.0 / (double)(WX * WY * WZ);
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  float2* ring = reinterpret_cast<float2*>(smem_raw);                       // [WZ][NCOL]
-  double* Zd = reinterpret_cast<double*>(smem_raw + G::ring_bytes);         // [4][NCOL]
-  float* Zm = reinterpret_cast<float*>(Zd + 4 * NCOL);                      // [2][NCOL]
-  double* Hd = reinterpret_cast<double*>(smem_raw + G::ring_bytes + G::z_bytes);  // [4][kOY][FX]
-  float* Hm = reinterpret_cast<float*>(Hd + 4 * kOY * FX);                  // [2][kOY][FX]
 
-  const int tid = threadIdx.x;
-  const int64_t x0 = (int64_t)blockIdx.x * kOX, y0 = (int64_t)blockIdx.y * kOY;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int64_t x0 = (int64_t)blockIdx.x * TX, y0 = (int64_t)blockIdx.y * Gm::TY;
   const int64_t zb = f.zown0 + (int64_t)blockIdx.z * p.zchunk;
-  int64_t zo_end = zb + p.zchunk;                        // origin planes [zb, zo_end)
+  int64_t zo_end = zb + p.zchunk;                         // origin planes [zb, zo_end)
   if (zo_end > f.zown1) zo_end = f.zown1;
   if (zo_end > f.nz - WZ + 1) zo_end = f.nz - WZ + 1;
+  const int64_t zend = zo_end > zb ? zo_end + WZ - 1 : zb; // planes [zb, zend)
 
-  // anchor: tile-centre sample of the first plane (clamped into the field)
-  int64_t ky = y0 + FY / 2, kx = x0 + FX / 2;
+  int64_t ky = y0 + FY / 2, kx = x0 + 16;
   if (ky > f.ny - 1) ky = f.ny - 1;
   if (kx > f.nx - 1) kx = f.nx - 1;
-  const double K = (zb < zo_end) ? (double)f.xp(zb)[ky * f.nx + kx] : 0.0;
+  const double K = (zb < zend) ? (double)f.xp(zb)[ky * f.nx + kx] : 0.0;
   const double Lglob = (double)res->p1.xmax - (double)res->p1.xmin;
 
-  // per-thread footprint columns and their running z-sums
-  double rs[KC][4];
-  int64_t cofs[KC];
-  bool cin[KC];
+  // in-plane offsets (a plane has < 2^31 elements; the launcher checks) and validity bits
+  const int64_t gx = x0 + lane;
+  int off[KC];
+  unsigned vbits = 0;
 #pragma unroll
   for (int k = 0; k < KC; k++) {
-    const int c = tid + k * kP3Threads;
-    const int r = c / FX, cc = c % FX;
-    const int64_t gy = y0 + r, gx = x0 + cc;
-    cin[k] = c < NCOL && gy < f.ny && gx < f.nx;
-    cofs[k] = cin[k] ? gy * f.nx + gx : 0;
-#pragma unroll
-    for (int m = 0; m < 4; m++) rs[k][m] = 0;
+    const int r = warp + kP3Warps * k;
+    const int64_t gy = y0 + r;
+    const bool v = r < FY && gy < f.ny && gx < f.nx;
+    vbits |= (v ? 1u : 0u) << k;
+    off[k] = v ? (int)(gy * f.nx + gx) : 0;
   }
+  // Prefetch of plane z (x, y) and of the y sample of the plane leaving the z-window (z - WZ),
+  // which is re-read from L2 instead of being kept in the register ring.
+  auto load = [&](int64_t z, float2 (&dst)[KC], float (&yold)[KC]) {
+    if (z < zend) {
+      const float* X = f.xp(z);
+      const float* Y = f.yp(z);
+      const bool has_old = z - zb >= WZ;
+      const float* Yo = has_old ? f.yp(z - WZ) : Y;
+#pragma unroll
+      for (int k = 0; k < KC; k++) {
+        const bool v = (vbits >> k) & 1u;
+        dst[k] = v ? make_float2(__ldg(X + off[k]), __ldg(Y + off[k])) : make_float2(0.f, 0.f);
+        yold[k] = (v && has_old) ? __ldg(Yo + off[k]) : 0.f;
+      }
+    }
+  };
+
+  double sm[KC][4];
+  float ring[KC][WZ];                                    // x of the last WZ planes
+#pragma unroll
+  for (int k = 0; k < KC; k++) {
+#pragma unroll
+    for (int m = 0; m < 4; m++) sm[k][m] = 0;
+#pragma unroll
+    for (int s = 0; s < WZ; s++) ring[k][s] = 0.f;
+  }
+  float2 nxt[KC];                                        // prefetched next plane
+  float nyo[KC];                                         // ... and its leaving y sample
+  load(zb, nxt, nyo);
 
   double ssum = 0, scnt = 0;
-  const int64_t zplanes_end = (zo_end > zb) ? zo_end + WZ - 1 : zb;
-  for (int64_t zi = zb; zi < zplanes_end; zi++) {
-    const int step = (int)(zi - zb);
-    const int slot = step % WZ;
-    const float* Xz = f.xp(zi);
-    const float* Yz = f.yp(zi);
-    // ---- (a) z-walk ------------------------------------------------------------------------
+  const bool range_global = p.range_mode != 0;
+  for (int64_t zz = zb; zz < zend; zz += WZ) {
 #pragma unroll
-    for (int k = 0; k < KC; k++) {
-      const int c = tid + k * kP3Threads;
-      if (c < NCOL) {
-        float xv = 0.f, yv = 0.f;
-        if (cin[k]) { xv = Xz[cofs[k]]; yv = Yz[cofs[k]]; }
-        float2* rp = ring + (size_t)slot * NCOL + c;
+    for (int s = 0; s < WZ; s++) {
+      const int64_t zi = zz + s;
+      if (zi >= zend) break;                             // block-uniform
+      const int step = (int)(zi - zb);                   // == s (mod WZ)
+      float2 v[KC];
+      float yo[KC];
+#pragma unroll
+      for (int k = 0; k < KC; k++) { v[k] = nxt[k]; yo[k] = nyo[k]; }
+      load(zi + 1, nxt, nyo);
+      const int buf = step & 1;
+      double* Zd = reinterpret_cast<double*>(smem_raw + buf * Gm::buf_bytes);
+      float* Zm = reinterpret_cast<float*>(Zd + 4 * ZS);
+      // ---- (a) z-walk --------------------------------------------------------------------
+#pragma unroll
+      for (int k = 0; k < KC; k++) {
         {
-          const double xd = xv, yd = yv;
+          const double xd = v[k].x, yd = v[k].y;
           const double a = xd - K, b = yd - K, e = yd - xd;
-          rs[k][0] += a; rs[k][1] += e; rs[k][2] = fma(a, b, rs[k][2]); rs[k][3] = fma(e, e, rs[k][3]);
+          sm[k][0] += a; sm[k][1] += e; sm[k][2] = fma(a, b, sm[k][2]); sm[k][3] = fma(e, e, sm[k][3]);
         }
         if (step >= WZ) {
-          const float2 o = *rp;
-          const double xd = o.x, yd = o.y;
+          const double xd = ring[k][s], yd = yo[k];
           const double a = xd - K, b = yd - K, e = yd - xd;
-          rs[k][0] -= a; rs[k][1] -= e; rs[k][2] = fma(-a, b, rs[k][2]); rs[k][3] = fma(-e, e, rs[k][3]);
+          sm[k][0] -= a; sm[k][1] -= e; sm[k][2] = fma(-a, b, sm[k][2]); sm[k][3] = fma(-e, e, sm[k][3]);
         }
-        *rp = make_float2(xv, yv);
-        if (step >= WZ - 1) {
-          float mn = xv, mx = xv;
+        ring[k][s] = v[k].x;
+        const int r = warp + kP3Warps * k;
+        if (step >= WZ - 1 && r < FY) {
+          float mn = ring[k][0], mx = ring[k][0];
 #pragma unroll
-          for (int s = 0; s < WZ; s++) {
-            const float v = ring[(size_t)s * NCOL + c].x;
-            mn = fminf(mn, v);
-            mx = fmaxf(mx, v);
-          }
+          for (int t = 1; t < WZ; t++) { mn = fminf(mn, ring[k][t]); mx = fmaxf(mx, ring[k][t]); }
+          const int c = r * 32 + lane;
 #pragma unroll
-          for (int m = 0; m < 4; m++) Zd[m * NCOL + c] = rs[k][m];
+          for (int m = 0; m < 4; m++) Zd[m * ZS + c] = sm[k][m];
           Zm[c] = mn;
-          Zm[NCOL + c] = mx;
+          Zm[ZS + c] = mx;
+        }
+      }
+      if (step < WZ - 1) continue;                       // no complete z-window yet
+      __syncthreads();
+      const int64_t oz = zi - WZ + 1;
+      const bool zok = (oz % p.sz) == 0;
+      // ---- (b) y-pass over WY rows, (c) x-pass with shuffles, mix ------------------------
+      double h[4];
+#pragma unroll
+      for (int g = 0; g < G; g++) {
+        const int oy = warp * G + g;
+        if (g == 0) {
+#pragma unroll
+          for (int m = 0; m < 4; m++) {
+            double acc = 0;
+#pragma unroll
+            for (int i = 0; i < WY; i++) acc += Zd[m * ZS + (oy + i) * 32 + lane];
+            h[m] = acc;
+          }
+        } else {
+#pragma unroll
+          for (int m = 0; m < 4; m++)
+            h[m] += Zd[m * ZS + (oy + WY - 1) * 32 + lane] - Zd[m * ZS + (oy - 1) * 32 + lane];
+        }
+        float hmn = Zm[oy * 32 + lane], hmx = Zm[ZS + oy * 32 + lane];
+#pragma unroll
+        for (int i = 1; i < WY; i++) {
+          hmn = fminf(hmn, Zm[(oy + i) * 32 + lane]);
+          hmx = fmaxf(hmx, Zm[ZS + (oy + i) * 32 + lane]);
+        }
+        const double S0 = lane_window_sum<WX>(h[0]);
+        const double S1 = lane_window_sum<WX>(h[1]);
+        const double S2 = lane_window_sum<WX>(h[2]);
+        const double S3 = lane_window_sum<WX>(h[3]);
+        const float mn = lane_window_ext<WX, false>(hmn);
+        const float mx = lane_window_ext<WX, true>(hmx);
+        const int64_t gy = y0 + oy;
+        const int64_t gxo = x0 + lane;
+        if (lane < TX && zok && gy <= f.ny - WY && (gy % p.sy) == 0 && gxo <= f.nx - WX && (gxo % p.sx) == 0) {
+          const double mua = S0 * invM, mue = S1 * invM;
+          const double mux = K + mua, muy = mux + mue;
+          const double sxy = S2 * invM - mua * (mua + mue);
+          const double see = S3 * invM - mue * mue;
+          double L = range_global ? Lglob : (double)mx - (double)mn;
+          if (L == 0) L = 1.0;
+          const double C1 = (0.01 * L) * (0.01 * L), C2 = (0.03 * L) * (0.03 * L);
+          const double A = 2.0 * mux * muy + C1, B = 2.0 * sxy + C2;
+          const double ssim = (A * B) / ((A + mue * mue) * (B + see));
+          ssum += ssim;
+          scnt += 1.0;
+          if (dbg) dbg[((oz / p.sz) * p.nwy + gy / p.sy) * p.nwx + gxo / p.sx] = ssim;
         }
       }
     }
-    if (step < WZ - 1) continue;           // no complete z-window yet (block-uniform)
-    const int64_t oz = zi - WZ + 1;        // origin plane of the windows completed now
-    __syncthreads();
-    // ---- (b) y-pass: columns of Z, running sums over WY rows --------------------------------
-    for (int item = tid; item < FX * (kOY / kSeg); item += kP3Threads) {
-      const int cx = item % FX, oy0 = (item / FX) * kSeg;
-#pragma unroll
-      for (int m = 0; m < 4; m++) {
-        double v[kSeg + WY - 1];
-#pragma unroll
-        for (int i = 0; i < kSeg + WY - 1; i++) v[i] = Zd[m * NCOL + (oy0 + i) * FX + cx];
-        double s = 0;
-#pragma unroll
-        for (int i = 0; i < WY; i++) s += v[i];
-        Hd[(m * kOY + oy0) * FX + cx] = s;
-#pragma unroll
-        for (int j = 1; j < kSeg; j++) {
-          s += v[j + WY - 1] - v[j - 1];
-          Hd[(m * kOY + oy0 + j) * FX + cx] = s;
-        }
-      }
-      float vn[kSeg + WY - 1], vx[kSeg + WY - 1];
-#pragma unroll
-      for (int i = 0; i < kSeg + WY - 1; i++) {
-        vn[i] = Zm[(oy0 + i) * FX + cx];
-        vx[i] = Zm[NCOL + (oy0 + i) * FX + cx];
-      }
-#pragma unroll
-      for (int j = 0; j < kSeg; j++) {
-        float mn = vn[j], mx = vx[j];
-#pragma unroll
-        for (int i = 1; i < WY; i++) { mn = fminf(mn, vn[j + i]); mx = fmaxf(mx, vx[j + i]); }
-        Hm[(oy0 + j) * FX + cx] = mn;
-        Hm[(kOY + oy0 + j) * FX + cx] = mx;
-      }
-    }
-    __syncthreads();
-    // ---- (c) x-pass + mix -------------------------------------------------------------------
-    const bool zok = (oz % p.sz) == 0;
-    for (int item = tid; item < kOY * (kOX / kSeg); item += kP3Threads) {
-      const int oy = item / (kOX / kSeg), ox0 = (item % (kOX / kSeg)) * kSeg;
-      double S[4][kSeg];
-#pragma unroll
-      for (int m = 0; m < 4; m++) {
-        double v[kSeg + WX - 1];
-#pragma unroll
-        for (int i = 0; i < kSeg + WX - 1; i++) v[i] = Hd[(m * kOY + oy) * FX + ox0 + i];
-        double s = 0;
-#pragma unroll
-        for (int i = 0; i < WX; i++) s += v[i];
-        S[m][0] = s;
-#pragma unroll
-        for (int j = 1; j < kSeg; j++) { s += v[j + WX - 1] - v[j - 1]; S[m][j] = s; }
-      }
-      float vn[kSeg + WX - 1], vx[kSeg + WX - 1];
-#pragma unroll
-      for (int i = 0; i < kSeg + WX - 1; i++) {
-        vn[i] = Hm[oy * FX + ox0 + i];
-        vx[i] = Hm[(kOY + oy) * FX + ox0 + i];
-      }
-      const int64_t gy = y0 + oy;
-      const bool yok = gy <= f.ny - WY && (gy % p.sy) == 0;
-#pragma unroll
-      for (int j = 0; j < kSeg; j++) {
-        const int64_t gx = x0 + ox0 + j;
-        if (!(zok && yok && gx <= f.nx - WX && (gx % p.sx) == 0)) continue;
-        float mn = vn[j], mx = vx[j];
-#pragma unroll
-        for (int i = 1; i < WX; i++) { mn = fminf(mn, vn[j + i]); mx = fmaxf(mx, vx[j + i]); }
-        const double mua = S[0][j] * invM, mue = S[1][j] * invM;
-        const double mux = K + mua, muy = mux + mue;
-        const double sxy = S[2][j] * invM - mua * (mua + mue);
-        const double see = S[3][j] * invM - mue * mue;
-        double L = p.range_mode ? Lglob : (double)mx - (double)mn;
-        if (L == 0) L = 1.0;
-        const double C1 = (0.01 * L) * (0.01 * L), C2 = (0.03 * L) * (0.03 * L);
-        const double A = 2.0 * mux * muy + C1, B = 2.0 * sxy + C2;
-        const double ssim = (A * B) / ((A + mue * mue) * (B + see));
-        ssum += ssim;
-        scnt += 1.0;
-        if (dbg) dbg[((oz / p.sz) * p.nwy + gy / p.sy) * p.nwx + gx / p.sx] = ssim;
-      }
-    }
-    // the next (a) only writes the ring / Z, which (c) does not read; (b) of the next plane is
-    // behind the __syncthreads after that (a), so H is not overwritten while (c) reads it.
   }
 
   double rec[kSsimSlots] = {ssum, scnt, 0.0};
   const unsigned bid = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
   struct Sum { __device__ int operator()(int) const { return OP_SUM; } };
+  __syncthreads();
   block_reduce_slots<kSsimSlots>(rec, Sum{}, parts + (size_t)bid * kSsimSlots);
   if (!last_block_arrive(ticket)) return;
   finish_slots<kSsimSlots>(parts, gridDim.x * gridDim.y * gridDim.z, Sum{}, res->ssim);
@@ -225,32 +261,35 @@ p3_kernel(Field3 f, SsimParams p,
 
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
-template <int WY, int WX, int WZ>
+template <int WX, int WY, int WZ, int G>
 static cudaError_t launch_t(const Field3& f, const SsimParams& p, double* parts,
                             DevResults* res, unsigned int* ticket, double* dbg, cudaStream_t st,
                             int64_t* nblocks_out) {
-  using G = SsimGeom<WY, WX, WZ>;
+  using Gm = SsimGeom<WX, WY, WZ, G>;
   int64_t zhi = f.zown1 < f.nz - WZ + 1 ? f.zown1 : f.nz - WZ + 1;
   const int64_t noz = zhi > f.zown0 ? zhi - f.zown0 : 1;
-  dim3 grid((unsigned)cdiv(f.nx - WX + 1, kOX), (unsigned)cdiv(f.ny - WY + 1, kOY), (unsigned)cdiv(noz, p.zchunk));
+  dim3 grid((unsigned)cdiv(f.nx - WX + 1, Gm::TX), (unsigned)cdiv(f.ny - WY + 1, Gm::TY),
+            (unsigned)cdiv(noz, p.zchunk));
   if (nblocks_out) { *nblocks_out = (int64_t)grid.x * grid.y * grid.z; return cudaSuccess; }
-  cudaError_t e = cudaFuncSetAttribute(p3_kernel<WY, WX, WZ>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)G::smem);
+  if (f.ny * f.nx >= (int64_t)1 << 31) return cudaErrorInvalidValue;   // 32-bit in-plane offsets
+  cudaError_t e = cudaFuncSetAttribute(p3_kernel<WX, WY, WZ, G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Gm::smem);
   if (e != cudaSuccess) return e;
-  p3_kernel<WY, WX, WZ><<<grid, kP3Threads, G::smem, st>>>(f, p, parts, res, ticket, dbg);
+  p3_kernel<WX, WY, WZ, G><<<grid, kP3Threads, Gm::smem, st>>>(f, p, parts, res, ticket, dbg);
   return cudaGetLastError();
 }
 
-// Dispatch on the (compile-time) window: cubic (3-D), square (2-D, WZ = 1) or 1-D (WY = WZ = 1).
+// kind 3: cubic window (3-D); 2: square window, z inactive (2-D); 1: x only (1-D).
 template <int W>
 static cudaError_t dispatch_w(int kind, const Field3& f, const SsimParams& p, double* parts,
                               DevResults* res, unsigned int* ticket, double* dbg, cudaStream_t st, int64_t* nb) {
-  if (kind == 3) return launch_t<W, W, W>(f, p, parts, res, ticket, dbg, st, nb);
-  if (kind == 2) return launch_t<W, W, 1>(f, p, parts, res, ticket, dbg, st, nb);
-  return launch_t<1, W, 1>(f, p, parts, res, ticket, dbg, st, nb);
+  constexpr int G = W <= 8 ? 2 : 1;                     // keep the z-walk state in registers
+  if (kind == 3) return launch_t<W, W, W, G>(f, p, parts, res, ticket, dbg, st, nb);
+  if (kind == 2) return launch_t<W, W, 1, 2>(f, p, parts, res, ticket, dbg, st, nb);
+  return launch_t<W, 1, 1, 1>(f, p, parts, res, ticket, dbg, st, nb);
 }
 
-// kind: 3 = (W,W,W) cubic window, 2 = (W,W) with z inactive, 1 = x only.  Returns
-// cudaErrorInvalidValue for unsupported W.  If nblocks_out != NULL only the grid size is returned.
+// Returns cudaErrorInvalidValue for unsupported W.  If nblocks_out != NULL only the grid size
+// is computed (no launch).
 cudaError_t launch_ssim(int kind, int W, const Field3& f, const SsimParams& p,
                         double* parts, DevResults* res, unsigned int* ticket, double* dbg,
                         cudaStream_t st, int64_t* nblocks_out) {
