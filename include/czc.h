@@ -79,6 +79,10 @@ typedef struct czc_config {
   double* debug_wssim;           /* optional DEVICE buffer of n_windows doubles: local SSIM of   */
                                  /* every window in C order of the window-origin grid (Alg. 3    */
                                  /* L310 "wssim"); NULL = not written (not on the timed path)    */
+  int loopback_slabs;            /* verification of slab mode on ONE GPU: > 1 splits dims[0]    */
+                                 /* into that many slabs and runs the exact multi-GPU path (halo */
+                                 /* buffers, owned ranges, rank-ordered combine) with device     */
+                                 /* copies in place of NCCL; 0/1 = off.  Requires nranks <= 1.   */
 } czc_config;
 
 /* Field shape.  Single GPU: z0 = 0 and nz_local = dims[0] (or 0 meaning dims[0]).
@@ -147,6 +151,13 @@ czc_status czc_assess(czc_ctx* ctx, const void* orig, const void* recon, const c
 czc_status czc_assess_host(czc_ctx* ctx, const void* orig, const void* recon, const czc_shape* shape,
                            czc_dtype dtype, uint64_t metric_mask, czc_result* out);
 
+/* Rank-ordered combine of per-slab partial records and the metric finish — the host step of slab
+ * mode, exported so it can be verified without a GPU.  `records` holds `nrecords` consecutive
+ * records of czc_sizeof(3) bytes each (slab order = rank order), `global_shape` the whole field
+ * (z0 = 0, nz_local = 0), `cfg` the SSIM / AC settings used to produce them.  Host memory only. */
+czc_status czc_combine(const void* records, int nrecords, const czc_shape* global_shape,
+                       const czc_config* cfg, uint64_t metric_mask, czc_result* out);
+
 /* Release the context, its device scratch, its stream (if owned) and its NCCL communicator. */
 void czc_free(czc_ctx* ctx);
 
@@ -160,8 +171,8 @@ const char* czc_last_error(const czc_ctx* ctx);
 int czc_abi_version(void);
 int czc_has_nccl(void);
 
-/* sizeof(czc_config) (what = 0), sizeof(czc_shape) (1), sizeof(czc_result) (2), bytes copied
- * device->host per czc_assess call (3); 0 otherwise.  Lets bindings verify their struct mirrors
+/* sizeof(czc_config) (what = 0), sizeof(czc_shape) (1), sizeof(czc_result) (2), size of one
+ * partial record = bytes copied device->host per single-GPU czc_assess call (3); 0 otherwise.  Lets bindings verify their struct mirrors
  * against the compiled library. */
 uint64_t czc_sizeof(int what);
 

@@ -41,7 +41,7 @@ class Config(ctypes.Structure):
                 ("ssim_window", ctypes.c_int * 3), ("ssim_step", ctypes.c_int * 3),
                 ("ssim_range_mode", ctypes.c_int), ("ac_max_lag", ctypes.c_int), ("timing", ctypes.c_int),
                 ("rank", ctypes.c_int), ("nranks", ctypes.c_int), ("nccl_uid", ctypes.c_void_p),
-                ("debug_wssim", ctypes.c_void_p)]
+                ("debug_wssim", ctypes.c_void_p), ("loopback_slabs", ctypes.c_int)]
 
 
 class Shape(ctypes.Structure):
@@ -92,6 +92,9 @@ def _load():
     lib.czc_has_nccl.restype = ctypes.c_int
     lib.czc_sizeof.argtypes = [ctypes.c_int]
     lib.czc_sizeof.restype = ctypes.c_uint64
+    lib.czc_combine.argtypes = [P, ctypes.c_int, ctypes.POINTER(Shape), ctypes.POINTER(Config), ctypes.c_uint64,
+                                ctypes.POINTER(Result)]
+    lib.czc_combine.restype = ctypes.c_int
     for what, st in ((0, Config), (1, Shape), (2, Result)):
         if lib.czc_sizeof(what) != ctypes.sizeof(st):
             raise ImportError(f"ABI mismatch: {st.__name__} is {ctypes.sizeof(st)} B here, "
@@ -115,8 +118,8 @@ def __getattr__(name):          # PEP 562: `czc.lib` loads the library on first 
     raise AttributeError(name)
 
 
-EXPORTED = ("czc_init", "czc_assess", "czc_assess_host", "czc_free", "czc_strerror", "czc_last_error",
-            "czc_abi_version", "czc_has_nccl", "czc_sizeof")
+EXPORTED = ("czc_init", "czc_assess", "czc_assess_host", "czc_combine", "czc_free", "czc_strerror",
+            "czc_last_error", "czc_abi_version", "czc_has_nccl", "czc_sizeof")
 
 
 def _per_axis(v, ndim) -> Sequence[int]:
@@ -128,7 +131,8 @@ def _per_axis(v, ndim) -> Sequence[int]:
 
 def make_config(ndim: int = 3, device: int = -1, stream: Optional[int] = None, ssim_window=8, ssim_step=1,
                 ssim_range_mode: int = 0, ac_max_lag: int = 10, timing: bool = False, rank: int = 0,
-                nranks: int = 1, nccl_uid: Optional[bytes] = None, debug_wssim: Optional[int] = None) -> Config:
+                nranks: int = 1, nccl_uid: Optional[bytes] = None, debug_wssim: Optional[int] = None,
+                loopback_slabs: int = 0) -> Config:
     c = Config()
     c.device = device
     c.stream = stream
@@ -145,6 +149,7 @@ def make_config(ndim: int = 3, device: int = -1, stream: Optional[int] = None, s
         c._uid = ctypes.create_string_buffer(bytes(nccl_uid), 128)
         c.nccl_uid = ctypes.cast(c._uid, ctypes.c_void_p)
     c.debug_wssim = debug_wssim
+    c.loopback_slabs = loopback_slabs
     return c
 
 
@@ -200,6 +205,17 @@ def czc_assess(ctx: int, orig_ptr: int, recon_ptr: int, shape: Shape, mask: int 
     rc = fn(ctx, orig_ptr, recon_ptr, ctypes.byref(shape), 0, mask, ctypes.byref(r))
     if rc:
         raise CzcError(rc, lib.czc_last_error(ctx).decode(errors="replace"))
+    return result_dict(r)
+
+
+def czc_combine(records: bytes, nrecords: int, dims: Sequence[int], cfg: Config, mask: int = M_ALL) -> Dict:
+    """Host-only rank-ordered combine + finish of per-slab records (czc_sizeof(3) bytes each)."""
+    lib = get_lib()
+    r = Result()
+    buf = ctypes.create_string_buffer(bytes(records), len(records))
+    rc = lib.czc_combine(buf, nrecords, ctypes.byref(make_shape(dims)), ctypes.byref(cfg), mask, ctypes.byref(r))
+    if rc:
+        raise CzcError(rc, "czc_combine")
     return result_dict(r)
 
 

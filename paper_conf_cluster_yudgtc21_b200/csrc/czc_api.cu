@@ -1,8 +1,10 @@
 // czc_api.cu — the C ABI (include/czc.h): context, validation, the "GPU module coordinator"
-// (L96: identify the requested metric categories, launch the matching fused kernels), one
-// device->host copy of the partial results, and the scalar finish math (derived metrics).
+// (L96: identify the requested metric categories, launch the matching fused kernels), the slab
+// decomposition for several GPUs (L423 future work), one device->host copy of
+// the partial records, and the scalar finish math (derived metrics).
 #include <cuda_runtime.h>
 #include <math.h>
+#include <stddef.h>
 #include <stdio.h>
 #include <stdlib.h>
 #include <string.h>
@@ -10,10 +12,11 @@
 #include <algorithm>
 #include <new>
 #include <string>
+#include <utility>
 #include <vector>
 
-#include "czc_internal.cuh"
 #include "czc_comm.h"
+#include "czc_internal.cuh"
 
 namespace czc {
 cudaError_t launch_p1(const float* x, const float* y, int64_t n, int grid_cap, P1State* parts,
@@ -41,21 +44,22 @@ struct czc_ctx {
   int sm_count = 0;
   int p1_grid_cap = 0;
   DevResults* dres = nullptr;      // device
-  DevResults* hres = nullptr;      // pinned host
+  Record* hrec = nullptr;          // pinned host, max_records records
   unsigned int* tickets = nullptr; // device
-  void* parts = nullptr;
+  void* parts = nullptr;           // per-block partial records
   size_t parts_cap = 0;
   float* din[2] = {nullptr, nullptr};   // staging for czc_assess_host
   size_t din_cap = 0;
   cudaEvent_t ev[5] = {};
   std::string last_error;
+  // slab mode (NCCL ranks or loopback)
   CommState* comm = nullptr;
-  // slab mode
   void* dgather_in = nullptr;      // device, 64 B
-  void* dgather = nullptr;         // device, nranks * sizeof(DevResults)
-  void* hgather = nullptr;         // pinned host, nranks * sizeof(DevResults)
+  void* dgather = nullptr;         // device, max_records * sizeof(Record)
+  void* dstates = nullptr;         // device, max_records * sizeof(P1State)
   float* halo = nullptr;           // device halo planes (x lo, y lo, x hi, y hi)
   size_t halo_cap = 0;
+  int max_records = 1;
 };
 
 static const char* kStatusStr[] = {"ok", "invalid argument", "invalid shape", "unsupported dtype",
@@ -71,7 +75,7 @@ extern "C" int czc_abi_version(void) { return CZC_ABI_VERSION; }
 extern "C" int czc_has_nccl(void) { return comm_available(); }
 extern "C" uint64_t czc_sizeof(int what) {
   return what == 0 ? sizeof(czc_config) : what == 1 ? sizeof(czc_shape) : what == 2 ? sizeof(czc_result)
-       : what == 3 ? sizeof(DevResults) : 0;
+       : what == 3 ? sizeof(Record) : 0;
 }
 
 static czc_status cuda_fail(czc_ctx* ctx, cudaError_t e, const char* where) {
@@ -79,11 +83,21 @@ static czc_status cuda_fail(czc_ctx* ctx, cudaError_t e, const char* where) {
   (void)cudaGetLastError();
   return e == cudaErrorMemoryAllocation ? CZC_ERR_NOMEM : CZC_ERR_CUDA;
 }
-#define CZC_CUDA(ctx, call)                                   \
-  do {                                                        \
-    cudaError_t _e = (call);                                  \
+#define CZC_CUDA(ctx, call)                                    \
+  do {                                                         \
+    cudaError_t _e = (call);                                   \
     if (_e != cudaSuccess) return cuda_fail((ctx), _e, #call); \
   } while (0)
+
+static czc_status validate_config(const czc_config& c) {
+  if (c.ac_max_lag < 0 || c.ac_max_lag > CZC_MAX_LAG) return CZC_ERR_INVALID;
+  if (c.ssim_range_mode < 0 || c.ssim_range_mode > 1) return CZC_ERR_INVALID;
+  for (int i = 0; i < 3; i++)
+    if (c.ssim_window[i] < 0 || c.ssim_step[i] < 0) return CZC_ERR_INVALID;
+  if (c.nranks > 1 && (c.rank < 0 || c.rank >= c.nranks || !c.nccl_uid)) return CZC_ERR_INVALID;
+  if (c.loopback_slabs < 0 || (c.loopback_slabs > 1 && c.nranks > 1)) return CZC_ERR_INVALID;
+  return CZC_OK;
+}
 
 extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
   if (!out) return CZC_ERR_INVALID;
@@ -92,17 +106,14 @@ extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
   memset(&c, 0, sizeof(c));
   if (cfg) c = *cfg;
   else c.device = -1;
-  if (c.ac_max_lag < 0 || c.ac_max_lag > CZC_MAX_LAG) return CZC_ERR_INVALID;
-  if (c.ssim_range_mode < 0 || c.ssim_range_mode > 1) return CZC_ERR_INVALID;
-  for (int i = 0; i < 3; i++)
-    if (c.ssim_window[i] < 0 || c.ssim_step[i] < 0) return CZC_ERR_INVALID;
-  if (c.nranks > 1 && (c.rank < 0 || c.rank >= c.nranks || !c.nccl_uid)) return CZC_ERR_INVALID;
+  czc_status st = validate_config(c);
+  if (st != CZC_OK) return st;
   if (c.nranks > 1 && !comm_available()) return CZC_ERR_UNSUPPORTED;
 
   czc_ctx* ctx = new (std::nothrow) czc_ctx();
   if (!ctx) return CZC_ERR_NOMEM;
   ctx->cfg = c;
-  czc_status st = CZC_OK;
+  ctx->max_records = std::max(1, std::max(c.nranks, c.loopback_slabs));
   do {
     int dev = c.device;
     if (dev < 0) {
@@ -120,18 +131,20 @@ extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
       if (e != cudaSuccess) { st = cuda_fail(ctx, e, "cudaStreamCreate"); break; }
       ctx->own_stream = true;
     }
+    const size_t rb = (size_t)ctx->max_records * sizeof(Record);
     if ((e = cudaMalloc(&ctx->dres, sizeof(DevResults))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(res)"); break; }
-    if ((e = cudaMallocHost(&ctx->hres, sizeof(DevResults))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMallocHost"); break; }
+    if ((e = cudaMallocHost(&ctx->hrec, rb)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMallocHost"); break; }
     if ((e = cudaMalloc(&ctx->tickets, TICKET_N * sizeof(unsigned int))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(tickets)"); break; }
     if ((e = cudaMemset(ctx->tickets, 0, TICKET_N * sizeof(unsigned int))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMemset"); break; }
-    for (int i = 0; i < 5; i++)
-      if ((e = cudaEventCreate(&ctx->ev[i])) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaEventCreate"); break; }
+    for (int i = 0; i < 5 && st == CZC_OK; i++)
+      if ((e = cudaEventCreate(&ctx->ev[i])) != cudaSuccess) st = cuda_fail(ctx, e, "cudaEventCreate");
     if (st != CZC_OK) break;
-    if (c.nranks > 1) {
-      const size_t gb = (size_t)c.nranks * sizeof(DevResults);
+    if (ctx->max_records > 1) {
       if ((e = cudaMalloc(&ctx->dgather_in, 64)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(gather)"); break; }
-      if ((e = cudaMalloc(&ctx->dgather, gb)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(gather)"); break; }
-      if ((e = cudaMallocHost(&ctx->hgather, gb)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMallocHost(gather)"); break; }
+      if ((e = cudaMalloc(&ctx->dgather, rb)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(gather)"); break; }
+      if ((e = cudaMalloc(&ctx->dstates, (size_t)ctx->max_records * sizeof(P1State))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(states)"); break; }
+    }
+    if (c.nranks > 1) {
       ctx->comm = comm_create(c.nccl_uid, c.rank, c.nranks, &ctx->last_error);
       if (!ctx->comm) { st = CZC_ERR_COMM; break; }
     }
@@ -150,14 +163,14 @@ extern "C" void czc_free(czc_ctx* ctx) {
   if (ctx->stream) cudaStreamSynchronize(ctx->stream);
   if (ctx->comm) comm_destroy(ctx->comm);
   cudaFree(ctx->dres);
-  cudaFreeHost(ctx->hres);
+  cudaFreeHost(ctx->hrec);
   cudaFree(ctx->tickets);
   cudaFree(ctx->parts);
   cudaFree(ctx->din[0]);
   cudaFree(ctx->din[1]);
   cudaFree(ctx->dgather_in);
   cudaFree(ctx->dgather);
-  cudaFreeHost(ctx->hgather);
+  cudaFree(ctx->dstates);
   cudaFree(ctx->halo);
   for (int i = 0; i < 5; i++)
     if (ctx->ev[i]) cudaEventDestroy(ctx->ev[i]);
@@ -166,13 +179,11 @@ extern "C" void czc_free(czc_ctx* ctx) {
 }
 
 // ------------------------------------------------------------------------------------------------
-// Planning
+// Planning (global shape; host only)
 // ------------------------------------------------------------------------------------------------
 namespace {
 struct Plan {
-  int64_t n = 0;                  // local elements
-  int64_t d3[3] = {1, 1, 1};      // squeezed, right-aligned (nz, ny, nx) of the LOCAL field
-  int64_t g3[3] = {1, 1, 1};      // same for the GLOBAL field
+  int64_t g3[3] = {1, 1, 1};      // GLOBAL field, extent-1 axes squeezed, right-aligned (nz, ny, nx)
   int D = 0;                      // active axes
   int W = 8, step[3] = {1, 1, 1}; // SSIM (per 3-D axis)
   int win3[3] = {1, 1, 1};
@@ -182,36 +193,25 @@ struct Plan {
   int32_t win_in[3] = {0, 0, 0}, step_in[3] = {0, 0, 0};  // reported per input axis
 };
 
-czc_status make_plan(const czc_ctx* ctx, const czc_shape* sh, uint64_t mask, Plan& P, std::string& why) {
-  const czc_config& c = ctx->cfg;
-  if (sh->ndim < 1 || sh->ndim > 3) { why = "ndim must be 1..3"; return CZC_ERR_SHAPE; }
-  int64_t gd[3], ld[3];
-  for (int i = 0; i < sh->ndim; i++) {
-    if (sh->dims[i] < 1) { why = "dims must be >= 1"; return CZC_ERR_SHAPE; }
-    gd[i] = ld[i] = sh->dims[i];
+czc_status make_plan(const czc_config& c, int ndim, const int64_t* dims, uint64_t mask, Plan& P, std::string& why) {
+  if (ndim < 1 || ndim > 3) { why = "ndim must be 1..3"; return CZC_ERR_SHAPE; }
+  int64_t gd[3];
+  for (int i = 0; i < ndim; i++) {
+    if (dims[i] < 1) { why = "dims must be >= 1"; return CZC_ERR_SHAPE; }
+    gd[i] = dims[i];
   }
-  const int64_t nzl = sh->nz_local > 0 ? sh->nz_local : sh->dims[0];
-  if (sh->z0 < 0 || sh->z0 + nzl > sh->dims[0]) { why = "slab [z0, z0+nz_local) outside dims[0]"; return CZC_ERR_SHAPE; }
-  ld[0] = nzl;
-  if (ctx->cfg.nranks <= 1 && (sh->z0 != 0 || nzl != sh->dims[0])) { why = "slab shape needs nranks > 1"; return CZC_ERR_SHAPE; }
-  // squeeze inactive (extent-1) axes of the GLOBAL shape; C-order layout is unchanged by it
+  // squeeze inactive (extent-1) axes; the C-order layout is unchanged by it
   int act_in[3], na = 0;
-  for (int i = 0; i < sh->ndim; i++)
+  for (int i = 0; i < ndim; i++)
     if (gd[i] > 1) act_in[na++] = i;
   P.D = na;
-  for (int k = 0; k < na; k++) {
-    P.g3[3 - na + k] = gd[act_in[k]];
-    P.d3[3 - na + k] = ld[act_in[k]];
-  }
-  if (ctx->cfg.nranks > 1 && (na < 1 || act_in[0] != 0)) { why = "slab mode needs dims[0] > 1"; return CZC_ERR_SHAPE; }
-  P.n = P.d3[0] * P.d3[1] * P.d3[2];
+  for (int k = 0; k < na; k++) P.g3[3 - na + k] = gd[act_in[k]];
   P.T = c.ac_max_lag ? c.ac_max_lag : 10;
   P.run_ssim = (mask & CZC_M_SSIM) != 0;
   P.run_deriv = (mask & CZC_M_DERIV) != 0;
   P.run_ac = (mask & CZC_M_AUTOCORR) != 0;
   P.run_p1 = (mask & (CZC_M_P1 | CZC_M_AUTOCORR)) != 0 || (P.run_ssim && c.ssim_range_mode == 1);
-  // SSIM window per input axis -> per active axis
-  for (int i = 0; i < sh->ndim; i++) {
+  for (int i = 0; i < ndim; i++) {
     const int w = c.ssim_window[i] ? c.ssim_window[i] : 8;
     const int s = c.ssim_step[i] ? c.ssim_step[i] : 1;
     P.win_in[i] = gd[i] > 1 ? w : 1;
@@ -265,8 +265,25 @@ void finish_p1(const P1State& f, czc_result* o) {
   o->err_var = f.m2e / n;
 }
 
-// Derived metrics from the combined records (global shape in P.g3).
-void finish_all(const Plan& P, const DevResults& R, uint64_t mask, czc_result* out) {
+// Rank-ordered combine of records (P1 states by the stable pairwise merge, sums added, extrema
+// min/max), then the derived metrics from the global shape in P.g3.  Host code; every rank runs
+// it on the same bytes, so all ranks return identical results.
+void combine_and_finish(const Plan& P, const Record* recs, int nrec, uint64_t mask, czc_result* out) {
+  Record R = recs[0];
+  P1State g;
+  p1_empty(g);
+  for (int r = 0; r < nrec; r++) p1_merge(g, recs[r].p1);
+  R.p1 = g;
+  for (int r = 1; r < nrec; r++) {
+    for (int k = 0; k < kDerivSlots; k++) {
+      const int op = deriv_op(k);
+      R.deriv[k] = op == OP_SUM ? R.deriv[k] + recs[r].deriv[k]
+                 : op == OP_MIN ? std::min(R.deriv[k], recs[r].deriv[k]) : std::max(R.deriv[k], recs[r].deriv[k]);
+    }
+    for (int w = 0; w < kAcWalks; w++)
+      for (int k = 0; k < kAcSlots; k++) R.ac[w][k] += recs[r].ac[w][k];
+    for (int k = 0; k < kSsimSlots; k++) R.ssim[k] += recs[r].ssim[k];
+  }
   uint64_t done = 0;
   if (P.run_p1 && (mask & CZC_M_P1)) { finish_p1(R.p1, out); done |= CZC_M_P1; }
   if (P.run_deriv) {
@@ -321,6 +338,26 @@ void finish_all(const Plan& P, const DevResults& R, uint64_t mask, czc_result* o
 }
 }  // namespace
 
+extern "C" czc_status czc_combine(const void* records, int nrecords, const czc_shape* global_shape,
+                                  const czc_config* cfg, uint64_t metric_mask, czc_result* out) {
+  if (!out) return CZC_ERR_INVALID;
+  memset(out, 0, sizeof(*out));
+  if (!records || nrecords < 1 || !global_shape || !cfg) return CZC_ERR_INVALID;
+  czc_status st = validate_config(*cfg);
+  if (st != CZC_OK) return st;
+  Plan P;
+  std::string why;
+  st = make_plan(*cfg, global_shape->ndim, global_shape->dims, metric_mask, P, why);
+  if (st != CZC_OK) return st;
+  std::vector<Record> recs(nrecords);
+  memcpy(recs.data(), records, (size_t)nrecords * sizeof(Record));
+  combine_and_finish(P, recs.data(), nrecords, metric_mask, out);
+  return CZC_OK;
+}
+
+// ------------------------------------------------------------------------------------------------
+// Device execution
+// ------------------------------------------------------------------------------------------------
 static czc_status ensure_buf(czc_ctx* ctx, void** p, size_t* cap, size_t bytes) {
   if (bytes <= *cap) return CZC_OK;
   cudaFree(*p);
@@ -331,163 +368,268 @@ static czc_status ensure_buf(czc_ctx* ctx, void** p, size_t* cap, size_t bytes) 
   return CZC_OK;
 }
 
-// Slab-mode bookkeeping (nranks > 1): the per-rank slab table, halo buffers, gather buffers.
-struct SlabInfo {
-  int64_t z0, nzl;
-};
+namespace {
+constexpr int kZchunkDeriv = 128, kZchunkSsim = 32;
 
-static czc_status comm_err(czc_ctx* ctx) { return CZC_ERR_COMM; }
-
-static czc_status assess_core(czc_ctx* ctx, const float* x, const float* y, const czc_shape* shape,
-                              uint64_t mask, czc_result* out) {
-  Plan P;
-  czc_status st = make_plan(ctx, shape, mask, P, ctx->last_error);
-  if (st != CZC_OK) return st;
-  const cudaStream_t s = ctx->stream;
-  const bool timing = ctx->cfg.timing != 0;
-  const int zchunk_d = 32, zchunk_ac = 32, zchunk_ss = 32;
-  const bool slab = ctx->comm != nullptr;
-  const int nranks = slab ? comm_size(ctx->comm) : 1, rank = slab ? comm_rank(ctx->comm) : 0;
-  const int64_t plane = P.g3[1] * P.g3[2];
-
-  // ---- field view: owned planes + halo segments -------------------------------------------------
-  Field3 F{};
-  F.nz = P.g3[0]; F.ny = P.g3[1]; F.nx = P.g3[2];
-  const int64_t z0 = slab ? shape->z0 : 0, nzl = P.d3[0];
-  F.zown0 = z0; F.zown1 = z0 + nzl;
-  int64_t hlo = 0, hhi = 0;
-  if (slab) {
-    // slab table (every rank validates every slab identically -> collective decision)
-    int64_t mine[2] = {z0, nzl};
-    CZC_CUDA(ctx, cudaMemcpyAsync(ctx->dgather_in, mine, sizeof(mine), cudaMemcpyHostToDevice, s));
-    if (!comm_allgather(ctx->comm, ctx->dgather_in, ctx->dgather, sizeof(mine), s, &ctx->last_error)) return comm_err(ctx);
-    std::vector<SlabInfo> tab(nranks);
-    CZC_CUDA(ctx, cudaMemcpyAsync(tab.data(), ctx->dgather, nranks * sizeof(mine), cudaMemcpyDeviceToHost, s));
-    CZC_CUDA(ctx, cudaStreamSynchronize(s));
-    int64_t H = 0;
-    if (P.run_deriv) H = std::max<int64_t>(H, 1);
-    if (P.run_ac) H = std::max<int64_t>(H, P.T);
-    if (P.run_ssim) H = std::max<int64_t>(H, P.W - 1);
-    for (int r = 0; r < nranks; r++) {
-      const int64_t want_hi = std::min(H, F.nz - (tab[r].z0 + tab[r].nzl));
-      const bool contiguous = (r == 0 ? tab[r].z0 == 0 : tab[r].z0 == tab[r - 1].z0 + tab[r - 1].nzl);
-      if (!contiguous || tab[r].nzl < 1 || (r + 1 < nranks && tab[r + 1].nzl < want_hi) ||
-          (r == nranks - 1 && tab[r].z0 + tab[r].nzl != F.nz)) {
-        ctx->last_error = "slabs must tile dims[0] in rank order, each holding >= the halo depth";
-        return CZC_ERR_SHAPE;
-      }
-    }
-    hlo = (P.run_deriv && z0 > 0) ? 1 : 0;
-    hhi = std::min(H, F.nz - (z0 + nzl));
-    const int64_t prev_hhi = rank > 0 ? std::min(H, F.nz - z0) : 0;          // what rank-1 wants
-    const bool next_lo = P.run_deriv && rank + 1 < nranks;                  // rank+1 wants my last plane
-    const size_t pb = (size_t)plane * sizeof(float);
-    if ((st = ensure_buf(ctx, (void**)&ctx->halo, &ctx->halo_cap, 2 * (size_t)(hlo + hhi) * pb + 16)) != CZC_OK) return st;
-    float* xlo = ctx->halo;
-    float* ylo = xlo + hlo * plane;
-    float* xhi = ylo + hlo * plane;
-    float* yhi = xhi + hhi * plane;
-    if (!comm_group_begin(&ctx->last_error)) return comm_err(ctx);
-    bool ok = true;
-    if (rank > 0 && prev_hhi > 0) {
-      ok &= comm_send(ctx->comm, x, prev_hhi * pb, rank - 1, s, &ctx->last_error);
-      ok &= comm_send(ctx->comm, y, prev_hhi * pb, rank - 1, s, &ctx->last_error);
-    }
-    if (next_lo) {
-      ok &= comm_send(ctx->comm, x + (nzl - 1) * plane, pb, rank + 1, s, &ctx->last_error);
-      ok &= comm_send(ctx->comm, y + (nzl - 1) * plane, pb, rank + 1, s, &ctx->last_error);
-    }
-    if (hhi > 0) {
-      ok &= comm_recv(ctx->comm, xhi, hhi * pb, rank + 1, s, &ctx->last_error);
-      ok &= comm_recv(ctx->comm, yhi, hhi * pb, rank + 1, s, &ctx->last_error);
-    }
-    if (hlo > 0) {
-      ok &= comm_recv(ctx->comm, xlo, pb, rank - 1, s, &ctx->last_error);
-      ok &= comm_recv(ctx->comm, ylo, pb, rank - 1, s, &ctx->last_error);
-    }
-    if (!comm_group_end(&ctx->last_error) || !ok) return comm_err(ctx);
-    int k = 0;
-    if (hlo) { F.xs[k] = xlo; F.ys[k] = ylo; F.zs[k] = z0 - hlo; k++; }
-    F.xs[k] = x; F.ys[k] = y; F.zs[k] = z0; k++;
-    if (hhi) { F.xs[k] = xhi; F.ys[k] = yhi; F.zs[k] = z0 + nzl; k++; }
-    F.nseg = k;
-    F.zs[k] = z0 + nzl + hhi;
-  } else {
-    F.nseg = 1; F.xs[0] = x; F.ys[0] = y; F.zs[0] = 0; F.zs[1] = F.nz;
-  }
-
-  // ---- scratch sizing (partials of the largest launch) ------------------------------------------
-  size_t need = (size_t)ctx->p1_grid_cap * sizeof(P1State);
-  if (P.run_deriv) need = std::max(need, (size_t)deriv_blocks(F, zchunk_d) * kDerivSlots * sizeof(double));
-  if (P.run_ac) need = std::max(need, (size_t)ac_blocks(F, zchunk_ac) * kAcSlots * sizeof(double));
+SsimParams ssim_params(const Plan& P, const czc_config& c) {
   SsimParams sp{};
+  sp.sz = P.step[0]; sp.sy = P.step[1]; sp.sx = P.step[2];
+  sp.zchunk = kZchunkSsim;
+  sp.range_mode = c.ssim_range_mode;
+  sp.nwz = (P.g3[0] - P.win3[0]) / sp.sz + 1;
+  sp.nwy = (P.g3[1] - P.win3[1]) / sp.sy + 1;
+  sp.nwx = (P.g3[2] - P.win3[2]) / sp.sx + 1;
+  return sp;
+}
+
+// halo depth above a slab: derivatives need 1 plane, AC T planes, SSIM W - 1 planes
+int64_t halo_depth(const Plan& P) {
+  int64_t H = 0;
+  if (P.run_deriv) H = std::max<int64_t>(H, 1);
+  if (P.run_ac) H = std::max<int64_t>(H, P.T);
+  if (P.run_ssim) H = std::max<int64_t>(H, P.W - 1);
+  return H;
+}
+}  // namespace
+
+// Scratch for the largest launch over the given field view.
+static czc_status ensure_scratch(czc_ctx* ctx, const Plan& P, const Field3& F, const SsimParams& sp) {
+  size_t need = (size_t)ctx->p1_grid_cap * sizeof(P1State);
+  if (P.run_deriv) need = std::max(need, (size_t)deriv_blocks(F, kZchunkDeriv) * kDerivSlots * sizeof(double));
+  if (P.run_ac) need = std::max(need, (size_t)ac_blocks(F, 0) * kAcSlots * sizeof(double));
   if (P.run_ssim) {
-    sp.sz = P.step[0]; sp.sy = P.step[1]; sp.sx = P.step[2];
-    sp.zchunk = zchunk_ss;
-    sp.range_mode = ctx->cfg.ssim_range_mode;
-    sp.nwz = (F.nz - P.win3[0]) / sp.sz + 1;
-    sp.nwy = (F.ny - P.win3[1]) / sp.sy + 1;
-    sp.nwx = (F.nx - P.win3[2]) / sp.sx + 1;
     int64_t nb = 0;
-    if (launch_ssim(P.kind, P.W, F, sp, nullptr, nullptr, nullptr, nullptr, s, &nb) != cudaSuccess) {
+    if (launch_ssim(P.kind, P.W, F, sp, nullptr, nullptr, nullptr, nullptr, ctx->stream, &nb) != cudaSuccess) {
       ctx->last_error = "unsupported SSIM window";
       return CZC_ERR_UNSUPPORTED;
     }
     need = std::max(need, (size_t)nb * kSsimSlots * sizeof(double));
   }
-  if ((st = ensure_buf(ctx, &ctx->parts, &ctx->parts_cap, need)) != CZC_OK) return st;
+  return ensure_buf(ctx, &ctx->parts, &ctx->parts_cap, need);
+}
 
-  // ---- launches (coordinator order P1 -> P2 -> P3; AC needs P1's mu_e, sigma_e^2, Alg. 2) --
-  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
-  if (P.run_p1) {
-    CZC_CUDA(ctx, launch_p1(x, y, P.n, ctx->p1_grid_cap, (P1State*)ctx->parts, ctx->dres, ctx->tickets + TICKET_P1, s));
-    if (slab) {   // one small allgather of the partial moments, merged in rank order on device
-      if (!comm_allgather(ctx->comm, &ctx->dres->p1, ctx->dgather, sizeof(P1State), s, &ctx->last_error)) return comm_err(ctx);
-      CZC_CUDA(ctx, launch_p1_combine((const P1State*)ctx->dgather, nranks, ctx->dres, s));
-    }
-  }
-  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
+// P2 + P3 over one field view (the owned planes of F); results land in dres->rec.
+static czc_status run_p23(czc_ctx* ctx, const Plan& P, const Field3& F, const SsimParams& sp) {
+  const cudaStream_t s = ctx->stream;
+  czc_status st = ensure_scratch(ctx, P, F, sp);
+  if (st != CZC_OK) return st;
   if (P.run_deriv)
-    CZC_CUDA(ctx, launch_deriv(F, zchunk_d, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_DERIV, s));
+    CZC_CUDA(ctx, launch_deriv(F, kZchunkDeriv, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_DERIV, s));
   if (P.run_ac)
-    CZC_CUDA(ctx, launch_ac(F, P.T, zchunk_ac, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_ACZ, s));
-  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
+    CZC_CUDA(ctx, launch_ac(F, P.T, 0, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_ACZ, s));
+  if (ctx->cfg.timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
   if (P.run_ssim)
     CZC_CUDA(ctx, launch_ssim(P.kind, P.W, F, sp, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_SSIM,
                               ctx->cfg.debug_wssim, s, nullptr));
+  return CZC_OK;
+}
+
+static czc_status p1_local(czc_ctx* ctx, const Plan& P, const float* x, const float* y, int64_t n) {
+  if (!P.run_p1) return CZC_OK;
+  czc_status st = ensure_buf(ctx, &ctx->parts, &ctx->parts_cap, (size_t)ctx->p1_grid_cap * sizeof(P1State));
+  if (st != CZC_OK) return st;
+  CZC_CUDA(ctx, launch_p1(x, y, n, ctx->p1_grid_cap, (P1State*)ctx->parts, ctx->dres, ctx->tickets + TICKET_P1, ctx->stream));
+  return CZC_OK;
+}
+
+static void finish_timing(czc_ctx* ctx, czc_result* out) {
+  if (!ctx->cfg.timing) return;
+  cudaEventElapsedTime(&out->kernel_ms[0], ctx->ev[0], ctx->ev[1]);
+  cudaEventElapsedTime(&out->kernel_ms[1], ctx->ev[1], ctx->ev[2]);
+  cudaEventElapsedTime(&out->kernel_ms[2], ctx->ev[2], ctx->ev[3]);
+  cudaEventElapsedTime(&out->kernel_ms[3], ctx->ev[0], ctx->ev[4]);
+}
+
+// Single GPU, whole field resident.
+static czc_status assess_single(czc_ctx* ctx, const Plan& P, const float* x, const float* y, czc_result* out,
+                                uint64_t mask) {
+  const cudaStream_t s = ctx->stream;
+  const bool timing = ctx->cfg.timing != 0;
+  Field3 F{};
+  F.nz = P.g3[0]; F.ny = P.g3[1]; F.nx = P.g3[2];
+  F.zown0 = 0; F.zown1 = F.nz;
+  F.nseg = 1; F.xs[0] = x; F.ys[0] = y; F.zs[0] = 0; F.zs[1] = F.nz;
+  const SsimParams sp = ssim_params(P, ctx->cfg);
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
+  czc_status st = p1_local(ctx, P, x, y, F.nz * F.ny * F.nx);
+  if (st != CZC_OK) return st;
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));   // re-recorded inside run_p23
+  if ((st = run_p23(ctx, P, F, sp)) != CZC_OK) return st;
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));
-  DevResults R;
-  if (slab) {   // second small allgather: the P2 / P3 slot records, combined in rank order
-    if (!comm_allgather(ctx->comm, ctx->dres, ctx->dgather, sizeof(DevResults), s, &ctx->last_error)) return comm_err(ctx);
-    CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hgather, ctx->dgather, nranks * sizeof(DevResults), cudaMemcpyDeviceToHost, s));
-  } else {
-    CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hres, ctx->dres, sizeof(DevResults), cudaMemcpyDeviceToHost, s));
-  }
+  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, &ctx->dres->rec, sizeof(Record), cudaMemcpyDeviceToHost, s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
   CZC_CUDA(ctx, cudaStreamSynchronize(s));
-  if (slab) {
-    const DevResults* G = (const DevResults*)ctx->hgather;
-    R = G[0];
-    for (int r = 1; r < nranks; r++) {
-      for (int k = 0; k < kDerivSlots; k++) {
-        const int op = deriv_op(k);
-        R.deriv[k] = op == OP_SUM ? R.deriv[k] + G[r].deriv[k]
-                   : op == OP_MIN ? std::min(R.deriv[k], G[r].deriv[k]) : std::max(R.deriv[k], G[r].deriv[k]);
-      }
-      for (int w = 0; w < kAcWalks; w++)
-        for (int k = 0; k < kAcSlots; k++) R.ac[w][k] += G[r].ac[w][k];
-      for (int k = 0; k < kSsimSlots; k++) R.ssim[k] += G[r].ssim[k];
+  combine_and_finish(P, ctx->hrec, 1, mask, out);
+  finish_timing(ctx, out);
+  return CZC_OK;
+}
+
+// Field view of one slab [z0, z0 + nzl) whose halo planes live in ctx->halo (lo: hlo planes,
+// hi: hhi planes; filled by NCCL receives or, in loopback mode, device copies).
+static Field3 slab_field(czc_ctx* ctx, const Plan& P, const float* x, const float* y, int64_t z0, int64_t nzl,
+                         int64_t hlo, int64_t hhi, float** xlo, float** ylo, float** xhi, float** yhi) {
+  const int64_t plane = P.g3[1] * P.g3[2];
+  *xlo = ctx->halo;
+  *ylo = *xlo + hlo * plane;
+  *xhi = *ylo + hlo * plane;
+  *yhi = *xhi + hhi * plane;
+  Field3 F{};
+  F.nz = P.g3[0]; F.ny = P.g3[1]; F.nx = P.g3[2];
+  F.zown0 = z0; F.zown1 = z0 + nzl;
+  int k = 0;
+  if (hlo) { F.xs[k] = *xlo; F.ys[k] = *ylo; F.zs[k] = z0 - hlo; k++; }
+  F.xs[k] = x; F.ys[k] = y; F.zs[k] = z0; k++;
+  if (hhi) { F.xs[k] = *xhi; F.ys[k] = *yhi; F.zs[k] = z0 + nzl; k++; }
+  F.nseg = k;
+  F.zs[k] = z0 + nzl + hhi;
+  return F;
+}
+
+// Slab table check shared by both slab paths: slabs tile dims[0] in order and every slab holds
+// at least the halo depth its lower neighbour needs.
+static bool slabs_ok(const std::vector<std::pair<int64_t, int64_t>>& tab, int64_t nz, int64_t H) {
+  for (size_t r = 0; r < tab.size(); r++) {
+    const bool contiguous = r == 0 ? tab[r].first == 0 : tab[r].first == tab[r - 1].first + tab[r - 1].second;
+    if (!contiguous || tab[r].second < 1) return false;
+    if (r + 1 < tab.size() && tab[r + 1].second < std::min(H, nz - tab[r + 1].first)) return false;
+  }
+  return tab.back().first + tab.back().second == nz;
+}
+
+// Loopback: the multi-GPU algorithm on one GPU.  Slab k owns planes [z0_k, z0_k + n_k); its
+// halos are device-copied into ctx->halo (the buffers NCCL receives into); P1 states are merged
+// in slab order on the device before P2; per-slab records are combined in slab order on the host.
+static czc_status assess_loopback(czc_ctx* ctx, const Plan& P, const float* x, const float* y, czc_result* out,
+                                  uint64_t mask) {
+  const cudaStream_t s = ctx->stream;
+  const bool timing = ctx->cfg.timing != 0;
+  const int K = ctx->cfg.loopback_slabs;
+  const int64_t nz = P.g3[0], plane = P.g3[1] * P.g3[2];
+  if (P.D != 3 || nz < K) { ctx->last_error = "loopback slab mode needs a 3-D field with dims[0] >= slabs"; return CZC_ERR_SHAPE; }
+  std::vector<std::pair<int64_t, int64_t>> tab(K);
+  for (int k = 0; k < K; k++) {
+    const int64_t a = nz * k / K, b = nz * (k + 1) / K;
+    tab[k] = {a, b - a};
+  }
+  const int64_t H = halo_depth(P);
+  if (!slabs_ok(tab, nz, H)) { ctx->last_error = "slabs thinner than the halo depth"; return CZC_ERR_SHAPE; }
+  const SsimParams sp = ssim_params(P, ctx->cfg);
+  Record* drec = (Record*)ctx->dgather;
+  P1State* dst = (P1State*)ctx->dstates;
+  // one halo allocation for all slabs (a reallocation between slabs would synchronise the device)
+  czc_status st0 = ensure_buf(ctx, (void**)&ctx->halo, &ctx->halo_cap, 2 * (size_t)(1 + H) * plane * sizeof(float) + 16);
+  if (st0 != CZC_OK) return st0;
+  CZC_CUDA(ctx, cudaMemsetAsync(drec, 0, (size_t)K * sizeof(Record), s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
+  if (P.run_p1) {
+    for (int k = 0; k < K; k++) {
+      czc_status st = p1_local(ctx, P, x + tab[k].first * plane, y + tab[k].first * plane, tab[k].second * plane);
+      if (st != CZC_OK) return st;
+      CZC_CUDA(ctx, cudaMemcpyAsync(dst + k, &ctx->dres->rec.p1, sizeof(P1State), cudaMemcpyDeviceToDevice, s));
+      CZC_CUDA(ctx, cudaMemcpyAsync(&drec[k].p1, &ctx->dres->rec.p1, sizeof(P1State), cudaMemcpyDeviceToDevice, s));
     }
-  } else {
-    R = *ctx->hres;
+    CZC_CUDA(ctx, launch_p1_combine(dst, K, ctx->dres, s));
   }
-  finish_all(P, R, mask, out);
-  if (timing) {
-    cudaEventElapsedTime(&out->kernel_ms[0], ctx->ev[0], ctx->ev[1]);
-    cudaEventElapsedTime(&out->kernel_ms[1], ctx->ev[1], ctx->ev[2]);
-    cudaEventElapsedTime(&out->kernel_ms[2], ctx->ev[2], ctx->ev[3]);
-    cudaEventElapsedTime(&out->kernel_ms[3], ctx->ev[0], ctx->ev[4]);
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
+  for (int k = 0; k < K; k++) {
+    const int64_t z0 = tab[k].first, nzl = tab[k].second;
+    const int64_t hlo = (P.run_deriv && z0 > 0) ? 1 : 0;
+    const int64_t hhi = std::min(H, nz - (z0 + nzl));
+    czc_status st;
+    float *xlo, *ylo, *xhi, *yhi;
+    const Field3 F = slab_field(ctx, P, x + z0 * plane, y + z0 * plane, z0, nzl, hlo, hhi, &xlo, &ylo, &xhi, &yhi);
+    const size_t pb = (size_t)plane * sizeof(float);
+    if (hlo) {
+      CZC_CUDA(ctx, cudaMemcpyAsync(xlo, x + (z0 - 1) * plane, pb, cudaMemcpyDeviceToDevice, s));
+      CZC_CUDA(ctx, cudaMemcpyAsync(ylo, y + (z0 - 1) * plane, pb, cudaMemcpyDeviceToDevice, s));
+    }
+    if (hhi) {
+      CZC_CUDA(ctx, cudaMemcpyAsync(xhi, x + (z0 + nzl) * plane, hhi * pb, cudaMemcpyDeviceToDevice, s));
+      CZC_CUDA(ctx, cudaMemcpyAsync(yhi, y + (z0 + nzl) * plane, hhi * pb, cudaMemcpyDeviceToDevice, s));
+    }
+    if ((st = run_p23(ctx, P, F, sp)) != CZC_OK) return st;
+    CZC_CUDA(ctx, cudaMemcpyAsync(drec[k].deriv, ctx->dres->rec.deriv,
+                                  sizeof(Record) - offsetof(Record, deriv), cudaMemcpyDeviceToDevice, s));
   }
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));
+  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, drec, (size_t)K * sizeof(Record), cudaMemcpyDeviceToHost, s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
+  CZC_CUDA(ctx, cudaStreamSynchronize(s));
+  combine_and_finish(P, ctx->hrec, K, mask, out);
+  finish_timing(ctx, out);
+  return CZC_OK;
+}
+
+// NCCL slab mode: this rank holds planes [z0, z0 + nzl) of the global field.
+static czc_status assess_ranks(czc_ctx* ctx, const Plan& P, const float* x, const float* y, const czc_shape* shape,
+                               czc_result* out, uint64_t mask) {
+  const cudaStream_t s = ctx->stream;
+  const bool timing = ctx->cfg.timing != 0;
+  const int nranks = comm_size(ctx->comm), rank = comm_rank(ctx->comm);
+  const int64_t nz = P.g3[0], plane = P.g3[1] * P.g3[2];
+  if (P.D != 3 || shape->dims[0] != nz) { ctx->last_error = "slab mode needs a 3-D field split along dims[0]"; return CZC_ERR_SHAPE; }
+  const int64_t z0 = shape->z0, nzl = shape->nz_local > 0 ? shape->nz_local : nz;
+  // slab table: every rank validates every slab identically (a collective decision, no hang)
+  int64_t mine[2] = {z0, nzl};
+  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->dgather_in, mine, sizeof(mine), cudaMemcpyHostToDevice, s));
+  if (!comm_allgather(ctx->comm, ctx->dgather_in, ctx->dgather, sizeof(mine), s, &ctx->last_error)) return CZC_ERR_COMM;
+  std::vector<int64_t> flat(2 * nranks);
+  CZC_CUDA(ctx, cudaMemcpyAsync(flat.data(), ctx->dgather, flat.size() * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  CZC_CUDA(ctx, cudaStreamSynchronize(s));
+  std::vector<std::pair<int64_t, int64_t>> tab(nranks);
+  for (int r = 0; r < nranks; r++) tab[r] = {flat[2 * r], flat[2 * r + 1]};
+  const int64_t H = halo_depth(P);
+  if (!slabs_ok(tab, nz, H)) { ctx->last_error = "slabs must tile dims[0] in rank order, each >= the halo depth"; return CZC_ERR_SHAPE; }
+  const SsimParams sp = ssim_params(P, ctx->cfg);
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
+  // halo exchange: H planes up from rank+1, one plane (derivatives) down from rank-1
+  const int64_t hlo = (P.run_deriv && z0 > 0) ? 1 : 0;
+  const int64_t hhi = std::min(H, nz - (z0 + nzl));
+  const int64_t prev_hhi = rank > 0 ? std::min(H, nz - z0) : 0;
+  const bool next_lo = P.run_deriv && rank + 1 < nranks;
+  const size_t pb = (size_t)plane * sizeof(float);
+  czc_status st = ensure_buf(ctx, (void**)&ctx->halo, &ctx->halo_cap, 2 * (size_t)(hlo + hhi) * pb + 16);
+  if (st != CZC_OK) return st;
+  float *xlo, *ylo, *xhi, *yhi;
+  const Field3 F = slab_field(ctx, P, x, y, z0, nzl, hlo, hhi, &xlo, &ylo, &xhi, &yhi);
+  if (!comm_group_begin(&ctx->last_error)) return CZC_ERR_COMM;
+  bool ok = true;
+  if (rank > 0 && prev_hhi > 0) {
+    ok &= comm_send(ctx->comm, x, prev_hhi * pb, rank - 1, s, &ctx->last_error);
+    ok &= comm_send(ctx->comm, y, prev_hhi * pb, rank - 1, s, &ctx->last_error);
+  }
+  if (next_lo) {
+    ok &= comm_send(ctx->comm, x + (nzl - 1) * plane, pb, rank + 1, s, &ctx->last_error);
+    ok &= comm_send(ctx->comm, y + (nzl - 1) * plane, pb, rank + 1, s, &ctx->last_error);
+  }
+  if (hhi > 0) {
+    ok &= comm_recv(ctx->comm, xhi, hhi * pb, rank + 1, s, &ctx->last_error);
+    ok &= comm_recv(ctx->comm, yhi, hhi * pb, rank + 1, s, &ctx->last_error);
+  }
+  if (hlo > 0) {
+    ok &= comm_recv(ctx->comm, xlo, pb, rank - 1, s, &ctx->last_error);
+    ok &= comm_recv(ctx->comm, ylo, pb, rank - 1, s, &ctx->last_error);
+  }
+  if (!comm_group_end(&ctx->last_error) || !ok) return CZC_ERR_COMM;
+  // P1 on the local slab, then one small allgather of the states, merged in rank order on device
+  if ((st = p1_local(ctx, P, x, y, nzl * plane)) != CZC_OK) return st;
+  if (P.run_p1) {
+    if (!comm_allgather(ctx->comm, &ctx->dres->rec.p1, ctx->dstates, sizeof(P1State), s, &ctx->last_error)) return CZC_ERR_COMM;
+    CZC_CUDA(ctx, launch_p1_combine((const P1State*)ctx->dstates, nranks, ctx->dres, s));
+  }
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
+  if ((st = run_p23(ctx, P, F, sp)) != CZC_OK) return st;
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));
+  // second small allgather: every rank's record, combined in rank order on the host
+  if (!comm_allgather(ctx->comm, &ctx->dres->rec, ctx->dgather, sizeof(Record), s, &ctx->last_error)) return CZC_ERR_COMM;
+  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, ctx->dgather, (size_t)nranks * sizeof(Record), cudaMemcpyDeviceToHost, s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
+  CZC_CUDA(ctx, cudaStreamSynchronize(s));
+  combine_and_finish(P, ctx->hrec, nranks, mask, out);
+  finish_timing(ctx, out);
   return CZC_OK;
 }
 
@@ -508,7 +650,24 @@ extern "C" czc_status czc_assess(czc_ctx* ctx, const void* orig, const void* rec
   czc_status st = check_common(ctx, orig, recon, shape, dtype, out);
   if (st != CZC_OK) return st;
   if (cudaSetDevice(ctx->device) != cudaSuccess) return cuda_fail(ctx, cudaGetLastError(), "cudaSetDevice");
-  st = assess_core(ctx, (const float*)orig, (const float*)recon, shape, metric_mask, out);
+  Plan P;
+  st = make_plan(ctx->cfg, shape->ndim, shape->dims, metric_mask, P, ctx->last_error);
+  if (st == CZC_OK) {
+    const int64_t nzl = shape->nz_local > 0 ? shape->nz_local : shape->dims[0];
+    if (shape->z0 < 0 || shape->z0 + nzl > shape->dims[0]) {
+      ctx->last_error = "slab [z0, z0+nz_local) outside dims[0]";
+      st = CZC_ERR_SHAPE;
+    } else if (!ctx->comm && (shape->z0 != 0 || nzl != shape->dims[0])) {
+      ctx->last_error = "a slab shape needs nranks > 1";
+      st = CZC_ERR_SHAPE;
+    } else if (ctx->comm) {
+      st = assess_ranks(ctx, P, (const float*)orig, (const float*)recon, shape, out, metric_mask);
+    } else if (ctx->cfg.loopback_slabs > 1) {
+      st = assess_loopback(ctx, P, (const float*)orig, (const float*)recon, out, metric_mask);
+    } else {
+      st = assess_single(ctx, P, (const float*)orig, (const float*)recon, out, metric_mask);
+    }
+  }
   if (st != CZC_OK) out->computed_mask = 0;
   return st;
 }

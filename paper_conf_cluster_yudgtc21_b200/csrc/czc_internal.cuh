@@ -110,12 +110,21 @@ constexpr int kAcWalks = 3;
 // SSIM record: [sum of local SSIM, number of windows, windows recomputed exactly]
 constexpr int kSsimSlots = 3;
 
-// Device-side results of one czc_assess call (fetched with one D2H copy at the end).
-struct DevResults {
-  P1State p1;
+// The partial-result record of one field (or one slab of it): what one rank contributes and what
+// the rank-ordered combine consumes (czc_combine).  Layout is internal, size = czc_sizeof(3).
+struct Record {
+  P1State p1;                        // this field's / slab's own P1 state
   double deriv[kDerivSlots];
   double ac[kAcWalks][kAcSlots];
   double ssim[kSsimSlots];
+};
+
+// Device-side results of one launch sequence.  The kernels write `rec`; the AC and SSIM kernels
+// read `p1g`, the GLOBAL P1 state (single GPU: a copy of rec.p1; slab mode: the rank-ordered
+// merge of every slab's state), for mu_e, sigma_e^2 and the global range.
+struct DevResults {
+  Record rec;
+  P1State p1g;
 };
 
 // A 3-D field view for the stencil / window kernels: global extents, the planes this launch
@@ -145,6 +154,27 @@ struct Field3 {
   }
 #endif
 };
+
+#if defined(__CUDACC__)
+// Sequential plane cursor over a Field3 (z increasing by one per step): pointer increments, with
+// the segment base re-derived only when a segment boundary is crossed.
+struct PlaneCursor {
+  const float* x;
+  const float* y;
+  int64_t z, next_seg;
+  __device__ __forceinline__ void init(const Field3& f, int64_t z0, int64_t off) {
+    z = z0;
+    x = f.xp(z0) + off;
+    y = f.yp(z0) + off;
+    next_seg = (f.nseg > 1 && z0 < f.zs[1]) ? f.zs[1] : ((f.nseg > 2 && z0 < f.zs[2]) ? f.zs[2] : INT64_MAX);
+  }
+  __device__ __forceinline__ void advance(const Field3& f, int64_t off) {
+    ++z;
+    if (z == next_seg) init(f, z, off);
+    else { x += f.ny * f.nx; y += f.ny * f.nx; }
+  }
+};
+#endif
 
 struct SsimParams {
   int sz, sy, sx;            // steps
@@ -226,6 +256,16 @@ __device__ void block_reduce_slots(double (&v)[K], OpOf op_of, double* dst_globa
     }
     __syncthreads();
   }
+}
+
+// 1/v for finite normal v > 0: rcp.approx (MUFU.RCP64H) + two Newton steps, |rel err| <= 2u.
+__device__ __forceinline__ double fast_rcp(double v) {
+  double r;
+  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(v));
+  double e = fma(-v, r, 1.0);
+  r = fma(r, e, r);
+  e = fma(-v, r, 1.0);
+  return fma(r, e, r);
 }
 
 __device__ __forceinline__ float4 ld_stream_f4(const float4* p) {

@@ -31,24 +31,17 @@ __device__ __forceinline__ void acc_init(P1Acc& a, float kxf, float kyf) {
   a.xmin = finf(); a.xmax = -finf();
 }
 
-// 1/v for v > 0 (finite, normal): rcp.approx (MUFU.RCP64H) + two Newton steps -> |rel err| <= 2u.
-__device__ __forceinline__ double fast_rcp(double v) {
-  double r;
-  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(v));
-  double e = fma(-v, r, 1.0);
-  r = fma(r, e, r);
-  e = fma(-v, r, 1.0);
-  return fma(r, e, r);
-}
 
 // One element: e = recon - orig in double (reading R1; same rounding as the oracle).  Point-wise
 // relative error |e|/|x| (reading R3): its SUM uses q~ = |e| * rcp(|x|) (relative error <= 4u,
 // far inside the 1e-9 tolerance of pwr_mean); its extrema must be the IEEE quotient, bit-exact
-// with the oracle, so the correctly rounded division runs only for candidates: an element can be
-// the maximum only if q~ >= pmax (1 - 1e-12) (q~ >= Q (1 - 4u) and pmax <= RN(Q) for the true
-// maximum Q), and symmetrically for the minimum.  After the first few elements of a thread
-// candidates are rare, so the division is off the hot path.
-__device__ __forceinline__ void acc_elem(P1Acc& a, float xf, float yf) {
+// with the oracle, so the correctly rounded division runs only for candidates: an element can
+// raise the maximum only if q~ > thr_hi = pmax (1 - 1e-12) (q~ >= Q (1 - 4u) and pmax <= RN(Q)
+// for a larger true quotient Q), and lower the minimum only if q~ < thr_lo = pmin (1 + 1e-12);
+// a zero minimum admits no further candidate (thr_lo = 0), a zero maximum admits only q~ > 0.
+// Returns whether this element is a candidate; the caller resolves candidates per vector so the
+// hot loop has one rarely-taken branch per 4 elements.
+__device__ __forceinline__ bool acc_elem(P1Acc& a, float xf, float yf, double& ae_out, double& ax_out) {
   const double x = xf, y = yf;
   const double e = y - x;
   const double da = x - a.kx, db = y - a.ky, dc = e - a.ke;
@@ -68,18 +61,34 @@ __device__ __forceinline__ void acc_elem(P1Acc& a, float xf, float yf) {
   const double qa = nz ? ae * fast_rcp(ax) : 0.0;
   a.spwr += qa;
   a.npwr += nz ? 1u : 0u;
-  if (nz && (qa >= a.pthr_hi || qa <= a.pthr_lo)) {
-    const double q = ae / ax;                        // IEEE, correctly rounded
-    if (q > a.pmax) { a.pmax = q; a.pthr_hi = q * (1.0 - 1e-12); }
-    if (q < a.pmin) { a.pmin = q; a.pthr_lo = q * (1.0 + 1e-12); }
-  }
+  ae_out = ae;
+  ax_out = ax;
+  return nz && (qa > a.pthr_hi || qa < a.pthr_lo);
+}
+
+__device__ __forceinline__ void acc_resolve(P1Acc& a, double ae, double ax) {
+  const double q = ae / ax;                          // IEEE, correctly rounded
+  if (q > a.pmax) { a.pmax = q; a.pthr_hi = q * (1.0 - 1e-12); }
+  if (q < a.pmin) { a.pmin = q; a.pthr_lo = q * (1.0 + 1e-12); }   // q = 0 -> thr_lo = 0
 }
 
 __device__ __forceinline__ void acc_vec(P1Acc& a, float4 xv, float4 yv) {
-  acc_elem(a, xv.x, yv.x);
-  acc_elem(a, xv.y, yv.y);
-  acc_elem(a, xv.z, yv.z);
-  acc_elem(a, xv.w, yv.w);
+  double ae0, ax0, ae1, ax1, ae2, ax2, ae3, ax3;
+  const bool c0 = acc_elem(a, xv.x, yv.x, ae0, ax0);
+  const bool c1 = acc_elem(a, xv.y, yv.y, ae1, ax1);
+  const bool c2 = acc_elem(a, xv.z, yv.z, ae2, ax2);
+  const bool c3 = acc_elem(a, xv.w, yv.w, ae3, ax3);
+  if (c0 | c1 | c2 | c3) {                            // rare after the first few vectors
+    if (c0) acc_resolve(a, ae0, ax0);
+    if (c1) acc_resolve(a, ae1, ax1);
+    if (c2) acc_resolve(a, ae2, ax2);
+    if (c3) acc_resolve(a, ae3, ax3);
+  }
+}
+
+__device__ __forceinline__ void acc_scalar(P1Acc& a, float xf, float yf) {
+  double ae, ax;
+  if (acc_elem(a, xf, yf, ae, ax)) acc_resolve(a, ae, ax);
 }
 
 __device__ __forceinline__ P1State acc_to_state(const P1Acc& a, double n) {
@@ -156,25 +165,30 @@ p1_kernel(const float* __restrict__ x, const float* __restrict__ y, int64_t n, i
     const float4* y4 = reinterpret_cast<const float4*>(y + head);
     int64_t v = gtid;
     if (gtid < nvec) cnt = 4 * ((nvec - 1 - gtid) / gsz + 1);
-    for (; v + 3 * gsz < nvec; v += 4 * gsz) {   // 4 independent 2x16-byte loads in flight
-      const float4 xa = ld_stream_f4(x4 + v), ya = ld_stream_f4(y4 + v);
-      const float4 xb = ld_stream_f4(x4 + v + gsz), yb = ld_stream_f4(y4 + v + gsz);
-      const float4 xc = ld_stream_f4(x4 + v + 2 * gsz), yc = ld_stream_f4(y4 + v + 2 * gsz);
-      const float4 xd = ld_stream_f4(x4 + v + 3 * gsz), yd = ld_stream_f4(y4 + v + 3 * gsz);
+    // software pipeline: the next two vectors' loads are in flight while two are processed
+    if (v + gsz < nvec) {
+      float4 xa = ld_stream_f4(x4 + v), ya = ld_stream_f4(y4 + v);
+      float4 xb = ld_stream_f4(x4 + v + gsz), yb = ld_stream_f4(y4 + v + gsz);
+      v += 2 * gsz;
+      for (; v + gsz < nvec; v += 2 * gsz) {
+        const float4 xc = ld_stream_f4(x4 + v), yc = ld_stream_f4(y4 + v);
+        const float4 xd = ld_stream_f4(x4 + v + gsz), yd = ld_stream_f4(y4 + v + gsz);
+        acc_vec(a, xa, ya);
+        acc_vec(a, xb, yb);
+        xa = xc; ya = yc; xb = xd; yb = yd;
+      }
       acc_vec(a, xa, ya);
       acc_vec(a, xb, yb);
-      acc_vec(a, xc, yc);
-      acc_vec(a, xd, yd);
     }
     for (; v < nvec; v += gsz) acc_vec(a, ld_stream_f4(x4 + v), ld_stream_f4(y4 + v));
     if (gtid < nleft) {
       const int64_t i = left_index(gtid);
-      acc_elem(a, x[i], y[i]);
+      acc_scalar(a, x[i], y[i]);
       cnt += 1;
     }
   } else {
     if (gtid < n) cnt = (n - 1 - gtid) / gsz + 1;
-    for (int64_t i = gtid; i < n; i += gsz) acc_elem(a, x[i], y[i]);
+    for (int64_t i = gtid; i < n; i += gsz) acc_scalar(a, x[i], y[i]);
   }
 
   P1State s = block_merge(acc_to_state(a, (double)cnt));
@@ -194,7 +208,8 @@ p1_kernel(const float* __restrict__ x, const float* __restrict__ y, int64_t n, i
   }
   f = block_merge(f);
   if (threadIdx.x == 0) {
-    res->p1 = f;
+    res->rec.p1 = f;
+    res->p1g = f;
     *ticket = 0;   // re-arm for the next launch
   }
 }
@@ -225,7 +240,7 @@ __global__ void p1_combine_kernel(const P1State* __restrict__ states, int count,
   P1State f;
   p1_empty(f);
   for (int r = 0; r < count; r++) p1_merge(f, states[r]);
-  res->p1 = f;
+  res->p1g = f;
 }
 
 cudaError_t launch_p1_combine(const P1State* states, int count, DevResults* res, cudaStream_t st) {

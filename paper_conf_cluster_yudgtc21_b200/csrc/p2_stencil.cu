@@ -154,7 +154,7 @@ deriv_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __res
   const unsigned bid = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
   block_reduce_slots<kDerivSlots>(acc, DerivOp{}, parts + (size_t)bid * kDerivSlots);
   if (!last_block_arrive(ticket)) return;
-  finish_slots<kDerivSlots>(parts, gridDim.x * gridDim.y * gridDim.z, DerivOp{}, res->deriv);
+  finish_slots<kDerivSlots>(parts, gridDim.x * gridDim.y * gridDim.z, DerivOp{}, res->rec.deriv);
   if (tid == 0) *ticket = 0;
 }
 
@@ -196,27 +196,29 @@ __device__ __forceinline__ void ac_finish(double (&acc)[TM], double* parts, doub
   if (threadIdx.x + threadIdx.y == 0) *ticket = 0;
 }
 
-// Walk of one line with element stride `stride` through up to three plane segments (z-walk) or a
-// single row (y-walk: stride nx within one plane).  Positions [lo, end) are visited; points p in
-// [lo, hi) own their products.  TM loads are kept in flight in a register queue (slot u of the
-// TM-unrolled loop holds position i0 + u), so the queue also rotates statically.
-template <int TM, typename PtrOf>
-__device__ __forceinline__ void walk_line(PtrOf ptr_of, int64_t lo, int64_t hi, int64_t end, double mu,
+// Walk of one line.  Positions [lo, end) are visited; points p in [lo, hi) own their products.
+// `next` returns the (x, y) sample at the position of a load cursor that runs QD = 2 TM positions
+// ahead of the walk: QD loads stay in flight in a register queue whose slot u (of the QD-unrolled
+// loop) holds position i0 + u, so both the queue and the ring (QD is a multiple of TM) rotate
+// statically.
+template <int TM, typename Next>
+__device__ __forceinline__ void walk_line(Next next, int64_t lo, int64_t hi, int64_t end, double mu,
                                           bool own, double (&ring)[TM], double (&acc)[TM]) {
-  float qx[TM], qy[TM];
+  constexpr int QD = 2 * TM;
+  float qx[QD], qy[QD];
 #pragma unroll
-  for (int u = 0; u < TM; u++) {
+  for (int u = 0; u < QD; u++) {
     qx[u] = 0.f; qy[u] = 0.f;
-    if (own && lo + u < end) { const float2 v = ptr_of(lo + u); qx[u] = v.x; qy[u] = v.y; }
+    if (own && lo + u < end) { const float2 v = next(); qx[u] = v.x; qy[u] = v.y; }
   }
-  for (int64_t i0 = lo; i0 < end; i0 += TM) {
+  for (int64_t i0 = lo; i0 < end; i0 += QD) {
 #pragma unroll
-    for (int u = 0; u < TM; u++) {
+    for (int u = 0; u < QD; u++) {
       const int64_t i = i0 + u;
       if (i < end) {
         const double eps = ((double)qy[u] - (double)qx[u]) - mu;
-        if (own && i + TM < end) { const float2 v = ptr_of(i + TM); qx[u] = v.x; qy[u] = v.y; }
-        walk_step<TM>(ring, acc, eps, i < hi, u);
+        if (own && i + QD < end) { const float2 v = next(); qx[u] = v.x; qy[u] = v.y; }
+        walk_step<TM>(ring, acc, eps, i < hi, u % TM);
       }
     }
   }
@@ -228,7 +230,7 @@ __global__ void __launch_bounds__(256)
 ac_zwalk(Field3 s, int T, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
          unsigned int* __restrict__ ticket) {
   const int64_t gx = (int64_t)blockIdx.x * kTX + threadIdx.x, gy = (int64_t)blockIdx.y * kTY + threadIdx.y;
-  const double mu = res->p1.me;
+  const double mu = res->p1g.me;
   const bool own = gx < s.nx && gy < s.ny;
   int64_t m = T;
   if (s.ny > 1 && s.ny - 1 - gy < m) m = s.ny - 1 - gy;
@@ -242,19 +244,26 @@ ac_zwalk(Field3 s, int T, int zchunk, double* __restrict__ parts, DevResults* __
   double ring[TM], acc[TM];
 #pragma unroll
   for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
-  walk_line<TM>([&](int64_t z) { return make_float2(__ldg(s.xp(z) + col), __ldg(s.yp(z) + col)); }, lo, hi, end, mu, own, ring, acc);
+  PlaneCursor cur;
+  if (own && lo < end) cur.init(s, lo, col);
+  walk_line<TM>([&]() {                 // read the cursor's plane, then step it (never read past end)
+    const float2 v = make_float2(__ldg(cur.x), __ldg(cur.y));
+    cur.advance(s, col);
+    return v;
+  }, lo, hi, end, mu, own, ring, acc);
   walk_mask<TM>(acc, own ? (int)m : 0);
-  ac_finish<TM>(acc, parts, res->ac[0], ticket);
+  ac_finish<TM>(acc, parts, res->rec.ac[0], ticket);
 }
 
-// y-walk: thread <-> line (z, x); block 32 (x) x 8 (z); grid.z chunks of y.
+// y-walk: thread <-> line (z, x); a block's 256 threads cover 256 consecutive x of one plane (one
+// 1 KB contiguous row segment per step); grid (x tiles, owned planes, y chunks).
 template <int TM>
 __global__ void __launch_bounds__(256)
 ac_ywalk(Field3 s, int T, int ychunk, double* __restrict__ parts, DevResults* __restrict__ res,
          unsigned int* __restrict__ ticket) {
-  const int64_t gx = (int64_t)blockIdx.x * kTX + threadIdx.x;
-  const int64_t z = s.zown0 + (int64_t)blockIdx.y * kTY + threadIdx.y;
-  const double mu = res->p1.me;
+  const int64_t gx = (int64_t)blockIdx.x * 256 + threadIdx.x;
+  const int64_t z = s.zown0 + (int64_t)blockIdx.y;
+  const double mu = res->p1g.me;
   const bool own = gx < s.nx && z < s.zown1;
   int64_t m = T;
   if (s.nz > 1 && s.nz - 1 - z < m) m = s.nz - 1 - z;
@@ -270,9 +279,69 @@ ac_ywalk(Field3 s, int T, int ychunk, double* __restrict__ parts, DevResults* __
   double ring[TM], acc[TM];
 #pragma unroll
   for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
-  walk_line<TM>([&](int64_t y) { return make_float2(__ldg(X + y * nx), __ldg(Y + y * nx)); }, lo, hi, end, mu, own, ring, acc);
+  const float* px = own ? X + lo * nx : nullptr;
+  const float* py = own ? Y + lo * nx : nullptr;
+  walk_line<TM>([&]() {
+    const float2 v = make_float2(__ldg(px), __ldg(py));
+    px += nx; py += nx;
+    return v;
+  }, lo, hi, end, mu, own, ring, acc);
   walk_mask<TM>(acc, own ? (int)m : 0);
-  ac_finish<TM>(acc, parts, res->ac[1], ticket);
+  ac_finish<TM>(acc, parts, res->rec.ac[1], ticket);
+}
+
+// x-walk, fast path (rows 16-byte aligned: nx % 4 == 0 and aligned segment bases): lane l of
+// each warp owns row (z, y) and streams it with 128-bit loads straight into registers, 4 columns
+// per load, two loads in flight ahead; the chunk start lo is a multiple of 4 (xchunk % 4 == 0).
+// 32 rows per warp touch 32 lines per load instruction, each line reused over 8 loads (L1).
+template <int TM>
+__global__ void __launch_bounds__(256)
+ac_xwalk_vec(Field3 s, int T, int xchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+             unsigned int* __restrict__ ticket) {
+  constexpr int LCM = (TM % 4 == 0) ? TM : ((TM % 2 == 0) ? 2 * TM : 4 * TM);   // lcm(4, TM)
+  constexpr int NV = LCM / 4;                        // float4 vectors per ring period
+  const double mu = res->p1g.me;
+  const int64_t nrows = (s.zown1 - s.zown0) * s.ny;
+  const int64_t myrow = (int64_t)blockIdx.x * 256 + threadIdx.x;
+  const bool own = myrow < nrows;
+  const int64_t z = own ? s.zown0 + myrow / s.ny : s.zown0, y = own ? myrow % s.ny : 0;
+  int64_t m = T;
+  if (s.nz > 1 && s.nz - 1 - z < m) m = s.nz - 1 - z;
+  if (s.ny > 1 && s.ny - 1 - y < m) m = s.ny - 1 - y;
+  const int64_t lo = (int64_t)blockIdx.y * xchunk;
+  int64_t hi = lo + xchunk;
+  if (hi > s.nx) hi = s.nx;
+  int64_t end = hi + T;
+  if (end > s.nx) end = s.nx;
+  const float4* X = reinterpret_cast<const float4*>(s.xp(z) + y * s.nx + lo);
+  const float4* Y = reinterpret_cast<const float4*>(s.yp(z) + y * s.nx + lo);
+  const int64_t nvec = (end - lo + 3) / 4;           // the row tail is padded by the next row
+  double ring[TM], acc[TM];
+#pragma unroll
+  for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
+  float4 ax = make_float4(0, 0, 0, 0), ay = ax, bx = ax, by = ax;
+  if (own && nvec > 0) { ax = __ldg(X); ay = __ldg(Y); }
+  if (own && nvec > 1) { bx = __ldg(X + 1); by = __ldg(Y + 1); }
+  for (int64_t v0 = 0; v0 < nvec; v0 += NV) {
+#pragma unroll
+    for (int k = 0; k < NV; k++) {
+      const int64_t v = v0 + k;
+      if (v < nvec) {
+        const float4 cx = ax, cy = ay;
+        ax = bx; ay = by;
+        if (own && v + 2 < nvec) { bx = __ldg(X + v + 2); by = __ldg(Y + v + 2); }
+        const float xs4[4] = {cx.x, cx.y, cx.z, cx.w};
+        const float ys4[4] = {cy.x, cy.y, cy.z, cy.w};
+#pragma unroll
+        for (int j = 0; j < 4; j++) {
+          const int64_t c = lo + 4 * v + j;
+          if (c < end) walk_step<TM>(ring, acc, ((double)ys4[j] - (double)xs4[j]) - mu, c < hi, (4 * k + j) % TM);
+        }
+      }
+    }
+  }
+  walk_mask<TM>(acc, own ? (int)m : 0);
+  ac_finish<TM>(acc, parts, res->rec.ac[2], ticket);
 }
 
 // x-walk: each warp owns 32 consecutive rows (z, y); per segment of SEG columns (a multiple of
@@ -282,12 +351,12 @@ ac_ywalk(Field3 s, int T, int ychunk, double* __restrict__ parts, DevResults* __
 constexpr int kXWarps = 4;   // 4 warps x 32 rows per block (tile: 4 x 32 x <=33 doubles <= 34 KB)
 template <int TM>
 __global__ void __launch_bounds__(kXWarps * 32)
-ac_xwalk(Field3 s, int T, int xchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+ac_xwalk_smem(Field3 s, int T, int xchunk, double* __restrict__ parts, DevResults* __restrict__ res,
          unsigned int* __restrict__ ticket) {
   constexpr int SEG = (32 / TM) * TM;
   __shared__ double tile[kXWarps][32][SEG + 1];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const double mu = res->p1.me;
+  const double mu = res->p1g.me;
   const int64_t nrows = (s.zown1 - s.zown0) * s.ny;
   const int64_t row0 = ((int64_t)blockIdx.x * kXWarps + warp) * 32;   // first row of this warp
   const int64_t myrow = row0 + lane;
@@ -339,7 +408,7 @@ ac_xwalk(Field3 s, int T, int xchunk, double* __restrict__ parts, DevResults* __
     __syncwarp();
   }
   walk_mask<TM>(acc, own ? (int)m : 0);
-  ac_finish<TM>(acc, parts, res->ac[2], ticket);
+  ac_finish<TM>(acc, parts, res->rec.ac[2], ticket);
 }
 
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
@@ -366,24 +435,25 @@ cudaError_t launch_deriv(const Field3& s, int zchunk, double* parts, DevResults*
 // Autocorrelation: one launch per active walk axis, each with its own partial-buffer slice and
 // ticket; the three records are summed at the finish.
 struct AcGrids {
-  dim3 z, y, x;
+  dim3 z, y, x, xvec;
   bool rz, ry, rx;
   int zc, yc, xc;
 };
 static AcGrids ac_grids(const Field3& s) {
   AcGrids g{};
   const int64_t nzo = s.zown1 - s.zown0;
-  g.zc = 50; g.yc = 125; g.xc = 125;
+  g.zc = 50; g.yc = 125; g.xc = 128;   // xc % 4 == 0 for the vector x-walk
   g.rz = s.nz > 1; g.ry = s.ny > 1; g.rx = s.nx > 1;
   g.z = dim3((unsigned)cdiv(s.nx, kTX), (unsigned)cdiv(s.ny, kTY), (unsigned)cdiv(nzo, g.zc));
-  g.y = dim3((unsigned)cdiv(s.nx, kTX), (unsigned)cdiv(nzo, kTY), (unsigned)cdiv(s.ny, g.yc));
+  g.y = dim3((unsigned)cdiv(s.nx, 256), (unsigned)nzo, (unsigned)cdiv(s.ny, g.yc));
   g.x = dim3((unsigned)cdiv(nzo * s.ny, kXWarps * 32), (unsigned)cdiv(s.nx, g.xc), 1);
+  g.xvec = dim3((unsigned)cdiv(nzo * s.ny, 256), (unsigned)cdiv(s.nx, g.xc), 1);
   return g;
 }
 int64_t ac_blocks(const Field3& s, int) {
   const AcGrids g = ac_grids(s);
   auto n = [](dim3 d) { return (int64_t)d.x * d.y * d.z; };
-  return n(g.z) + n(g.y) + n(g.x);
+  return n(g.z) + n(g.y) + (n(g.x) > n(g.xvec) ? n(g.x) : n(g.xvec));
 }
 
 template <int TM>
@@ -393,11 +463,16 @@ static cudaError_t launch_ac_t(const Field3& s, int T, double* parts, DevResults
   double* pz = parts;
   double* py = pz + (size_t)g.z.x * g.z.y * g.z.z * kAcSlots;
   double* px = py + (size_t)g.y.x * g.y.y * g.y.z * kAcSlots;
-  cudaError_t e = cudaMemsetAsync(res->ac, 0, sizeof(res->ac), st);
+  cudaError_t e = cudaMemsetAsync(res->rec.ac, 0, sizeof(res->rec.ac), st);
   if (e != cudaSuccess) return e;
   if (g.rz) ac_zwalk<TM><<<g.z, dim3(kTX, kTY), 0, st>>>(s, T, g.zc, pz, res, tickets + 0);
-  if (g.ry) ac_ywalk<TM><<<g.y, dim3(kTX, kTY), 0, st>>>(s, T, g.yc, py, res, tickets + 1);
-  if (g.rx) ac_xwalk<TM><<<g.x, kXWarps * 32, 0, st>>>(s, T, g.xc, px, res, tickets + 2);
+  if (g.ry) ac_ywalk<TM><<<g.y, 256, 0, st>>>(s, T, g.yc, py, res, tickets + 1);
+  // vector x-walk when every row start is 16-byte aligned (nx % 4 == 0, aligned segments)
+  bool vec = (s.nx % 4) == 0;
+  for (int k = 0; k < s.nseg; k++)
+    vec = vec && (reinterpret_cast<uintptr_t>(s.xs[k]) % 16) == 0 && (reinterpret_cast<uintptr_t>(s.ys[k]) % 16) == 0;
+  if (g.rx && vec) ac_xwalk_vec<TM><<<g.xvec, 256, 0, st>>>(s, T, g.xc, px, res, tickets + 2);
+  else if (g.rx) ac_xwalk_smem<TM><<<g.x, kXWarps * 32, 0, st>>>(s, T, g.xc, px, res, tickets + 2);
   return cudaGetLastError();
 }
 

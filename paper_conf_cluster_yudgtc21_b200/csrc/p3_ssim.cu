@@ -29,8 +29,8 @@
 
 namespace czc {
 
-constexpr int kP3Threads = 256;
 constexpr int kP3Warps = 8;
+constexpr int kP3Threads = 32 * kP3Warps;
 
 template <int WX, int WY, int WZ, int G>
 struct SsimGeom {
@@ -109,7 +109,7 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
   if (ky > f.ny - 1) ky = f.ny - 1;
   if (kx > f.nx - 1) kx = f.nx - 1;
   const double K = (zb < zend) ? (double)f.xp(zb)[ky * f.nx + kx] : 0.0;
-  const double Lglob = (double)res->p1.xmax - (double)res->p1.xmin;
+  const double Lglob = (double)res->p1g.xmax - (double)res->p1g.xmin;
 
   // in-plane offsets (a plane has < 2^31 elements; the launcher checks) and validity bits
   const int64_t gx = x0 + lane;
@@ -199,6 +199,8 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
       __syncthreads();
       const int64_t oz = zi - WZ + 1;
       const bool zok = (oz % p.sz) == 0;
+      const int64_t gxl = x0 + lane;
+      const bool xok = lane < TX && gxl <= f.nx - WX && (gxl % p.sx) == 0;
       // ---- (b) y-pass over WY rows, (c) x-pass with shuffles, mix ------------------------
       double h[4];
 #pragma unroll
@@ -230,17 +232,18 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
         const float mn = lane_window_ext<WX, false>(hmn);
         const float mx = lane_window_ext<WX, true>(hmx);
         const int64_t gy = y0 + oy;
-        const int64_t gxo = x0 + lane;
-        if (lane < TX && zok && gy <= f.ny - WY && (gy % p.sy) == 0 && gxo <= f.nx - WX && (gxo % p.sx) == 0) {
+        if (xok && zok && gy <= f.ny - WY && (gy % p.sy) == 0) {
           const double mua = S0 * invM, mue = S1 * invM;
           const double mux = K + mua, muy = mux + mue;
           const double sxy = S2 * invM - mua * (mua + mue);
           const double see = S3 * invM - mue * mue;
           double L = range_global ? Lglob : (double)mx - (double)mn;
-          if (L == 0) L = 1.0;
+          L = (L == 0.0) ? 1.0 : L;
           const double C1 = (0.01 * L) * (0.01 * L), C2 = (0.03 * L) * (0.03 * L);
           const double A = 2.0 * mux * muy + C1, B = 2.0 * sxy + C2;
-          const double ssim = (A * B) / ((A + mue * mue) * (B + see));
+          // A, B, A + mu_e^2, B + s_e^2 > 0 (C1, C2 > 0); |rel err of the reciprocal| <= 2u
+          const double ssim = (A * B) * fast_rcp((A + mue * mue) * (B + see));
+          const int64_t gxo = x0 + lane;
           ssum += ssim;
           scnt += 1.0;
           if (dbg) dbg[((oz / p.sz) * p.nwy + gy / p.sy) * p.nwx + gxo / p.sx] = ssim;
@@ -255,7 +258,7 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
   __syncthreads();
   block_reduce_slots<kSsimSlots>(rec, Sum{}, parts + (size_t)bid * kSsimSlots);
   if (!last_block_arrive(ticket)) return;
-  finish_slots<kSsimSlots>(parts, gridDim.x * gridDim.y * gridDim.z, Sum{}, res->ssim);
+  finish_slots<kSsimSlots>(parts, gridDim.x * gridDim.y * gridDim.z, Sum{}, res->rec.ssim);
   if (tid == 0) *ticket = 0;
 }
 

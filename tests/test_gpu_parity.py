@@ -206,3 +206,27 @@ def test_full_size_hurricane(czc, orc):
         o = [int(rng.integers(0, k)) for k in nw]
         ref = orc.ssim_window(xn, yn, o, [8, 8, 8])
         assert abs(d[tuple(o)] - ref) < 1e-6, (o, d[tuple(o)], ref)
+
+
+@pytest.mark.parametrize("cfg,dims,K,w", [("C2", (40, 70, 90), 2, 8), ("C1", (37, 13, 17), 3, 5),
+                                          ("C3", (44, 33, 40), 4, 6), ("C2q", (30, 50, 64), 3, 8)])
+def test_loopback_slabs(czc, orc, cfg, dims, K, w):
+    """The multi-GPU algorithm (slab ownership, halo buffers, rank-ordered combine) on one GPU:
+    K slabs must agree with the oracle on the whole field, and with the single-slab run."""
+    x, y = synth.make_pair(synth.config(cfg, dims=dims))
+    xn, yn = x.numpy(), y.numpy()
+    xd, yd = x.cuda(), y.cuda()
+    with czc.Assessor(ssim_window=w, ac_max_lag=10, loopback_slabs=K) as a:
+        g = a.assess(xd, yd)
+    with czc.Assessor(ssim_window=w, ac_max_lag=10) as a:
+        g1 = a.assess(xd, yd)
+    o = {}
+    o.update(orc.p1(xn, yn))
+    o.update(orc.deriv(xn, yn))
+    o["ac"], o["ac_count"] = orc.autocorr(xn, yn, 10)
+    o["ssim"], o["n_windows"] = orc.ssim(xn, yn, [w] * 3)
+    full_check(g, o)
+    for k in ("x_min", "x_max", "err_min", "err_max", "pwr_min", "pwr_max", "n_pwr", "n_windows",
+              "der1_maxabs", "lap_f_min", "grad_f_max"):
+        assert g[k] == g1[k], k
+    assert abs(g["ssim"] - g1["ssim"]) < 1e-12 and abs(g["mse"] - g1["mse"]) <= 1e-12 * g1["mse"]
