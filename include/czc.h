@@ -125,7 +125,8 @@ typedef struct czc_result {
   uint64_t n_ssim_exact;         /* windows whose fast-path error bound failed and were          */
                                  /* recomputed by the exact per-window path                      */
   /* ---- timing (cfg.timing) ------------------------------------------------------------------- */
-  float kernel_ms[4];            /* device ms on the context stream: P1, P2, P3, whole call      */
+  float kernel_ms[6];            /* device ms on the context stream: P1, P2 derivatives, P2      */
+                                 /* autocorrelation, P3 SSIM, whole call, (reserved = 0)         */
 } czc_result;
 
 typedef struct czc_ctx czc_ctx;

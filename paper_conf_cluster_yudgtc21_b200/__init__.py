@@ -67,7 +67,7 @@ class Result(ctypes.Structure):
                    ("ac", ctypes.c_double * (MAX_LAG + 1)), ("ac_count", ctypes.c_uint64 * (MAX_LAG + 1)),
                    ("ssim_window", ctypes.c_int32 * 3), ("ssim_step", ctypes.c_int32 * 3),
                    ("n_windows", ctypes.c_uint64), ("ssim", ctypes.c_double),
-                   ("n_ssim_exact", ctypes.c_uint64), ("kernel_ms", ctypes.c_float * 4)])
+                   ("n_ssim_exact", ctypes.c_uint64), ("kernel_ms", ctypes.c_float * 6)])
 
 
 def _load():

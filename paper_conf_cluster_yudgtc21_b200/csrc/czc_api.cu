@@ -50,7 +50,7 @@ struct czc_ctx {
   size_t parts_cap = 0;
   float* din[2] = {nullptr, nullptr};   // staging for czc_assess_host
   size_t din_cap = 0;
-  cudaEvent_t ev[5] = {};
+  cudaEvent_t ev[6] = {};   // P1 start, P1 end, deriv end, AC end, SSIM end, call end
   std::string last_error;
   // slab mode (NCCL ranks or loopback)
   CommState* comm = nullptr;
@@ -136,7 +136,7 @@ extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
     if ((e = cudaMallocHost(&ctx->hrec, rb)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMallocHost"); break; }
     if ((e = cudaMalloc(&ctx->tickets, TICKET_N * sizeof(unsigned int))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(tickets)"); break; }
     if ((e = cudaMemset(ctx->tickets, 0, TICKET_N * sizeof(unsigned int))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMemset"); break; }
-    for (int i = 0; i < 5 && st == CZC_OK; i++)
+    for (int i = 0; i < 6 && st == CZC_OK; i++)
       if ((e = cudaEventCreate(&ctx->ev[i])) != cudaSuccess) st = cuda_fail(ctx, e, "cudaEventCreate");
     if (st != CZC_OK) break;
     if (ctx->max_records > 1) {
@@ -172,7 +172,7 @@ extern "C" void czc_free(czc_ctx* ctx) {
   cudaFree(ctx->dgather);
   cudaFree(ctx->dstates);
   cudaFree(ctx->halo);
-  for (int i = 0; i < 5; i++)
+  for (int i = 0; i < 6; i++)
     if (ctx->ev[i]) cudaEventDestroy(ctx->ev[i]);
   if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
   delete ctx;
@@ -415,9 +415,10 @@ static czc_status run_p23(czc_ctx* ctx, const Plan& P, const Field3& F, const Ss
   if (st != CZC_OK) return st;
   if (P.run_deriv)
     CZC_CUDA(ctx, launch_deriv(F, kZchunkDeriv, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_DERIV, s));
+  if (ctx->cfg.timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
   if (P.run_ac)
     CZC_CUDA(ctx, launch_ac(F, P.T, 0, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_ACZ, s));
-  if (ctx->cfg.timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
+  if (ctx->cfg.timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));
   if (P.run_ssim)
     CZC_CUDA(ctx, launch_ssim(P.kind, P.W, F, sp, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_SSIM,
                               ctx->cfg.debug_wssim, s, nullptr));
@@ -434,10 +435,9 @@ static czc_status p1_local(czc_ctx* ctx, const Plan& P, const float* x, const fl
 
 static void finish_timing(czc_ctx* ctx, czc_result* out) {
   if (!ctx->cfg.timing) return;
-  cudaEventElapsedTime(&out->kernel_ms[0], ctx->ev[0], ctx->ev[1]);
-  cudaEventElapsedTime(&out->kernel_ms[1], ctx->ev[1], ctx->ev[2]);
-  cudaEventElapsedTime(&out->kernel_ms[2], ctx->ev[2], ctx->ev[3]);
-  cudaEventElapsedTime(&out->kernel_ms[3], ctx->ev[0], ctx->ev[4]);
+  for (int i = 0; i < 4; i++) cudaEventElapsedTime(&out->kernel_ms[i], ctx->ev[i], ctx->ev[i + 1]);
+  cudaEventElapsedTime(&out->kernel_ms[4], ctx->ev[0], ctx->ev[5]);
+  out->kernel_ms[5] = 0.f;
 }
 
 // Single GPU, whole field resident.
@@ -454,11 +454,10 @@ static czc_status assess_single(czc_ctx* ctx, const Plan& P, const float* x, con
   czc_status st = p1_local(ctx, P, x, y, F.nz * F.ny * F.nx);
   if (st != CZC_OK) return st;
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
-  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));   // re-recorded inside run_p23
   if ((st = run_p23(ctx, P, F, sp)) != CZC_OK) return st;
-  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));
-  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, &ctx->dres->rec, sizeof(Record), cudaMemcpyDeviceToHost, s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
+  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, &ctx->dres->rec, sizeof(Record), cudaMemcpyDeviceToHost, s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[5], s));
   CZC_CUDA(ctx, cudaStreamSynchronize(s));
   combine_and_finish(P, ctx->hrec, 1, mask, out);
   finish_timing(ctx, out);
@@ -532,7 +531,6 @@ static czc_status assess_loopback(czc_ctx* ctx, const Plan& P, const float* x, c
     CZC_CUDA(ctx, launch_p1_combine(dst, K, ctx->dres, s));
   }
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
-  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
   for (int k = 0; k < K; k++) {
     const int64_t z0 = tab[k].first, nzl = tab[k].second;
     const int64_t hlo = (P.run_deriv && z0 > 0) ? 1 : 0;
@@ -553,9 +551,9 @@ static czc_status assess_loopback(czc_ctx* ctx, const Plan& P, const float* x, c
     CZC_CUDA(ctx, cudaMemcpyAsync(drec[k].deriv, ctx->dres->rec.deriv,
                                   sizeof(Record) - offsetof(Record, deriv), cudaMemcpyDeviceToDevice, s));
   }
-  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));
-  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, drec, (size_t)K * sizeof(Record), cudaMemcpyDeviceToHost, s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
+  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, drec, (size_t)K * sizeof(Record), cudaMemcpyDeviceToHost, s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[5], s));
   CZC_CUDA(ctx, cudaStreamSynchronize(s));
   combine_and_finish(P, ctx->hrec, K, mask, out);
   finish_timing(ctx, out);
@@ -620,13 +618,12 @@ static czc_status assess_ranks(czc_ctx* ctx, const Plan& P, const float* x, cons
     CZC_CUDA(ctx, launch_p1_combine((const P1State*)ctx->dstates, nranks, ctx->dres, s));
   }
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
-  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
   if ((st = run_p23(ctx, P, F, sp)) != CZC_OK) return st;
-  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
   // second small allgather: every rank's record, combined in rank order on the host
   if (!comm_allgather(ctx->comm, &ctx->dres->rec, ctx->dgather, sizeof(Record), s, &ctx->last_error)) return CZC_ERR_COMM;
   CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, ctx->dgather, (size_t)nranks * sizeof(Record), cudaMemcpyDeviceToHost, s));
-  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[5], s));
   CZC_CUDA(ctx, cudaStreamSynchronize(s));
   combine_and_finish(P, ctx->hrec, nranks, mask, out);
   finish_timing(ctx, out);

@@ -68,6 +68,11 @@ def to_us(v, unit):
 def main():
     args = sys.argv[1:]
     launches = None
+    dominant = None
+    if "--dominant" in args:                 # --dominant PATTERN KERNEL_SUBSTRING
+        i = args.index("--dominant")
+        dominant = (args[i + 1], args[i + 2])
+        args = args[:i] + args[i + 3:]
     if "--launches" in args:
         i = args.index("--launches")
         launches = args[i + 1]
@@ -108,6 +113,18 @@ def main():
                "| kernel | launches | mean us | share of step |", "|---|---|---|---|"]
         for k, s in sorted(summary["launches"].items(), key=lambda kv: -kv[1]["share"]):
             md.append(f"| {k[:60]} | {s['count']} | {s['mean_us']:.1f} | {100 * s['share']:.1f}% |")
+    if dominant:
+        pat, sub = dominant
+        ks = [k for k in summary["kernels"] if sub in k["kernel"]]
+        if ks:
+            k = ks[0]
+            import os
+            out = {"kernel_pattern": pat, "kernel": k["kernel"], "source": reps,
+                   "dram_bytes_per_launch": k["dram_read_bytes"] + k["dram_write_bytes"],
+                   "dram_read_bytes": k["dram_read_bytes"], "dram_write_bytes": k["dram_write_bytes"],
+                   "duration_us_cold": k["duration_us"]}
+            with open(os.path.join(os.path.dirname(prefix) or ".", "ncu_dominant.json"), "w") as f:
+                json.dump(out, f, indent=1)
     with open(prefix + ".json", "w") as f:
         json.dump(summary, f, indent=1)
     with open(prefix + ".md", "w") as f:

@@ -22,7 +22,7 @@ with czc.Assessor(ndim=x.dim(), ssim_window=w, timing=True) as a:
             flush.zero_()
             r = a.assess(xd, yd, mask)
             ts.append(r["kernel_ms"])
-        best = [min(t[i] for t in ts) for i in range(4)]
-        tot = sum(best[:3])
-        print(f"{cfg} {name:6s} p1={best[0]:.4f}ms p2={best[1]:.4f}ms p3={best[2]:.4f}ms call={best[3]:.4f}ms "
-              f"-> {nbytes/ (tot*1e-3) / 1e9:.1f} GB/s (kernels)")
+        best = [min(t[i] for t in ts) for i in range(5)]
+        tot = sum(best[:4])
+        print(f"{cfg} {name:6s} p1={best[0]:.4f} deriv={best[1]:.4f} ac={best[2]:.4f} ssim={best[3]:.4f} "
+              f"call={best[4]:.4f} ms -> {nbytes/ (tot*1e-3) / 1e9:.1f} GB/s (kernels)")
