@@ -75,7 +75,8 @@ typedef struct czc_config {
   int ac_max_lag;                /* autocorrelation lags 1..ac_max_lag (<= CZC_MAX_LAG); 0 -> 10 */
   int timing;                    /* 1: record per-pattern device time into czc_result.kernel_ms  */
   int rank, nranks;              /* slab mode over nranks GPUs; nranks <= 1: single GPU          */
-  const void* nccl_uid;          /* 128-byte ncclUniqueId (from rank 0), required if nranks > 1 */
+  const void* nccl_uid;          /* 128-byte ncclUniqueId (from rank 0), required if nranks > 1; */
+                                 /* given with nranks = 1 it runs the NCCL slab path on 1 rank  */
   double* debug_wssim;           /* optional DEVICE buffer of n_windows doubles: local SSIM of   */
                                  /* every window in C order of the window-origin grid (Alg. 3    */
                                  /* L310 "wssim"); NULL = not written (not on the timed path)    */

@@ -95,7 +95,8 @@ static czc_status validate_config(const czc_config& c) {
   for (int i = 0; i < 3; i++)
     if (c.ssim_window[i] < 0 || c.ssim_step[i] < 0) return CZC_ERR_INVALID;
   if (c.nranks > 1 && (c.rank < 0 || c.rank >= c.nranks || !c.nccl_uid)) return CZC_ERR_INVALID;
-  if (c.loopback_slabs < 0 || (c.loopback_slabs > 1 && c.nranks > 1)) return CZC_ERR_INVALID;
+  if (c.nccl_uid && (c.nranks < 1 || c.rank < 0 || c.rank >= c.nranks)) return CZC_ERR_INVALID;
+  if (c.loopback_slabs < 0 || (c.loopback_slabs > 1 && (c.nranks > 1 || c.nccl_uid))) return CZC_ERR_INVALID;
   return CZC_OK;
 }
 
@@ -108,12 +109,13 @@ extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
   else c.device = -1;
   czc_status st = validate_config(c);
   if (st != CZC_OK) return st;
-  if (c.nranks > 1 && !comm_available()) return CZC_ERR_UNSUPPORTED;
+  const bool slab_mode = c.nranks > 1 || c.nccl_uid != nullptr;   // NCCL comm (also valid with 1 rank)
+  if (slab_mode && !comm_available()) return CZC_ERR_UNSUPPORTED;
 
   czc_ctx* ctx = new (std::nothrow) czc_ctx();
   if (!ctx) return CZC_ERR_NOMEM;
   ctx->cfg = c;
-  ctx->max_records = std::max(1, std::max(c.nranks, c.loopback_slabs));
+  ctx->max_records = std::max(2, std::max(c.nranks, c.loopback_slabs));
   do {
     int dev = c.device;
     if (dev < 0) {
@@ -139,13 +141,13 @@ extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
     for (int i = 0; i < 6 && st == CZC_OK; i++)
       if ((e = cudaEventCreate(&ctx->ev[i])) != cudaSuccess) st = cuda_fail(ctx, e, "cudaEventCreate");
     if (st != CZC_OK) break;
-    if (ctx->max_records > 1) {
+    {
       if ((e = cudaMalloc(&ctx->dgather_in, 64)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(gather)"); break; }
       if ((e = cudaMalloc(&ctx->dgather, rb)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(gather)"); break; }
       if ((e = cudaMalloc(&ctx->dstates, (size_t)ctx->max_records * sizeof(P1State))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(states)"); break; }
     }
-    if (c.nranks > 1) {
-      ctx->comm = comm_create(c.nccl_uid, c.rank, c.nranks, &ctx->last_error);
+    if (slab_mode) {
+      ctx->comm = comm_create(c.nccl_uid, c.rank, std::max(1, c.nranks), &ctx->last_error);
       if (!ctx->comm) { st = CZC_ERR_COMM; break; }
     }
   } while (0);

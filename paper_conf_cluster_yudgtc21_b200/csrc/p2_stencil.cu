@@ -197,14 +197,14 @@ __device__ __forceinline__ void ac_finish(double (&acc)[TM], double* parts, doub
 }
 
 // Walk of one line.  Positions [lo, end) are visited; points p in [lo, hi) own their products.
-// `next` returns the (x, y) sample at the position of a load cursor that runs QD = 2 TM positions
+// `next` returns the (x, y) sample at the position of a load cursor that runs QD positions
 // ahead of the walk: QD loads stay in flight in a register queue whose slot u (of the QD-unrolled
 // loop) holds position i0 + u, so both the queue and the ring (QD is a multiple of TM) rotate
 // statically.
-template <int TM, typename Next>
+template <int TM, int QD, typename Next>
 __device__ __forceinline__ void walk_line(Next next, int64_t lo, int64_t hi, int64_t end, double mu,
                                           bool own, double (&ring)[TM], double (&acc)[TM]) {
-  constexpr int QD = 2 * TM;
+  static_assert(QD % TM == 0, "queue depth must be a multiple of the ring length");
   float qx[QD], qy[QD];
 #pragma unroll
   for (int u = 0; u < QD; u++) {
@@ -246,7 +246,7 @@ ac_zwalk(Field3 s, int T, int zchunk, double* __restrict__ parts, DevResults* __
   for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
   PlaneCursor cur;
   if (own && lo < end) cur.init(s, lo, col);
-  walk_line<TM>([&]() {                 // read the cursor's plane, then step it (never read past end)
+  walk_line<TM, 2 * TM>([&]() {         // read the cursor's plane, then step it (never read past end)
     const float2 v = make_float2(__ldg(cur.x), __ldg(cur.y));
     cur.advance(s, col);
     return v;
@@ -281,7 +281,7 @@ ac_ywalk(Field3 s, int T, int ychunk, double* __restrict__ parts, DevResults* __
   for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
   const float* px = own ? X + lo * nx : nullptr;
   const float* py = own ? Y + lo * nx : nullptr;
-  walk_line<TM>([&]() {
+  walk_line<TM, TM>([&]() {
     const float2 v = make_float2(__ldg(px), __ldg(py));
     px += nx; py += nx;
     return v;
@@ -442,7 +442,7 @@ struct AcGrids {
 static AcGrids ac_grids(const Field3& s) {
   AcGrids g{};
   const int64_t nzo = s.zown1 - s.zown0;
-  g.zc = 50; g.yc = 125; g.xc = 128;   // xc % 4 == 0 for the vector x-walk
+  g.zc = 50; g.yc = 50; g.xc = 128;    // xc % 4 == 0 for the vector x-walk
   g.rz = s.nz > 1; g.ry = s.ny > 1; g.rx = s.nx > 1;
   g.z = dim3((unsigned)cdiv(s.nx, kTX), (unsigned)cdiv(s.ny, kTY), (unsigned)cdiv(nzo, g.zc));
   g.y = dim3((unsigned)cdiv(s.nx, 256), (unsigned)nzo, (unsigned)cdiv(s.ny, g.yc));

@@ -203,6 +203,14 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
       const bool xok = lane < TX && gxl <= f.nx - WX && (gxl % p.sx) == 0;
       // ---- (b) y-pass over WY rows, (c) x-pass with shuffles, mix ------------------------
       double h[4];
+      // y-window min/max: rows [warp G, warp G + G + WY - 1) of this lane's column; the WY - G + 1
+      // rows shared by all G windows of the warp are reduced once
+      float cmn = Zm[(warp * G + G - 1) * 32 + lane], cmx = Zm[ZS + (warp * G + G - 1) * 32 + lane];
+#pragma unroll
+      for (int i = G; i < WY; i++) {
+        cmn = fminf(cmn, Zm[(warp * G + i) * 32 + lane]);
+        cmx = fmaxf(cmx, Zm[ZS + (warp * G + i) * 32 + lane]);
+      }
 #pragma unroll
       for (int g = 0; g < G; g++) {
         const int oy = warp * G + g;
@@ -219,11 +227,16 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
           for (int m = 0; m < 4; m++)
             h[m] += Zd[m * ZS + (oy + WY - 1) * 32 + lane] - Zd[m * ZS + (oy - 1) * 32 + lane];
         }
-        float hmn = Zm[oy * 32 + lane], hmx = Zm[ZS + oy * 32 + lane];
+        float hmn = cmn, hmx = cmx;                      // rows [G-1, WY) relative to warp*G
 #pragma unroll
-        for (int i = 1; i < WY; i++) {
-          hmn = fminf(hmn, Zm[(oy + i) * 32 + lane]);
-          hmx = fmaxf(hmx, Zm[ZS + (oy + i) * 32 + lane]);
+        for (int i = g; i < G - 1; i++) {                // rows oy .. warp*G + G - 2
+          hmn = fminf(hmn, Zm[(warp * G + i) * 32 + lane]);
+          hmx = fmaxf(hmx, Zm[ZS + (warp * G + i) * 32 + lane]);
+        }
+#pragma unroll
+        for (int i = WY; i < WY + g; i++) {              // rows warp*G + WY .. oy + WY - 1
+          hmn = fminf(hmn, Zm[(warp * G + i) * 32 + lane]);
+          hmx = fmaxf(hmx, Zm[ZS + (warp * G + i) * 32 + lane]);
         }
         const double S0 = lane_window_sum<WX>(h[0]);
         const double S1 = lane_window_sum<WX>(h[1]);

@@ -230,3 +230,23 @@ def test_loopback_slabs(czc, orc, cfg, dims, K, w):
               "der1_maxabs", "lap_f_min", "grad_f_max"):
         assert g[k] == g1[k], k
     assert abs(g["ssim"] - g1["ssim"]) < 1e-12 and abs(g["mse"] - g1["mse"]) <= 1e-12 * g1["mse"]
+
+
+def test_nccl_slab_path_single_rank(czc):
+    """The NCCL slab path (slab table allgather, halo group, P1 allgather + device merge, record
+    allgather + host combine) on a 1-rank communicator must reproduce single-GPU mode."""
+    import bench
+    if not czc.lib.czc_has_nccl():
+        pytest.skip("built without NCCL")
+    x, y = synth.make_pair(synth.config("C2", dims=(30, 40, 52)))
+    xd, yd = x.cuda(), y.cuda()
+    with czc.Assessor(ssim_window=8) as a:
+        g1 = a.assess(xd, yd)
+    uid = bench.czc_nccl_uid()
+    with czc.Assessor(ssim_window=8, rank=0, nranks=1, nccl_uid=uid) as a:
+        g = a.assess(xd, yd, dims=xd.shape, z0=0)
+    for k in ("x_min", "x_max", "err_min", "err_max", "pwr_max", "n_pwr", "n_windows", "der1_maxabs"):
+        assert g[k] == g1[k], k
+    for k in ("mse", "psnr", "pearson", "ssim", "der1_mae", "lap_mse"):
+        assert abs(g[k] - g1[k]) <= 1e-12 * max(1.0, abs(g1[k])), k
+    assert np.allclose(g["ac"], g1["ac"], rtol=0, atol=1e-13)
