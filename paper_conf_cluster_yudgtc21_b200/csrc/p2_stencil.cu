@@ -224,6 +224,130 @@ __device__ __forceinline__ void walk_line(Next next, int64_t lo, int64_t hi, int
   }
 }
 
+// ---- TMA line walks (rows 16-byte aligned: nx % 4 == 0 and aligned segment bases) ------------
+// A block's 256 threads own 256 consecutive x of a line family (a row y for the z-walk, a plane z
+// for the y-walk) and walk positions i in [lo, end).  Thread 0 streams the contiguous row segment
+// of each position (<= 1 KB per field) into a ring of S = 2 TM shared-memory slots with one bulk
+// copy per field, completing on the slot's mbarrier; after every TM positions the block
+// synchronises once and the consumed half of the ring is refilled S positions ahead.  Threads past
+// the row end read stale slot data; their products are discarded by walk_mask (lim = 0).
+constexpr int kWalkThreads = 256;
+template <int TM>
+struct BulkWalkSmem {
+  static constexpr int S = 2 * TM;
+  float x[S][kWalkThreads];
+  float y[S][kWalkThreads];
+  uint64_t bar[S];
+};
+
+// RowPtr(i) -> (const float* xrow, const float* yrow) for position i (already offset to x0).
+// Positions are tracked relative to lo in 32 bits.  Lane v < S of warp 0 issues slot v's copies
+// (after the barrier that frees the slot), so the refill costs one bulk copy pair per lane.
+template <int TM, typename RowPtr>
+__device__ __forceinline__ void bulk_walk(BulkWalkSmem<TM>& sm, RowPtr row_ptr, uint32_t bytes, int64_t lo,
+                                          int64_t hi, int64_t end, double mu,
+                                          double (&ring)[TM], double (&acc)[TM]) {
+  constexpr int S = 2 * TM;
+  const int tid = threadIdx.x;
+  const int jend = (int)(end - lo), jhi = (int)(hi - lo);
+  if (tid == 0) {
+#pragma unroll
+    for (int v = 0; v < S; v++) mbar_init(&sm.bar[v], 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  auto issue = [&](int slot, int j) {
+    const float* xr;
+    const float* yr;
+    row_ptr(lo + j, xr, yr);
+    mbar_expect_tx(&sm.bar[slot], 2 * bytes);
+    bulk_g2s(sm.x[slot], xr, bytes, &sm.bar[slot]);
+    bulk_g2s(sm.y[slot], yr, bytes, &sm.bar[slot]);
+  };
+  if (tid < S && tid < jend) issue(tid, tid);
+  uint32_t parity = 0;
+  for (int j0 = 0; j0 < jend; j0 += S) {
+#pragma unroll
+    for (int u = 0; u < S; u++) {
+      const int j = j0 + u;
+      if (j < jend) {                                  // block-uniform
+        mbar_wait(&sm.bar[u], parity);
+        const double eps = ((double)sm.y[u][tid] - (double)sm.x[u][tid]) - mu;
+        walk_step<TM>(ring, acc, eps, j < jhi, u % TM);
+      }
+      if (u == TM - 1 || u == S - 1) {                 // half of the ring consumed
+        __syncthreads();
+        const int v = u - TM + 1 + tid;                // lanes 0..TM-1 refill slots u-TM+1..u
+        if (tid < TM && j0 + v + S < jend) issue(v, j0 + v + S);
+      }
+    }
+    parity ^= 1u;
+  }
+}
+
+// z-walk, TMA: block = 256 consecutive x of row y; grid (x tiles, ny, z chunks).
+template <int TM>
+__global__ void __launch_bounds__(kWalkThreads, 3)
+ac_zwalk_tma(Field3 s, int T, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+             unsigned int* __restrict__ ticket) {
+  extern __shared__ __align__(128) unsigned char walk_smem[];
+  BulkWalkSmem<TM>& sm = *reinterpret_cast<BulkWalkSmem<TM>*>(walk_smem);
+  const int64_t x0 = (int64_t)blockIdx.x * kWalkThreads, gy = blockIdx.y;
+  const int64_t gx = x0 + threadIdx.x;
+  const double mu = res->p1g.me;
+  const bool own = gx < s.nx;
+  int64_t m = T;
+  if (s.ny > 1 && s.ny - 1 - gy < m) m = s.ny - 1 - gy;
+  if (s.nx > 1 && s.nx - 1 - gx < m) m = s.nx - 1 - gx;
+  const int64_t lo = s.zown0 + (int64_t)blockIdx.z * zchunk;
+  int64_t hi = lo + zchunk;
+  if (hi > s.zown1) hi = s.zown1;
+  int64_t end = hi + T;
+  if (end > s.nz) end = s.nz;
+  const int64_t ncols = (s.nx - x0) < kWalkThreads ? (s.nx - x0) : kWalkThreads;
+  const int64_t off = gy * s.nx + x0;
+  double ring[TM], acc[TM];
+#pragma unroll
+  for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
+  bulk_walk<TM>(sm, [&](int64_t z, const float*& xr, const float*& yr) { xr = s.xp(z) + off; yr = s.yp(z) + off; },
+                (uint32_t)(ncols * 4), lo, hi, end, mu, ring, acc);
+  walk_mask<TM>(acc, own ? (int)m : 0);
+  ac_finish<TM>(acc, parts, res->rec.ac[0], ticket);
+}
+
+// y-walk, TMA: block = 256 consecutive x of plane z; grid (x tiles, owned planes, y chunks).
+template <int TM>
+__global__ void __launch_bounds__(kWalkThreads, 3)
+ac_ywalk_tma(Field3 s, int T, int ychunk, double* __restrict__ parts, DevResults* __restrict__ res,
+             unsigned int* __restrict__ ticket) {
+  extern __shared__ __align__(128) unsigned char walk_smem[];
+  BulkWalkSmem<TM>& sm = *reinterpret_cast<BulkWalkSmem<TM>*>(walk_smem);
+  const int64_t x0 = (int64_t)blockIdx.x * kWalkThreads;
+  const int64_t gx = x0 + threadIdx.x;
+  const int64_t z = s.zown0 + (int64_t)blockIdx.y;
+  const double mu = res->p1g.me;
+  const bool own = gx < s.nx;
+  int64_t m = T;
+  if (s.nz > 1 && s.nz - 1 - z < m) m = s.nz - 1 - z;
+  if (s.nx > 1 && s.nx - 1 - gx < m) m = s.nx - 1 - gx;
+  const int64_t lo = (int64_t)blockIdx.z * ychunk;
+  int64_t hi = lo + ychunk;
+  if (hi > s.ny) hi = s.ny;
+  int64_t end = hi + T;
+  if (end > s.ny) end = s.ny;
+  const int64_t ncols = (s.nx - x0) < kWalkThreads ? (s.nx - x0) : kWalkThreads;
+  double ring[TM], acc[TM];
+#pragma unroll
+  for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
+  bulk_walk<TM>(sm, [&](int64_t y, const float*& xr, const float*& yr) {
+                  xr = s.xp(z) + y * s.nx + x0;
+                  yr = s.yp(z) + y * s.nx + x0;
+                },
+                (uint32_t)(ncols * 4), lo, hi, end, mu, ring, acc);
+  walk_mask<TM>(acc, own ? (int)m : 0);
+  ac_finish<TM>(acc, parts, res->rec.ac[1], ticket);
+}
+
 // z-walk: thread <-> column (y, x); block 32 x 8 columns; grid.z chunks of owned planes.
 template <int TM>
 __global__ void __launch_bounds__(256)
@@ -435,7 +559,7 @@ cudaError_t launch_deriv(const Field3& s, int zchunk, double* parts, DevResults*
 // Autocorrelation: one launch per active walk axis, each with its own partial-buffer slice and
 // ticket; the three records are summed at the finish.
 struct AcGrids {
-  dim3 z, y, x, xvec;
+  dim3 z, y, x, xvec, zt, yt;
   bool rz, ry, rx;
   int zc, yc, xc;
 };
@@ -448,29 +572,40 @@ static AcGrids ac_grids(const Field3& s) {
   g.y = dim3((unsigned)cdiv(s.nx, 256), (unsigned)nzo, (unsigned)cdiv(s.ny, g.yc));
   g.x = dim3((unsigned)cdiv(nzo * s.ny, kXWarps * 32), (unsigned)cdiv(s.nx, g.xc), 1);
   g.xvec = dim3((unsigned)cdiv(nzo * s.ny, 256), (unsigned)cdiv(s.nx, g.xc), 1);
+  g.zt = dim3((unsigned)cdiv(s.nx, kWalkThreads), (unsigned)s.ny, (unsigned)cdiv(nzo, g.zc));
+  g.yt = dim3((unsigned)cdiv(s.nx, kWalkThreads), (unsigned)nzo, (unsigned)cdiv(s.ny, g.yc));
   return g;
 }
 int64_t ac_blocks(const Field3& s, int) {
   const AcGrids g = ac_grids(s);
   auto n = [](dim3 d) { return (int64_t)d.x * d.y * d.z; };
-  return n(g.z) + n(g.y) + (n(g.x) > n(g.xvec) ? n(g.x) : n(g.xvec));
+  auto mx = [](int64_t a, int64_t b) { return a > b ? a : b; };
+  return mx(n(g.z), n(g.zt)) + mx(n(g.y), n(g.yt)) + mx(n(g.x), n(g.xvec));
 }
 
 template <int TM>
 static cudaError_t launch_ac_t(const Field3& s, int T, double* parts, DevResults* res,
                                unsigned int* tickets, cudaStream_t st) {
   const AcGrids g = ac_grids(s);
-  double* pz = parts;
-  double* py = pz + (size_t)g.z.x * g.z.y * g.z.z * kAcSlots;
-  double* px = py + (size_t)g.y.x * g.y.y * g.y.z * kAcSlots;
-  cudaError_t e = cudaMemsetAsync(res->rec.ac, 0, sizeof(res->rec.ac), st);
-  if (e != cudaSuccess) return e;
-  if (g.rz) ac_zwalk<TM><<<g.z, dim3(kTX, kTY), 0, st>>>(s, T, g.zc, pz, res, tickets + 0);
-  if (g.ry) ac_ywalk<TM><<<g.y, 256, 0, st>>>(s, T, g.yc, py, res, tickets + 1);
-  // vector x-walk when every row start is 16-byte aligned (nx % 4 == 0, aligned segments)
+  auto n = [](dim3 d) { return (size_t)d.x * d.y * d.z; };
+  // rows 16-byte aligned (nx % 4 == 0, aligned segments): TMA bulk-copy walks and the vector x-walk
   bool vec = (s.nx % 4) == 0;
   for (int k = 0; k < s.nseg; k++)
     vec = vec && (reinterpret_cast<uintptr_t>(s.xs[k]) % 16) == 0 && (reinterpret_cast<uintptr_t>(s.ys[k]) % 16) == 0;
+  double* pz = parts;
+  double* py = pz + (vec ? n(g.zt) : n(g.z)) * kAcSlots;
+  double* px = py + (vec ? n(g.yt) : n(g.y)) * kAcSlots;
+  cudaError_t e = cudaMemsetAsync(res->rec.ac, 0, sizeof(res->rec.ac), st);
+  if (e != cudaSuccess) return e;
+  constexpr int wsm = (int)sizeof(BulkWalkSmem<TM>);
+  if (vec) {
+    if ((e = cudaFuncSetAttribute(ac_zwalk_tma<TM>, cudaFuncAttributeMaxDynamicSharedMemorySize, wsm)) != cudaSuccess) return e;
+    if ((e = cudaFuncSetAttribute(ac_ywalk_tma<TM>, cudaFuncAttributeMaxDynamicSharedMemorySize, wsm)) != cudaSuccess) return e;
+  }
+  if (g.rz && vec) ac_zwalk_tma<TM><<<g.zt, kWalkThreads, wsm, st>>>(s, T, g.zc, pz, res, tickets + 0);
+  else if (g.rz) ac_zwalk<TM><<<g.z, dim3(kTX, kTY), 0, st>>>(s, T, g.zc, pz, res, tickets + 0);
+  if (g.ry && vec) ac_ywalk_tma<TM><<<g.yt, kWalkThreads, wsm, st>>>(s, T, g.yc, py, res, tickets + 1);
+  else if (g.ry) ac_ywalk<TM><<<g.y, 256, 0, st>>>(s, T, g.yc, py, res, tickets + 1);
   if (g.rx && vec) ac_xwalk_vec<TM><<<g.xvec, 256, 0, st>>>(s, T, g.xc, px, res, tickets + 2);
   else if (g.rx) ac_xwalk_smem<TM><<<g.x, kXWarps * 32, 0, st>>>(s, T, g.xc, px, res, tickets + 2);
   return cudaGetLastError();
