@@ -36,6 +36,8 @@ cudaError_t launch_ssim(int kind, int W, const Field3& f, const SsimParams& p,
 
 using namespace czc;
 
+static constexpr int kMaxHostChunks = 16;   // z-chunks of the pipelined czc_assess_host
+
 struct czc_ctx {
   czc_config cfg;
   int device = 0;
@@ -60,6 +62,9 @@ struct czc_ctx {
   float* halo = nullptr;           // device halo planes (x lo, y lo, x hi, y hi)
   size_t halo_cap = 0;
   int max_records = 1;
+  // pipelined host path
+  cudaStream_t copy_stream[2] = {nullptr, nullptr};   // [0]: H2D chunks (x then y); [1] unused
+  cudaEvent_t copy_ev[2][kMaxHostChunks] = {};
 };
 
 static const char* kStatusStr[] = {"ok", "invalid argument", "invalid shape", "unsupported dtype",
@@ -115,7 +120,7 @@ extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
   czc_ctx* ctx = new (std::nothrow) czc_ctx();
   if (!ctx) return CZC_ERR_NOMEM;
   ctx->cfg = c;
-  ctx->max_records = std::max(2, std::max(c.nranks, c.loopback_slabs));
+  ctx->max_records = std::max(kMaxHostChunks, std::max(c.nranks, c.loopback_slabs));
   do {
     int dev = c.device;
     if (dev < 0) {
@@ -176,6 +181,11 @@ extern "C" void czc_free(czc_ctx* ctx) {
   cudaFree(ctx->halo);
   for (int i = 0; i < 6; i++)
     if (ctx->ev[i]) cudaEventDestroy(ctx->ev[i]);
+  for (int c = 0; c < 2; c++) {
+    for (int i = 0; i < kMaxHostChunks; i++)
+      if (ctx->copy_ev[c][i]) cudaEventDestroy(ctx->copy_ev[c][i]);
+    if (ctx->copy_stream[c]) cudaStreamDestroy(ctx->copy_stream[c]);
+  }
   if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
   delete ctx;
 }
@@ -671,6 +681,97 @@ extern "C" czc_status czc_assess(czc_ctx* ctx, const void* orig, const void* rec
   return st;
 }
 
+// Pipelined host path (single GPU, 3-D field): the pair is copied host->device in K z-chunks on a
+// copy stream while P1, the derivatives and SSIM of chunk k run on the compute stream as soon as
+// chunk k and the halo planes above it have arrived (records per chunk, owned ranges as in slab
+// mode); the autocorrelation, which needs the global mean / variance of the error, runs once the
+// whole field is resident.  Same combine as slab mode.
+static czc_status assess_host_pipelined(czc_ctx* ctx, const Plan& P, const float* hx, const float* hy,
+                                        czc_result* out, uint64_t mask, int K) {
+  const cudaStream_t s = ctx->stream;
+  const bool timing = ctx->cfg.timing != 0;
+  const int64_t nz = P.g3[0], plane = P.g3[1] * P.g3[2];
+  const size_t pb = (size_t)plane * sizeof(float);
+  float* x = ctx->din[0];
+  float* y = ctx->din[1];
+  if (!ctx->copy_stream[0]) {
+    for (int c = 0; c < 2; c++) {
+      CZC_CUDA(ctx, cudaStreamCreateWithFlags(&ctx->copy_stream[c], cudaStreamNonBlocking));
+      for (int i = 0; i < kMaxHostChunks; i++)
+        CZC_CUDA(ctx, cudaEventCreateWithFlags(&ctx->copy_ev[c][i], cudaEventDisableTiming));
+    }
+  }
+  std::vector<int64_t> b(K + 1);
+  for (int k = 0; k <= K; k++) b[k] = nz * k / K;
+  const int64_t H = halo_depth(P);
+  // the copy streams start after everything already queued on the compute stream (which may
+  // still read the device buffers of the previous call)
+  CZC_CUDA(ctx, cudaEventRecord(ctx->copy_ev[0][0], s));
+  CZC_CUDA(ctx, cudaStreamWaitEvent(ctx->copy_stream[0], ctx->copy_ev[0][0], 0));
+  for (int k = 0; k < K; k++) {
+    const size_t bytes = (size_t)(b[k + 1] - b[k]) * pb;
+    CZC_CUDA(ctx, cudaMemcpyAsync(x + b[k] * plane, hx + b[k] * plane, bytes, cudaMemcpyHostToDevice, ctx->copy_stream[0]));
+    CZC_CUDA(ctx, cudaMemcpyAsync(y + b[k] * plane, hy + b[k] * plane, bytes, cudaMemcpyHostToDevice, ctx->copy_stream[0]));
+    CZC_CUDA(ctx, cudaEventRecord(ctx->copy_ev[0][k], ctx->copy_stream[0]));
+  }
+  // index of the last chunk that must be resident before chunk k's stencils / windows can run
+  auto ready_for = [&](int k) {
+    int j = k;
+    while (j + 1 < K && b[j + 1] < std::min(nz, b[k + 1] + H)) j++;
+    return j;
+  };
+  Field3 F{};
+  F.nz = nz; F.ny = P.g3[1]; F.nx = P.g3[2];
+  F.nseg = 1; F.xs[0] = x; F.ys[0] = y; F.zs[0] = 0; F.zs[1] = nz;
+  const SsimParams sp = ssim_params(P, ctx->cfg);
+  Record* drec = (Record*)ctx->dgather;
+  P1State* dst = (P1State*)ctx->dstates;
+  CZC_CUDA(ctx, cudaMemsetAsync(drec, 0, (size_t)K * sizeof(Record), s));
+  Plan P23 = P;                                       // per chunk: derivatives + SSIM only
+  P23.run_ac = false;
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
+  int waited = -1;
+  for (int k = 0; k < K; k++) {
+    const int need = (P.run_deriv || P.run_ssim) ? ready_for(k) : k;
+    for (int j = waited + 1; j <= need; j++) CZC_CUDA(ctx, cudaStreamWaitEvent(s, ctx->copy_ev[0][j], 0));
+    waited = std::max(waited, need);
+    if (P.run_p1) {
+      czc_status st = p1_local(ctx, P, x + b[k] * plane, y + b[k] * plane, (b[k + 1] - b[k]) * plane);
+      if (st != CZC_OK) return st;
+      CZC_CUDA(ctx, cudaMemcpyAsync(dst + k, &ctx->dres->rec.p1, sizeof(P1State), cudaMemcpyDeviceToDevice, s));
+      CZC_CUDA(ctx, cudaMemcpyAsync(&drec[k].p1, &ctx->dres->rec.p1, sizeof(P1State), cudaMemcpyDeviceToDevice, s));
+    }
+    if (P.run_deriv || P.run_ssim) {
+      F.zown0 = b[k];
+      F.zown1 = b[k + 1];
+      czc_status st = run_p23(ctx, P23, F, sp);
+      if (st != CZC_OK) return st;
+      CZC_CUDA(ctx, cudaMemcpyAsync(drec[k].deriv, ctx->dres->rec.deriv, sizeof(drec[k].deriv), cudaMemcpyDeviceToDevice, s));
+      CZC_CUDA(ctx, cudaMemcpyAsync(drec[k].ssim, ctx->dres->rec.ssim, sizeof(drec[k].ssim), cudaMemcpyDeviceToDevice, s));
+    }
+  }
+  for (int j = waited + 1; j < K; j++) CZC_CUDA(ctx, cudaStreamWaitEvent(s, ctx->copy_ev[0][j], 0));
+  if (P.run_p1) CZC_CUDA(ctx, launch_p1_combine(dst, K, ctx->dres, s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
+  if (P.run_ac) {
+    F.zown0 = 0;
+    F.zown1 = nz;
+    czc_status st = ensure_scratch(ctx, P, F, sp);
+    if (st != CZC_OK) return st;
+    CZC_CUDA(ctx, launch_ac(F, P.T, 0, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_ACZ, s));
+    CZC_CUDA(ctx, cudaMemcpyAsync(drec[0].ac, ctx->dres->rec.ac, sizeof(drec[0].ac), cudaMemcpyDeviceToDevice, s));
+  }
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
+  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, drec, (size_t)K * sizeof(Record), cudaMemcpyDeviceToHost, s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[5], s));
+  CZC_CUDA(ctx, cudaStreamSynchronize(s));
+  combine_and_finish(P, ctx->hrec, K, mask, out);
+  finish_timing(ctx, out);
+  return CZC_OK;
+}
+
 extern "C" czc_status czc_assess_host(czc_ctx* ctx, const void* orig, const void* recon, const czc_shape* shape,
                                       czc_dtype dtype, uint64_t metric_mask, czc_result* out) {
   czc_status st = check_common(ctx, orig, recon, shape, dtype, out);
@@ -691,6 +792,21 @@ extern "C" czc_status czc_assess_host(czc_ctx* ctx, const void* orig, const void
     CZC_CUDA(ctx, cudaMalloc(&ctx->din[0], bytes));
     CZC_CUDA(ctx, cudaMalloc(&ctx->din[1], bytes));
     ctx->din_cap = bytes;
+  }
+  // pipelined path: single GPU, 3-D field, chunks at least as thick as the halo depth
+  Plan P;
+  std::string why;
+  const bool plain = !ctx->comm && ctx->cfg.loopback_slabs <= 1 &&
+                     make_plan(ctx->cfg, shape->ndim, shape->dims, metric_mask, P, why) == CZC_OK && P.D == 3 &&
+                     (shape->nz_local == 0 || shape->nz_local == shape->dims[0]);
+  if (plain) {
+    const int64_t H = std::max<int64_t>(halo_depth(P), 1);
+    const int K = (int)std::min<int64_t>(std::min<int64_t>(8, kMaxHostChunks), P.g3[0] / H);
+    if (K >= 2) {
+      st = assess_host_pipelined(ctx, P, (const float*)orig, (const float*)recon, out, metric_mask, K);
+      if (st != CZC_OK) out->computed_mask = 0;
+      return st;
+    }
   }
   CZC_CUDA(ctx, cudaMemcpyAsync(ctx->din[0], orig, bytes, cudaMemcpyHostToDevice, ctx->stream));
   CZC_CUDA(ctx, cudaMemcpyAsync(ctx->din[1], recon, bytes, cudaMemcpyHostToDevice, ctx->stream));

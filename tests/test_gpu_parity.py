@@ -250,3 +250,22 @@ def test_nccl_slab_path_single_rank(czc):
     for k in ("mse", "psnr", "pearson", "ssim", "der1_mae", "lap_mse"):
         assert abs(g[k] - g1[k]) <= 1e-12 * max(1.0, abs(g1[k])), k
     assert np.allclose(g["ac"], g1["ac"], rtol=0, atol=1e-13)
+
+
+@pytest.mark.parametrize("dims,w", [((100, 120, 96), 8), ((23, 31, 40), 5), ((9, 300, 41), 3)])
+def test_assess_host_pipelined(czc, orc, dims, w):
+    """czc_assess_host (chunked H2D overlapped with per-chunk kernels) vs the oracle and vs
+    czc_assess on the same data."""
+    x, y = synth.make_pair(synth.config("C2", dims=dims))
+    xn, yn = x.numpy(), y.numpy()
+    with czc.Assessor(ssim_window=w) as a:
+        g = a.assess_host(x.pin_memory(), y.pin_memory())
+        gd = a.assess(x.cuda(), y.cuda())
+    o = {}
+    o.update(orc.p1(xn, yn))
+    o.update(orc.deriv(xn, yn))
+    o["ac"], o["ac_count"] = orc.autocorr(xn, yn, 10)
+    o["ssim"], o["n_windows"] = orc.ssim(xn, yn, [w] * 3)
+    full_check(g, o)
+    for k in ("x_min", "x_max", "err_maxabs", "pwr_min", "pwr_max", "n_pwr", "n_windows", "n_interior"):
+        assert g[k] == gd[k], k
