@@ -45,20 +45,21 @@ __device__ __forceinline__ double dmin(double a, double b) { return a < b ? a : 
 
 // Derived fields of one point.  AXES is compile-time: 3 -> (z, y, x), 2 -> (y, x), 1 -> (x).
 // Axis order z, y, x (slowest first) as in the oracle.
+// The /2 of the central differences D_a = delta_a / 2 is applied once per point: sum D_a =
+// 0.5 sum delta_a and sum D_a^2 = 0.25 sum delta_a^2 hold exactly (power-of-two scaling).
 template <int AXES>
 __device__ __forceinline__ void deriv_fields(const double c, const double zp, const double zm,
                                              const double yp, const double ym, const double xp,
                                              const double xm, double F[CZC_NDERIV]) {
-  double der1 = 0, der2 = 0, g2 = 0, div = 0, lap = 0;
+  double der1 = 0, der2 = 0, d2 = 0, dsum = 0, lap = 0;
 #define CZC_AXIS(P, M)                          \
   {                                             \
     const double delta = (P) - (M);             \
-    const double D = delta * 0.5;               \
     const double l = (P) - 2.0 * c + (M);       \
     der1 += fabs(delta);                        \
     der2 += fabs(l);                            \
-    g2 = fma(D, D, g2);                         \
-    div += D;                                   \
+    d2 = fma(delta, delta, d2);                 \
+    dsum += delta;                              \
     lap += l;                                   \
   }
   if (AXES >= 3) CZC_AXIS(zp, zm)
@@ -67,8 +68,8 @@ __device__ __forceinline__ void deriv_fields(const double c, const double zp, co
 #undef CZC_AXIS
   F[CZC_DER1] = der1;
   F[CZC_DER2] = der2;
-  F[CZC_GRAD] = fast_sqrt(g2);
-  F[CZC_DIV] = div;
+  F[CZC_GRAD] = 0.5 * fast_sqrt(d2);
+  F[CZC_DIV] = 0.5 * dsum;
   F[CZC_LAP] = lap;
 }
 
@@ -115,20 +116,27 @@ deriv_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __res
 
   double xm = 0, x0 = 0, ym = 0, y0 = 0;
   float nxv = 0.f, nyv = 0.f, nhx = 0.f, nhy = 0.f;   // prefetched: own at z+1, halo at z
+  PlaneCursor cown, chalo;                            // own column at z+2, halo cell at z+1
   if (zb < ze) {
     if (own) {
       x0 = s.xp(zb)[col]; y0 = s.yp(zb)[col];
-      if (az) { xm = s.xp(zb - 1)[col]; ym = s.yp(zb - 1)[col]; nxv = s.xp(zb + 1)[col]; nyv = s.yp(zb + 1)[col]; }
+      if (az) {
+        xm = s.xp(zb - 1)[col]; ym = s.yp(zb - 1)[col]; nxv = s.xp(zb + 1)[col]; nyv = s.yp(zb + 1)[col];
+        if (zb + 2 <= s.nz - 1) cown.init(s, zb + 2, col);
+      }
     }
-    if (hown) { nhx = s.xp(zb)[hcol]; nhy = s.yp(zb)[hcol]; }
+    if (hown) {
+      nhx = s.xp(zb)[hcol]; nhy = s.yp(zb)[hcol];
+      if (zb + 1 < ze) chalo.init(s, zb + 1, hcol);
+    }
   }
   for (int64_t z = zb; z < ze; z++) {
     const int buf = (int)((z - zb) & 1);
     const double xp = az ? (double)nxv : 0.0, yp = az ? (double)nyv : 0.0;
     const float hxv = nhx, hyv = nhy;
-    // prefetch: own column at z+2, halo at z+1
-    if (own && az && z + 2 <= s.nz - 1 && z + 1 < ze) { nxv = __ldg(s.xp(z + 2) + col); nyv = __ldg(s.yp(z + 2) + col); }
-    if (hown && z + 1 < ze) { nhx = __ldg(s.xp(z + 1) + hcol); nhy = __ldg(s.yp(z + 1) + hcol); }
+    // prefetch: own column at z+2, halo at z+1 (cursors advance one plane per step)
+    if (own && az && z + 2 <= s.nz - 1 && z + 1 < ze) { nxv = __ldg(cown.x); nyv = __ldg(cown.y); cown.advance(s, col); }
+    if (hown && z + 1 < ze) { nhx = __ldg(chalo.x); nhy = __ldg(chalo.y); chalo.advance(s, hcol); }
     pl[buf][ty + 1][tx + 1] = make_double2(x0, y0);
     if (tid < kHalo) pl[buf][hr][hc] = make_double2(hxv, hyv);
     __syncthreads();

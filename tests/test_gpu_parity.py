@@ -269,3 +269,84 @@ def test_assess_host_pipelined(czc, orc, dims, w):
     full_check(g, o)
     for k in ("x_min", "x_max", "err_maxabs", "pwr_min", "pwr_max", "n_pwr", "n_windows", "n_interior"):
         assert g[k] == gd[k], k
+
+
+@pytest.mark.parametrize("dims,w", [((20, 24, 40), 2), ((22, 20, 40), 16), ((19, 40, 44), 11), ((24, 33, 50), 12)])
+def test_window_extents(czc, orc, dims, w):
+    """Small and large window extents (W >= 10 uses the register-heavier 1-block/SM variant)."""
+    x, y = synth.make_pair(synth.config("C1", dims=dims))
+    xn, yn = x.numpy(), y.numpy()
+    with czc.Assessor(ssim_window=w) as a:
+        g = a.assess(x.cuda(), y.cuda(), czc.M_SSIM | czc.M_P1)
+    s, nw = orc.ssim(xn, yn, [w] * 3)
+    errors = []
+    check_ssim(g["ssim"], g["n_windows"], s, nw, errors)
+    report(errors)
+
+
+def test_context_reuse_across_shapes(czc, orc):
+    """One context, shapes growing and shrinking (scratch reallocation), masks varying."""
+    with czc.Assessor(ssim_window=5, ac_max_lag=6) as a:
+        for dims, mask in (((10, 12, 14), czc.M_ALL), ((40, 50, 60), czc.M_ALL), ((8, 9, 10), czc.M_P1),
+                           ((30, 31, 32), czc.M_DERIV | czc.M_AUTOCORR), ((12, 13, 14), czc.M_SSIM)):
+            x, y = synth.make_pair(synth.config("C1", dims=dims))
+            xn, yn = x.numpy(), y.numpy()
+            g = a.assess(x.cuda(), y.cuda(), mask)
+            errors = []
+            if mask & czc.M_P1:
+                check_p1(g, orc.p1(xn, yn), errors)
+            if mask & czc.M_DERIV:
+                check_deriv(g, orc.deriv(xn, yn), errors)
+            if mask & czc.M_AUTOCORR:
+                ac, cnt = orc.autocorr(xn, yn, 6)
+                check_ac(g["ac"], g["ac_count"], ac, cnt, errors)
+            if mask & czc.M_SSIM:
+                s, nw = orc.ssim(xn, yn, [5, 5, 5])
+                check_ssim(g["ssim"], g["n_windows"], s, nw, errors)
+            report(errors)
+            assert g["computed_mask"] == mask
+
+
+def test_status_codes(czc):
+    import ctypes
+    lib = czc.get_lib()
+    x = torch.zeros((6, 7, 8), device="cuda")
+    with czc.Assessor() as a:
+        r = czc.Result()
+        shape = czc.make_shape([6, 7, 8])
+        assert lib.czc_assess(a.ctx, x.data_ptr(), x.data_ptr(), ctypes.byref(shape), 1, czc.M_P1, ctypes.byref(r)) == 3
+        bad = czc.make_shape([6, 0, 8])
+        assert lib.czc_assess(a.ctx, x.data_ptr(), x.data_ptr(), ctypes.byref(bad), 0, czc.M_P1, ctypes.byref(r)) == 2
+        slab = czc.make_shape([6, 7, 8], z0=2, nz_local=3)            # slab shape without ranks
+        assert lib.czc_assess(a.ctx, x.data_ptr(), x.data_ptr(), ctypes.byref(slab), 0, czc.M_P1, ctypes.byref(r)) == 2
+        assert r.computed_mask == 0
+        assert lib.czc_last_error(a.ctx)
+
+
+def test_timing_fields(czc):
+    x, y = synth.make_pair(synth.config("C1", dims=(40, 40, 40)))
+    with czc.Assessor(timing=True) as a:
+        g = a.assess(x.cuda(), y.cuda())
+    ms = g["kernel_ms"]
+    assert all(v > 0 for v in ms[:5]) and ms[4] >= sum(ms[:4]) * 0.99
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("cfg,dims", [("C3", (96, 128, 160)), ("C2q", (100, 160, 200))])
+def test_sampled_windows_large(czc, orc, cfg, dims):
+    """Per-window SSIM on log-normal (>= 4 decades) and 70 %-zero fields, sampled against the
+    oracle's brute-force window; prints the worst error seen (tolerance 1e-6)."""
+    x, y = synth.make_pair(synth.config(cfg, dims=dims))
+    xn, yn = x.numpy(), y.numpy()
+    nw = [n - 8 + 1 for n in dims]
+    dbg = torch.empty(nw, dtype=torch.float64, device="cuda")
+    with czc.Assessor(ssim_window=8, debug_wssim=dbg.data_ptr()) as a:
+        a.assess(x.cuda(), y.cuda(), czc.M_SSIM)
+    d = dbg.cpu().numpy()
+    rng = np.random.default_rng(5)
+    worst = 0.0
+    for _ in range(600):
+        o = [int(rng.integers(0, k)) for k in nw]
+        worst = max(worst, abs(d[tuple(o)] - orc.ssim_window(xn, yn, o, [8, 8, 8])))
+    print(f"{cfg} worst sampled window error {worst:.3e}")
+    assert worst < 1e-6
