@@ -202,65 +202,74 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
       const int64_t gxl = x0 + lane;
       const bool xok = lane < TX && gxl <= f.nx - WX && (gxl % p.sx) == 0;
       // ---- (b) y-pass over WY rows, (c) x-pass with shuffles, mix ------------------------
-      double h[4];
-      // y-window min/max: rows [warp G, warp G + G + WY - 1) of this lane's column; the WY - G + 1
-      // rows shared by all G windows of the warp are reduced once
-      float cmn = Zm[(warp * G + G - 1) * 32 + lane], cmx = Zm[ZS + (warp * G + G - 1) * 32 + lane];
+      // ---- (b) y-pass: the G origin rows of this warp (running sums over WY rows) ------------
+      double h[G][4];
+      float hmn[G], hmx[G];
+      {
+        // y-window min/max: the WY - G + 1 rows shared by all G windows are reduced once
+        float cmn = Zm[(warp * G + G - 1) * 32 + lane], cmx = Zm[ZS + (warp * G + G - 1) * 32 + lane];
 #pragma unroll
-      for (int i = G; i < WY; i++) {
-        cmn = fminf(cmn, Zm[(warp * G + i) * 32 + lane]);
-        cmx = fmaxf(cmx, Zm[ZS + (warp * G + i) * 32 + lane]);
+        for (int i = G; i < WY; i++) {
+          cmn = fminf(cmn, Zm[(warp * G + i) * 32 + lane]);
+          cmx = fmaxf(cmx, Zm[ZS + (warp * G + i) * 32 + lane]);
+        }
+#pragma unroll
+        for (int g = 0; g < G; g++) {
+          const int oy = warp * G + g;
+#pragma unroll
+          for (int m = 0; m < 4; m++) {
+            if (g == 0) {
+              double acc = 0;
+#pragma unroll
+              for (int i = 0; i < WY; i++) acc += Zd[m * ZS + (oy + i) * 32 + lane];
+              h[g][m] = acc;
+            } else {
+              h[g][m] = h[g - 1][m] + (Zd[m * ZS + (oy + WY - 1) * 32 + lane] - Zd[m * ZS + (oy - 1) * 32 + lane]);
+            }
+          }
+          float mn = cmn, mx = cmx;                      // rows [G-1, WY) relative to warp*G
+#pragma unroll
+          for (int i = g; i < G - 1; i++) {              // rows oy .. warp*G + G - 2
+            mn = fminf(mn, Zm[(warp * G + i) * 32 + lane]);
+            mx = fmaxf(mx, Zm[ZS + (warp * G + i) * 32 + lane]);
+          }
+#pragma unroll
+          for (int i = WY; i < WY + g; i++) {            // rows warp*G + WY .. oy + WY - 1
+            mn = fminf(mn, Zm[(warp * G + i) * 32 + lane]);
+            mx = fmaxf(mx, Zm[ZS + (warp * G + i) * 32 + lane]);
+          }
+          hmn[g] = mn;
+          hmx[g] = mx;
+        }
+      }
+      // ---- (c) x-pass for all G rows together (independent shuffle chains -> ILP), then mix --
+      double S[G][4];
+      float wmn[G], wmx[G];
+#pragma unroll
+      for (int g = 0; g < G; g++) {
+#pragma unroll
+        for (int m = 0; m < 4; m++) S[g][m] = lane_window_sum<WX>(h[g][m]);
+        wmn[g] = lane_window_ext<WX, false>(hmn[g]);
+        wmx[g] = lane_window_ext<WX, true>(hmx[g]);
       }
 #pragma unroll
       for (int g = 0; g < G; g++) {
-        const int oy = warp * G + g;
-        if (g == 0) {
-#pragma unroll
-          for (int m = 0; m < 4; m++) {
-            double acc = 0;
-#pragma unroll
-            for (int i = 0; i < WY; i++) acc += Zd[m * ZS + (oy + i) * 32 + lane];
-            h[m] = acc;
-          }
-        } else {
-#pragma unroll
-          for (int m = 0; m < 4; m++)
-            h[m] += Zd[m * ZS + (oy + WY - 1) * 32 + lane] - Zd[m * ZS + (oy - 1) * 32 + lane];
-        }
-        float hmn = cmn, hmx = cmx;                      // rows [G-1, WY) relative to warp*G
-#pragma unroll
-        for (int i = g; i < G - 1; i++) {                // rows oy .. warp*G + G - 2
-          hmn = fminf(hmn, Zm[(warp * G + i) * 32 + lane]);
-          hmx = fmaxf(hmx, Zm[ZS + (warp * G + i) * 32 + lane]);
-        }
-#pragma unroll
-        for (int i = WY; i < WY + g; i++) {              // rows warp*G + WY .. oy + WY - 1
-          hmn = fminf(hmn, Zm[(warp * G + i) * 32 + lane]);
-          hmx = fmaxf(hmx, Zm[ZS + (warp * G + i) * 32 + lane]);
-        }
-        const double S0 = lane_window_sum<WX>(h[0]);
-        const double S1 = lane_window_sum<WX>(h[1]);
-        const double S2 = lane_window_sum<WX>(h[2]);
-        const double S3 = lane_window_sum<WX>(h[3]);
-        const float mn = lane_window_ext<WX, false>(hmn);
-        const float mx = lane_window_ext<WX, true>(hmx);
-        const int64_t gy = y0 + oy;
-        if (xok && zok && gy <= f.ny - WY && (gy % p.sy) == 0) {
-          const double mua = S0 * invM, mue = S1 * invM;
-          const double mux = K + mua, muy = mux + mue;
-          const double sxy = S2 * invM - mua * (mua + mue);
-          const double see = S3 * invM - mue * mue;
-          double L = range_global ? Lglob : (double)mx - (double)mn;
-          L = (L == 0.0) ? 1.0 : L;
-          const double C1 = (0.01 * L) * (0.01 * L), C2 = (0.03 * L) * (0.03 * L);
-          const double A = 2.0 * mux * muy + C1, B = 2.0 * sxy + C2;
-          // A, B, A + mu_e^2, B + s_e^2 > 0 (C1, C2 > 0); |rel err of the reciprocal| <= 2u
-          const double ssim = (A * B) * fast_rcp((A + mue * mue) * (B + see));
-          const int64_t gxo = x0 + lane;
-          ssum += ssim;
-          scnt += 1.0;
-          if (dbg) dbg[((oz / p.sz) * p.nwy + gy / p.sy) * p.nwx + gxo / p.sx] = ssim;
-        }
+        const int64_t gy = y0 + warp * G + g;
+        const bool ok = xok && zok && gy <= f.ny - WY && (gy % p.sy) == 0;
+        // computed by every lane (no divergence); invalid lanes are masked out of the sums
+        const double mua = S[g][0] * invM, mue = S[g][1] * invM;
+        const double mux = K + mua, muy = mux + mue;
+        const double sxy = S[g][2] * invM - mua * (mua + mue);
+        const double see = S[g][3] * invM - mue * mue;
+        double L = range_global ? Lglob : (double)wmx[g] - (double)wmn[g];
+        L = (L == 0.0) ? 1.0 : L;
+        const double C1 = (0.01 * L) * (0.01 * L), C2 = (0.03 * L) * (0.03 * L);
+        const double A = 2.0 * mux * muy + C1, B = 2.0 * sxy + C2;
+        // A, B, A + mu_e^2, B + s_e^2 > 0 (C1, C2 > 0); |rel err of the reciprocal| <= 2u
+        const double ssim = (A * B) * fast_rcp((A + mue * mue) * (B + see));
+        ssum += ok ? ssim : 0.0;
+        scnt += ok ? 1.0 : 0.0;
+        if (dbg && ok) dbg[((oz / p.sz) * p.nwy + gy / p.sy) * p.nwx + (x0 + lane) / p.sx] = ssim;
       }
     }
   }
