@@ -24,7 +24,7 @@ cudaError_t launch_p1(const float* x, const float* y, int64_t n, int grid_cap, P
 cudaError_t launch_p1_combine(const P1State* states, int count, DevResults* res, cudaStream_t st);
 int p1_max_blocks_per_sm();
 int64_t deriv_blocks(const Field3& s, int zchunk);
-int64_t ac_blocks(const Field3& s, int zchunk);
+int64_t ac_blocks(const Field3& s, int T);
 cudaError_t launch_deriv(const Field3& s, int zchunk, double* parts, DevResults* res,
                          unsigned int* ticket, cudaStream_t st);
 cudaError_t launch_ac(const Field3& s, int T, int zchunk, double* parts, DevResults* res,
@@ -408,7 +408,7 @@ int64_t halo_depth(const Plan& P) {
 static czc_status ensure_scratch(czc_ctx* ctx, const Plan& P, const Field3& F, const SsimParams& sp) {
   size_t need = (size_t)ctx->p1_grid_cap * sizeof(P1State);
   if (P.run_deriv) need = std::max(need, (size_t)deriv_blocks(F, kZchunkDeriv) * kDerivSlots * sizeof(double));
-  if (P.run_ac) need = std::max(need, (size_t)ac_blocks(F, 0) * kAcSlots * sizeof(double));
+  if (P.run_ac) need = std::max(need, (size_t)ac_blocks(F, P.T) * kAcSlots * sizeof(double));
   if (P.run_ssim) {
     int64_t nb = 0;
     if (launch_ssim(P.kind, P.W, F, sp, nullptr, nullptr, nullptr, nullptr, ctx->stream, &nb) != cudaSuccess) {

@@ -174,6 +174,25 @@ struct PlaneCursor {
     else { x += f.ny * f.nx; y += f.ny * f.nx; }
   }
 };
+
+// Lighter cursor for hot loops: plane pointers plus the number of planes left in the current
+// segment (32-bit); the caller passes the next plane's index only for the rare re-init.
+struct SegCursor {
+  const float* x;
+  const float* y;
+  int left;
+  __device__ __forceinline__ void init(const Field3& f, int64_t z0) {
+    x = f.xp(z0);
+    y = f.yp(z0);
+    const int64_t last = f.nseg == 1 ? f.zs[1] : (f.nseg == 2 ? f.zs[2] : f.zs[3]);   // static indices
+    const int64_t e = (f.nseg > 1 && z0 < f.zs[1]) ? f.zs[1] : ((f.nseg > 2 && z0 < f.zs[2]) ? f.zs[2] : last);
+    left = (int)(e - z0 < INT32_MAX ? e - z0 : INT32_MAX);
+  }
+  __device__ __forceinline__ void advance(const Field3& f, int64_t znext) {
+    if (--left <= 0) init(f, znext);
+    else { x += f.ny * f.nx; y += f.ny * f.nx; }
+  }
+};
 #endif
 
 struct SsimParams {
@@ -210,31 +229,6 @@ __device__ __forceinline__ bool last_block_arrive(unsigned int* ticket) {
   return s_last;
 }
 
-// Deterministic combine of K-slot records (run by every thread of the last block, 1-D view of
-// the block).  Thread t folds records t, t+T, t+2T, ... in increasing order; then a fixed
-// shuffle + shared-memory tree.  Result depends only on nblocks, never on arrival order.
-template <int K, typename OpOf>
-__device__ void finish_slots(const double* parts, int nblocks, OpOf op_of, double* out) {
-  __shared__ double s_red[32];
-  const int tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
-  const int nthr = blockDim.x * blockDim.y * blockDim.z;
-  const int lane = tid & 31, warp = tid >> 5, nwarps = (nthr + 31) >> 5;
-  for (int k = 0; k < K; k++) {
-    const int op = op_of(k);
-    double v = op_identity(op);
-    for (int b = tid; b < nblocks; b += nthr) v = op_apply(op, v, __ldcg(parts + (size_t)b * K + k));
-    for (int off = 16; off > 0; off >>= 1) v = op_apply(op, v, __shfl_down_sync(0xffffffffu, v, off));
-    if (lane == 0) s_red[warp] = v;
-    __syncthreads();
-    if (warp == 0) {
-      double w = lane < nwarps ? s_red[lane] : op_identity(op);
-      for (int off = 16; off > 0; off >>= 1) w = op_apply(op, w, __shfl_down_sync(0xffffffffu, w, off));
-      if (lane == 0) out[k] = w;
-    }
-    __syncthreads();
-  }
-}
-
 // Block-level combine of a per-thread K-slot record into slot values held by thread 0.
 template <int K, typename OpOf>
 __device__ void block_reduce_slots(double (&v)[K], OpOf op_of, double* dst_global) {
@@ -257,6 +251,26 @@ __device__ void block_reduce_slots(double (&v)[K], OpOf op_of, double* dst_globa
     __syncthreads();
   }
 }
+
+// Deterministic combine of K-slot records (run by every thread of the last block, 1-D view of
+// the block).  Thread t folds records t, t+T, t+2T, ... in increasing order, all K slots at once
+// (K independent loads in flight per record), then the fixed block tree of block_reduce_slots.
+// The result depends only on nblocks, never on arrival order.
+template <int K, typename OpOf>
+__device__ void finish_slots(const double* parts, int nblocks, OpOf op_of, double* out) {
+  const int tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  const int nthr = blockDim.x * blockDim.y * blockDim.z;
+  double v[K];
+#pragma unroll
+  for (int k = 0; k < K; k++) v[k] = op_identity(op_of(k));
+  for (int b = tid; b < nblocks; b += nthr) {
+    const double* p = parts + (size_t)b * K;
+#pragma unroll
+    for (int k = 0; k < K; k++) v[k] = op_apply(op_of(k), v[k], __ldcg(p + k));
+  }
+  block_reduce_slots<K>(v, op_of, out);
+}
+
 
 // 1/v for finite normal v > 0: rcp.approx (MUFU.RCP64H) + two Newton steps, |rel err| <= 2u.
 __device__ __forceinline__ double fast_rcp(double v) {

@@ -43,11 +43,12 @@ __device__ __forceinline__ double fast_sqrt(double a) {
 __device__ __forceinline__ double dmax(double a, double b) { return a > b ? a : b; }
 __device__ __forceinline__ double dmin(double a, double b) { return a < b ? a : b; }
 
-// Derived fields of one point.  AXES is compile-time: 3 -> (z, y, x), 2 -> (y, x), 1 -> (x).
-// Axis order z, y, x (slowest first) as in the oracle.
+// Derived fields of one point.  ZA / YA: the streamed (slow) axis / the in-plane y axis are
+// active; x is always active.  Axis order slow, y, x (slowest first) as in the oracle.  A 2-D
+// field is streamed along its rows: its y axis plays the slow axis (ZA, !YA).
 // The /2 of the central differences D_a = delta_a / 2 is applied once per point: sum D_a =
 // 0.5 sum delta_a and sum D_a^2 = 0.25 sum delta_a^2 hold exactly (power-of-two scaling).
-template <int AXES>
+template <bool ZA, bool YA>
 __device__ __forceinline__ void deriv_fields(const double c, const double zp, const double zm,
                                              const double yp, const double ym, const double xp,
                                              const double xm, double F[CZC_NDERIV]) {
@@ -62,8 +63,8 @@ __device__ __forceinline__ void deriv_fields(const double c, const double zp, co
     dsum += delta;                              \
     lap += l;                                   \
   }
-  if (AXES >= 3) CZC_AXIS(zp, zm)
-  if (AXES >= 2) CZC_AXIS(yp, ym)
+  if (ZA) CZC_AXIS(zp, zm)
+  if (YA) CZC_AXIS(yp, ym)
   CZC_AXIS(xp, xm)
 #undef CZC_AXIS
   F[CZC_DER1] = der1;
@@ -80,17 +81,21 @@ struct SumOp {
   __device__ int operator()(int) const { return OP_SUM; }
 };
 
-constexpr int kHalo = 2 * (kTX + 2) + 2 * kTY;   // halo cells of one plane tile
-
-// grid: (ceil(nx/32), ceil(ny/8), zchunks); block (32, 8).  AXES: active axes (3, 2 or 1).
-template <int AXES>
-__global__ void __launch_bounds__(kTX * kTY, 2)
+// grid: (ceil(nx/BX), ceil(ny/BY), zchunks); block (BX, BY), BX * BY = 256.
+//   3-D: <true, true, 32, 8>; 2-D row view (slow axis = rows): <true, false, 256, 1>;
+//   1-D: <false, false, 256, 1>.
+template <bool ZA, bool YA, int BX, int BY>
+__global__ void __launch_bounds__(BX * BY, 2)
 deriv_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
              unsigned int* __restrict__ ticket) {
+  constexpr int kTX = BX, kTY = BY;
+  // halo cells of one plane tile: the full ring with a y axis, the two x ends without
+  constexpr int kHalo = YA ? 2 * (kTX + 2) + 2 * kTY : 2;
+  static_assert(kHalo <= BX * BY, "halo larger than the block");
   __shared__ double2 pl[2][kTY + 2][kTX + 2];     // (x, y) of the current plane, double-buffered
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * kTX + tx;
   const int64_t gx = (int64_t)blockIdx.x * kTX + tx, gy = (int64_t)blockIdx.y * kTY + ty;
-  constexpr bool az = AXES >= 3, ay = AXES >= 2;
+  constexpr bool az = ZA, ay = YA;
   // interior ranges (reading R11), restricted to the owned planes
   int64_t zlo = az ? 1 : 0, zhi = az ? s.nz - 1 : 1;
   if (zlo < s.zown0) zlo = s.zown0;
@@ -108,7 +113,8 @@ deriv_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __res
   const int64_t col = own ? gy * s.nx + gx : 0;
   // halo cell of this thread (tid < kHalo): row hr, column hc of the padded tile
   int hr = 0, hc = 0;
-  if (tid < 2 * (kTX + 2)) { hr = tid < kTX + 2 ? 0 : kTY + 1; hc = tid % (kTX + 2); }
+  if (!YA) { hr = 1; hc = tid == 0 ? 0 : kTX + 1; }
+  else if (tid < 2 * (kTX + 2)) { hr = tid < kTX + 2 ? 0 : kTY + 1; hc = tid % (kTX + 2); }
   else if (tid < kHalo) { const int t = tid - 2 * (kTX + 2); hr = 1 + t % kTY; hc = t < kTY ? 0 : kTX + 1; }
   const int64_t hy = (int64_t)blockIdx.y * kTY + hr - 1, hx = (int64_t)blockIdx.x * kTX + hc - 1;
   const bool hown = tid < kHalo && hy >= 0 && hy < s.ny && hx >= 0 && hx < s.nx;
@@ -144,8 +150,8 @@ deriv_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __res
       const double2 yn = pl[buf][ty + 2][tx + 1], ys = pl[buf][ty][tx + 1];
       const double2 xe = pl[buf][ty + 1][tx + 2], xw = pl[buf][ty + 1][tx];
       double Fx[CZC_NDERIV], Fy[CZC_NDERIV];
-      deriv_fields<AXES>(x0, xp, xm, yn.x, ys.x, xe.x, xw.x, Fx);
-      deriv_fields<AXES>(y0, yp, ym, yn.y, ys.y, xe.y, xw.y, Fy);
+      deriv_fields<ZA, YA>(x0, xp, xm, yn.x, ys.x, xe.x, xw.x, Fx);
+      deriv_fields<ZA, YA>(y0, yp, ym, yn.y, ys.y, xe.y, xw.y, Fy);
 #pragma unroll
       for (int fi = 0; fi < CZC_NDERIV; fi++) {
         const double d = Fy[fi] - Fx[fi];
@@ -323,39 +329,6 @@ ac_zwalk_tma(Field3 s, int T, int zchunk, double* __restrict__ parts, DevResults
   ac_finish<TM>(acc, parts, res->rec.ac[0], ticket);
 }
 
-// y-walk, TMA: block = 256 consecutive x of plane z; grid (x tiles, owned planes, y chunks).
-template <int TM>
-__global__ void __launch_bounds__(kWalkThreads, 3)
-ac_ywalk_tma(Field3 s, int T, int ychunk, double* __restrict__ parts, DevResults* __restrict__ res,
-             unsigned int* __restrict__ ticket) {
-  extern __shared__ __align__(128) unsigned char walk_smem[];
-  BulkWalkSmem<TM>& sm = *reinterpret_cast<BulkWalkSmem<TM>*>(walk_smem);
-  const int64_t x0 = (int64_t)blockIdx.x * kWalkThreads;
-  const int64_t gx = x0 + threadIdx.x;
-  const int64_t z = s.zown0 + (int64_t)blockIdx.y;
-  const double mu = res->p1g.me;
-  const bool own = gx < s.nx;
-  int64_t m = T;
-  if (s.nz > 1 && s.nz - 1 - z < m) m = s.nz - 1 - z;
-  if (s.nx > 1 && s.nx - 1 - gx < m) m = s.nx - 1 - gx;
-  const int64_t lo = (int64_t)blockIdx.z * ychunk;
-  int64_t hi = lo + ychunk;
-  if (hi > s.ny) hi = s.ny;
-  int64_t end = hi + T;
-  if (end > s.ny) end = s.ny;
-  const int64_t ncols = (s.nx - x0) < kWalkThreads ? (s.nx - x0) : kWalkThreads;
-  double ring[TM], acc[TM];
-#pragma unroll
-  for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
-  bulk_walk<TM>(sm, [&](int64_t y, const float*& xr, const float*& yr) {
-                  xr = s.xp(z) + y * s.nx + x0;
-                  yr = s.yp(z) + y * s.nx + x0;
-                },
-                (uint32_t)(ncols * 4), lo, hi, end, mu, ring, acc);
-  walk_mask<TM>(acc, own ? (int)m : 0);
-  ac_finish<TM>(acc, parts, res->rec.ac[1], ticket);
-}
-
 // z-walk: thread <-> column (y, x); block 32 x 8 columns; grid.z chunks of owned planes.
 template <int TM>
 __global__ void __launch_bounds__(256)
@@ -385,41 +358,6 @@ ac_zwalk(Field3 s, int T, int zchunk, double* __restrict__ parts, DevResults* __
   }, lo, hi, end, mu, own, ring, acc);
   walk_mask<TM>(acc, own ? (int)m : 0);
   ac_finish<TM>(acc, parts, res->rec.ac[0], ticket);
-}
-
-// y-walk: thread <-> line (z, x); a block's 256 threads cover 256 consecutive x of one plane (one
-// 1 KB contiguous row segment per step); grid (x tiles, owned planes, y chunks).
-template <int TM>
-__global__ void __launch_bounds__(256)
-ac_ywalk(Field3 s, int T, int ychunk, double* __restrict__ parts, DevResults* __restrict__ res,
-         unsigned int* __restrict__ ticket) {
-  const int64_t gx = (int64_t)blockIdx.x * 256 + threadIdx.x;
-  const int64_t z = s.zown0 + (int64_t)blockIdx.y;
-  const double mu = res->p1g.me;
-  const bool own = gx < s.nx && z < s.zown1;
-  int64_t m = T;
-  if (s.nz > 1 && s.nz - 1 - z < m) m = s.nz - 1 - z;
-  if (s.nx > 1 && s.nx - 1 - gx < m) m = s.nx - 1 - gx;
-  const int64_t lo = (int64_t)blockIdx.z * ychunk;
-  int64_t hi = lo + ychunk;
-  if (hi > s.ny) hi = s.ny;
-  int64_t end = hi + T;
-  if (end > s.ny) end = s.ny;
-  const float* X = own ? s.xp(z) + gx : nullptr;
-  const float* Y = own ? s.yp(z) + gx : nullptr;
-  const int64_t nx = s.nx;
-  double ring[TM], acc[TM];
-#pragma unroll
-  for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
-  const float* px = own ? X + lo * nx : nullptr;
-  const float* py = own ? Y + lo * nx : nullptr;
-  walk_line<TM, TM>([&]() {
-    const float2 v = make_float2(__ldg(px), __ldg(py));
-    px += nx; py += nx;
-    return v;
-  }, lo, hi, end, mu, own, ring, acc);
-  walk_mask<TM>(acc, own ? (int)m : 0);
-  ac_finish<TM>(acc, parts, res->rec.ac[1], ticket);
 }
 
 // x-walk, fast path (rows 16-byte aligned: nx % 4 == 0 and aligned segment bases): lane l of
@@ -543,7 +481,211 @@ ac_xwalk_smem(Field3 s, int T, int xchunk, double* __restrict__ parts, DevResult
   ac_finish<TM>(acc, parts, res->rec.ac[2], ticket);
 }
 
+// ---- in-plane lags (x and y) on 2-D tiles ------------------------------------------------------
+// For a plane z, the x- and y-lag products of the points of a 64 x 32 tile need eps on the tile
+// plus a +TM halo in x and y.  The block stages the raw (x, y) samples of that (32+TM) x (64+TM)
+// window with cp.async (16-byte granules when rows are 16-byte aligned, zero-fill outside the
+// field), converts them once to eps = (y - x) - mu in a shared double tile (0 outside the field),
+// and then every thread walks two short segments with all their values in registers:
+//   y-role: column c = tid % 64, rows 8 s .. 8 s + 7 (s = tid / 64): 8 + TM loads, 8 TM FMAs;
+//   x-role: row r = tid % 32, columns 8 s .. 8 s + 7 (s = tid / 32): 8 + TM loads, 8 TM FMAs.
+// A product eps_p eps_{p + t e_a} belongs to p and counts when p is in Eq. 2's R_t (p + t e_b
+// inside the field on every active axis b).  Along the walk axis that holds by the zero fill; the
+// other two axes give one bound per thread segment (lim), applied to the segment's lag sums.
+// Tiles far from the field ends (all t <= TM valid) skip even that.  The next plane's copies
+// overlap the walks of the current one.
+// Work split: the (tile, plane) pairs in tile-major order are cut into gridDim.x equal ranges,
+// one per block (a persistent grid of the resident block count): no tail wave, and the
+// assignment is static, so the result is deterministic.
+constexpr int kPlTX = 64, kPlTY = 32, kPlThreads = 256, kPlSeg = 8;
+template <int TM>
+struct PlaneTile {
+  static_assert(TM % 2 == 0, "even lag templates only");
+  static constexpr int HX = kPlTX + TM, HY = kPlTY + TM;
+  static constexpr int NV = (HX + 3) / 4;        // 16-byte groups per staged row
+  static constexpr int PF = 4 * NV;              // staged row pitch (floats), 16-byte multiple
+  static constexpr int PE = (PF + 1) | 1;        // eps row pitch (doubles), odd: conflict-free columns
+  double e[HY][PE];
+  float fx[HY][PF];
+  float fy[HY][PF];
+};
+
+__device__ __forceinline__ void cp_async4(unsigned dst, const void* src, int src_bytes) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
+}
+__device__ __forceinline__ void cp_async16(unsigned dst, const void* src, int src_bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
+
+// Stage the window of one plane.  Warp w copies staged rows w, w + 8, ...; VEC: lane g < NV copies
+// the 16-byte group g of the row (vb = bytes of that group inside the field, fixed per thread);
+// scalar: lanes copy single samples.  xt / yt point at the tile origin (y0, x0) of the plane.
+template <int TM, bool VEC>
+__device__ __forceinline__ void plane_stage(unsigned sfx, const float* xt, const float* yt, int64_t nx, int rv,
+                                            int cv, int vb, int warp, int lane) {
+  constexpr int HX = PlaneTile<TM>::HX, HY = PlaneTile<TM>::HY, NV = PlaneTile<TM>::NV, PF = PlaneTile<TM>::PF;
+  constexpr int RS = kPlThreads / 32;                             // row stride
+  constexpr unsigned dy = (unsigned)(sizeof(float) * HY * PF);   // fx -> fy
+  if (VEC) {
+    if (lane < NV) {
+      const float* px = xt + warp * nx + 4 * lane;
+      const float* py = yt + warp * nx + 4 * lane;
+      unsigned d = sfx + (unsigned)(sizeof(float) * (warp * PF + 4 * lane));
+      for (int r = warp; r < HY; r += RS) {
+        if (r < rv) {
+          cp_async16(d, px, vb);
+          cp_async16(d + dy, py, vb);
+        } else {                                                  // below the field: zero fill
+          cp_async16(d, xt, 0);
+          cp_async16(d + dy, yt, 0);
+        }
+        px += RS * nx; py += RS * nx; d += sizeof(float) * RS * PF;
+      }
+    }
+  } else {
+    for (int r = warp; r < HY; r += RS) {
+#pragma unroll
+      for (int c0 = 0; c0 < HX; c0 += 32) {
+        const int c = c0 + lane;
+        if (c < HX) {
+          const bool ok = r < rv && c < cv;
+          const int64_t o = ok ? r * nx + c : 0;
+          const unsigned d = sfx + (unsigned)(sizeof(float) * (r * PF + c));
+          cp_async4(d, xt + o, ok ? 4 : 0);
+          cp_async4(d + dy, yt + o, ok ? 4 : 0);
+        }
+      }
+    }
+  }
+  cp_async_commit();
+}
+
+// Lag products of one segment v[0 .. 8 + TM): points j < 8 own v[j] * v[j + t].  With LIM, the
+// segment's lag-t sum counts only if t <= lim.
+template <int TM, bool LIM>
+__device__ __forceinline__ void seg_products(const double (&v)[kPlSeg + TM], int lim, double (&acc)[TM]) {
+#pragma unroll
+  for (int t = 1; t <= TM; t++) {
+    if (!LIM) {
+#pragma unroll
+      for (int j = 0; j < kPlSeg; j++) acc[t - 1] = fma(v[j], v[j + t], acc[t - 1]);
+    } else {
+      double part = 0.0;
+#pragma unroll
+      for (int j = 0; j < kPlSeg; j++) part = fma(v[j], v[j + t], part);
+      acc[t - 1] += t <= lim ? part : 0.0;
+    }
+  }
+}
+
+// limx: R_t bound of the y-role's column (from x), limy: of the x-role's row (from y), both
+// already capped by the plane's z bound.
+template <int TM, bool LIM>
+__device__ __forceinline__ void plane_walks(const PlaneTile<TM>& sm, int tid, int limx, int limy, double (&acc)[TM]) {
+  double v[kPlSeg + TM];
+  {  // y-role
+    const int c = tid & (kPlTX - 1), ys = (tid / kPlTX) * kPlSeg;
+#pragma unroll
+    for (int j = 0; j < kPlSeg + TM; j++) v[j] = sm.e[ys + j][c];
+    seg_products<TM, LIM>(v, limx, acc);
+  }
+  {  // x-role
+    const int r = tid & 31, xs = (tid / 32) * kPlSeg;
+#pragma unroll
+    for (int j = 0; j < kPlSeg + TM; j++) v[j] = sm.e[r][xs + j];
+    seg_products<TM, LIM>(v, limy, acc);
+  }
+}
+
+// grid: persistent (gridDim.x blocks); block 256; requires ny > 1.
+// VEC: rows 16-byte aligned (nx % 4 == 0, aligned plane segments) and (32 + TM) * nx < 2^31.
+template <int TM, bool VEC>
+__global__ void __launch_bounds__(kPlThreads, TM <= 10 ? 3 : 2)
+ac_plane(Field3 s, double* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket) {
+  extern __shared__ __align__(128) unsigned char plane_smem[];
+  PlaneTile<TM>& sm = *reinterpret_cast<PlaneTile<TM>*>(plane_smem);
+  constexpr int HY = PlaneTile<TM>::HY, NV = PlaneTile<TM>::NV;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const unsigned sfx = (unsigned)__cvta_generic_to_shared(&sm.fx[0][0]);
+  const int r0 = tid / NV, g0 = tid % NV;          // this thread's first conversion group
+  const double mu = res->p1g.me;
+  const int64_t nzo = s.zown1 - s.zown0, ntx = (s.nx + kPlTX - 1) / kPlTX;
+  const int64_t ntiles = ntx * ((s.ny + kPlTY - 1) / kPlTY), W = ntiles * nzo;
+  const int64_t jb = W * blockIdx.x / gridDim.x, je = W * (blockIdx.x + 1) / gridDim.x;
+  double acc[TM];
+#pragma unroll
+  for (int t = 0; t < TM; t++) acc[t] = 0;
+  for (int64_t j = jb; j < je;) {
+    const int64_t tile = j / nzo, zb = s.zown0 + (j - tile * nzo);
+    int64_t run = je - j;
+    if (run > s.zown1 - zb) run = s.zown1 - zb;
+    j += run;
+    const int64_t ze = zb + run;
+    const int64_t x0 = (tile % ntx) * kPlTX, y0 = (tile / ntx) * kPlTY;
+    const bool xy_inner = x0 + kPlTX + TM <= s.nx && y0 + kPlTY + TM <= s.ny;
+    // staged cells outside the field hold eps = 0
+    const int rv = (int)(s.ny - y0 < HY ? s.ny - y0 : HY);
+    const int cv = (int)(s.nx - x0 < PlaneTile<TM>::PF ? s.nx - x0 : PlaneTile<TM>::PF);
+    int vb = cv - 4 * lane;
+    vb = vb <= 0 ? 0 : (vb >= 4 ? 16 : 4 * vb);
+    const int64_t torg = y0 * s.nx + x0;
+    // per-segment R_t bounds from x (y-role column) and y (x-role row)
+    const int64_t mx = s.nx - 1 - (x0 + (tid & (kPlTX - 1))), my = s.ny - 1 - (y0 + (tid & 31));
+    const int limx0 = mx < TM ? (int)(mx < -1 ? -1 : mx) : TM, limy0 = my < TM ? (int)(my < -1 ? -1 : my) : TM;
+    __syncthreads();                       // previous run's walks are done with the tile
+    PlaneCursor cur;
+    cur.init(s, zb, torg);
+    plane_stage<TM, VEC>(sfx, cur.x, cur.y, s.nx, rv, cv, vb, warp, lane);
+    for (int64_t z = zb; z < ze; z++) {
+      cp_async_wait_all();
+      __syncthreads();                     // plane z staged; previous walks done with sm.e
+      {
+        // all 16-byte groups of the staged window, 256 at a time (row r, group g of the row)
+        int r = r0, g = g0;
+        for (int i = tid; i < HY * NV; i += kPlThreads) {
+          const float4 a = *reinterpret_cast<const float4*>(&sm.fx[r][4 * g]);
+          const float4 b = *reinterpret_cast<const float4*>(&sm.fy[r][4 * g]);
+          double e0 = ((double)b.x - (double)a.x) - mu, e1 = ((double)b.y - (double)a.y) - mu;
+          double e2 = ((double)b.z - (double)a.z) - mu, e3 = ((double)b.w - (double)a.w) - mu;
+          if (!xy_inner) {
+            const int c = 4 * g;
+            const bool rin = r < rv;
+            e0 = rin && c < cv ? e0 : 0.0;
+            e1 = rin && c + 1 < cv ? e1 : 0.0;
+            e2 = rin && c + 2 < cv ? e2 : 0.0;
+            e3 = rin && c + 3 < cv ? e3 : 0.0;
+          }
+          double* er = &sm.e[r][4 * g];
+          er[0] = e0; er[1] = e1; er[2] = e2; er[3] = e3;
+          r += kPlThreads / NV;
+          g += kPlThreads % NV;
+          if (g >= NV) { g -= NV; r++; }
+        }
+      }
+      __syncthreads();                     // eps ready, staging buffer free
+      if (z + 1 < ze) {
+        cur.advance(s, torg);
+        plane_stage<TM, VEC>(sfx, cur.x, cur.y, s.nx, rv, cv, vb, warp, lane);
+      }
+      // R_t bound from the z axis (active only for 3-D fields)
+      const int64_t mz64 = s.nz > 1 ? s.nz - 1 - z : TM;
+      const int mz = mz64 > TM ? TM : (int)mz64;
+      if (xy_inner && mz >= TM) plane_walks<TM, false>(sm, tid, TM, TM, acc);
+      else plane_walks<TM, true>(sm, tid, limx0 < mz ? limx0 : mz, limy0 < mz ? limy0 : mz, acc);
+    }
+  }
+  ac_finish<TM>(acc, parts, res->rec.ac[1], ticket);
+}
+
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+static int sm_count() {
+  int d = 0, n = 0;
+  cudaGetDevice(&d);
+  cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, d);
+  return n > 0 ? n : 1;
+}
 
 static int64_t deriv_zplanes(const Field3& s) {
   int64_t zlo = s.nz > 1 ? 1 : 0, zhi = s.nz > 1 ? s.nz - 1 : 1;
@@ -551,71 +693,108 @@ static int64_t deriv_zplanes(const Field3& s) {
   if (zhi > s.zown1) zhi = s.zown1;
   return zhi > zlo ? zhi - zlo : 1;
 }
-int64_t deriv_blocks(const Field3& s, int zchunk) {
-  return cdiv(s.nx, kTX) * cdiv(s.ny, kTY) * cdiv(deriv_zplanes(s), zchunk);
+// 2-D fields (one plane, never slab-sharded) are streamed along their rows: view (ny, 1, nx).
+static Field3 deriv_view(const Field3& s) {
+  if (!(s.nz == 1 && s.ny > 1)) return s;
+  Field3 v = s;
+  v.nz = s.ny; v.ny = 1;
+  v.zown0 = 0; v.zown1 = s.ny;
+  v.zs[0] = 0; v.zs[1] = s.ny;
+  return v;
+}
+// Launch shape: (BX, BY) tiles x chunks of the streamed axis; the chunk length is the requested
+// one unless that leaves fewer than ~8 blocks per SM (short or 2-D fields), never below 8 planes.
+static dim3 deriv_grid(const Field3& s, int zchunk, int* zc) {
+  const int bx = s.ny > 1 ? kTX : 256, by = s.ny > 1 ? kTY : 1;
+  const int64_t tiles = cdiv(s.nx, bx) * cdiv(s.ny, by), planes = deriv_zplanes(s);
+  int64_t c = zchunk;
+  const int64_t fill = cdiv(planes * tiles, 148 * 8);
+  if (fill < c) c = fill < 8 ? 8 : fill;
+  c = cdiv(planes, cdiv(planes, c));          // equal chunks
+  *zc = (int)c;
+  return dim3((unsigned)cdiv(s.nx, bx), (unsigned)cdiv(s.ny, by), (unsigned)cdiv(planes, c));
+}
+int64_t deriv_blocks(const Field3& s0, int zchunk) {
+  int zc;
+  const dim3 g = deriv_grid(deriv_view(s0), zchunk, &zc);
+  return (int64_t)g.x * g.y * g.z;
 }
 
-cudaError_t launch_deriv(const Field3& s, int zchunk, double* parts, DevResults* res,
+cudaError_t launch_deriv(const Field3& s0, int zchunk, double* parts, DevResults* res,
                          unsigned int* ticket, cudaStream_t st) {
-  dim3 grid((unsigned)cdiv(s.nx, kTX), (unsigned)cdiv(s.ny, kTY), (unsigned)cdiv(deriv_zplanes(s), zchunk));
-  if (s.nz > 1) deriv_kernel<3><<<grid, dim3(kTX, kTY), 0, st>>>(s, zchunk, parts, res, ticket);
-  else if (s.ny > 1) deriv_kernel<2><<<grid, dim3(kTX, kTY), 0, st>>>(s, zchunk, parts, res, ticket);
-  else deriv_kernel<1><<<grid, dim3(kTX, kTY), 0, st>>>(s, zchunk, parts, res, ticket);
+  const Field3 s = deriv_view(s0);
+  int zc;
+  const dim3 grid = deriv_grid(s, zchunk, &zc);
+  if (s.ny > 1) deriv_kernel<true, true, kTX, kTY><<<grid, dim3(kTX, kTY), 0, st>>>(s, zc, parts, res, ticket);
+  else if (s.nz > 1) deriv_kernel<true, false, 256, 1><<<grid, dim3(256, 1), 0, st>>>(s, zc, parts, res, ticket);
+  else deriv_kernel<false, false, 256, 1><<<grid, dim3(256, 1), 0, st>>>(s, zc, parts, res, ticket);
   return cudaGetLastError();
 }
 
-// Autocorrelation: one launch per active walk axis, each with its own partial-buffer slice and
-// ticket; the three records are summed at the finish.
+// Autocorrelation: the z-walk (3-D fields) and the in-plane tile kernel (x and y lags, ny > 1),
+// or the x-walk alone for 1-D fields; each launch has its own partial-buffer slice and ticket and
+// writes its own record slot (z -> ac[0], in-plane -> ac[1], x-walk -> ac[2]); the finish sums them.
 struct AcGrids {
-  dim3 z, y, x, xvec, zt, yt;
+  dim3 z, zt, pl, x, xvec;
   bool rz, ry, rx;
-  int zc, yc, xc;
+  int zc, pzc, xc;
 };
-static AcGrids ac_grids(const Field3& s) {
+static AcGrids ac_grids(const Field3& s, int T) {
   AcGrids g{};
   const int64_t nzo = s.zown1 - s.zown0;
-  g.zc = 50; g.yc = 50; g.xc = 128;    // xc % 4 == 0 for the vector x-walk
+  g.zc = 50; g.xc = 128;    // xc % 4 == 0 for the vector x-walk
   g.rz = s.nz > 1; g.ry = s.ny > 1; g.rx = s.nx > 1;
+  // persistent in-plane grid: the resident block count (3 per SM for TM <= 10, else 2)
+  const int64_t W = cdiv(s.nx, kPlTX) * cdiv(s.ny, kPlTY) * nzo;
+  const int64_t G = (int64_t)sm_count() * (T <= 10 ? 3 : 2);
+  g.pzc = 0;
   g.z = dim3((unsigned)cdiv(s.nx, kTX), (unsigned)cdiv(s.ny, kTY), (unsigned)cdiv(nzo, g.zc));
-  g.y = dim3((unsigned)cdiv(s.nx, 256), (unsigned)nzo, (unsigned)cdiv(s.ny, g.yc));
+  g.zt = dim3((unsigned)cdiv(s.nx, kWalkThreads), (unsigned)s.ny, (unsigned)cdiv(nzo, g.zc));
+  g.pl = dim3((unsigned)(W < G ? W : G), 1, 1);
   g.x = dim3((unsigned)cdiv(nzo * s.ny, kXWarps * 32), (unsigned)cdiv(s.nx, g.xc), 1);
   g.xvec = dim3((unsigned)cdiv(nzo * s.ny, 256), (unsigned)cdiv(s.nx, g.xc), 1);
-  g.zt = dim3((unsigned)cdiv(s.nx, kWalkThreads), (unsigned)s.ny, (unsigned)cdiv(nzo, g.zc));
-  g.yt = dim3((unsigned)cdiv(s.nx, kWalkThreads), (unsigned)nzo, (unsigned)cdiv(s.ny, g.yc));
   return g;
 }
-int64_t ac_blocks(const Field3& s, int) {
-  const AcGrids g = ac_grids(s);
+int64_t ac_blocks(const Field3& s, int T) {
+  const AcGrids g = ac_grids(s, T);
   auto n = [](dim3 d) { return (int64_t)d.x * d.y * d.z; };
   auto mx = [](int64_t a, int64_t b) { return a > b ? a : b; };
-  return mx(n(g.z), n(g.zt)) + mx(n(g.y), n(g.yt)) + mx(n(g.x), n(g.xvec));
+  return mx(n(g.z), n(g.zt)) + n(g.pl) + mx(n(g.x), n(g.xvec));
 }
 
 template <int TM>
 static cudaError_t launch_ac_t(const Field3& s, int T, double* parts, DevResults* res,
                                unsigned int* tickets, cudaStream_t st) {
-  const AcGrids g = ac_grids(s);
+  const AcGrids g = ac_grids(s, T);
   auto n = [](dim3 d) { return (size_t)d.x * d.y * d.z; };
-  // rows 16-byte aligned (nx % 4 == 0, aligned segments): TMA bulk-copy walks and the vector x-walk
+  // rows 16-byte aligned (nx % 4 == 0, aligned segments): TMA bulk-copy z-walk and vector x-walk
   bool vec = (s.nx % 4) == 0;
   for (int k = 0; k < s.nseg; k++)
     vec = vec && (reinterpret_cast<uintptr_t>(s.xs[k]) % 16) == 0 && (reinterpret_cast<uintptr_t>(s.ys[k]) % 16) == 0;
   double* pz = parts;
-  double* py = pz + (vec ? n(g.zt) : n(g.z)) * kAcSlots;
-  double* px = py + (vec ? n(g.yt) : n(g.y)) * kAcSlots;
+  double* pp = pz + (vec ? n(g.zt) : n(g.z)) * kAcSlots;
+  double* px = pp + n(g.pl) * kAcSlots;
   cudaError_t e = cudaMemsetAsync(res->rec.ac, 0, sizeof(res->rec.ac), st);
   if (e != cudaSuccess) return e;
-  constexpr int wsm = (int)sizeof(BulkWalkSmem<TM>);
-  if (vec) {
+  if (g.rz && vec) {
+    constexpr int wsm = (int)sizeof(BulkWalkSmem<TM>);
     if ((e = cudaFuncSetAttribute(ac_zwalk_tma<TM>, cudaFuncAttributeMaxDynamicSharedMemorySize, wsm)) != cudaSuccess) return e;
-    if ((e = cudaFuncSetAttribute(ac_ywalk_tma<TM>, cudaFuncAttributeMaxDynamicSharedMemorySize, wsm)) != cudaSuccess) return e;
+    ac_zwalk_tma<TM><<<g.zt, kWalkThreads, wsm, st>>>(s, T, g.zc, pz, res, tickets + 0);
+  } else if (g.rz) {
+    ac_zwalk<TM><<<g.z, dim3(kTX, kTY), 0, st>>>(s, T, g.zc, pz, res, tickets + 0);
   }
-  if (g.rz && vec) ac_zwalk_tma<TM><<<g.zt, kWalkThreads, wsm, st>>>(s, T, g.zc, pz, res, tickets + 0);
-  else if (g.rz) ac_zwalk<TM><<<g.z, dim3(kTX, kTY), 0, st>>>(s, T, g.zc, pz, res, tickets + 0);
-  if (g.ry && vec) ac_ywalk_tma<TM><<<g.yt, kWalkThreads, wsm, st>>>(s, T, g.yc, py, res, tickets + 1);
-  else if (g.ry) ac_ywalk<TM><<<g.y, 256, 0, st>>>(s, T, g.yc, py, res, tickets + 1);
-  if (g.rx && vec) ac_xwalk_vec<TM><<<g.xvec, 256, 0, st>>>(s, T, g.xc, px, res, tickets + 2);
-  else if (g.rx) ac_xwalk_smem<TM><<<g.x, kXWarps * 32, 0, st>>>(s, T, g.xc, px, res, tickets + 2);
+  if (g.ry) {
+    constexpr int psm = (int)sizeof(PlaneTile<TM>);
+    // 16-byte staging needs aligned rows; tile-relative offsets are 32-bit
+    const bool pvec = vec && (int64_t)(kPlTY + TM) * s.nx < ((int64_t)1 << 31);
+    auto kern = pvec ? ac_plane<TM, true> : ac_plane<TM, false>;
+    if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, psm)) != cudaSuccess) return e;
+    kern<<<g.pl, kPlThreads, psm, st>>>(s, pp, res, tickets + 1);
+  } else if (g.rx && vec) {
+    ac_xwalk_vec<TM><<<g.xvec, 256, 0, st>>>(s, T, g.xc, px, res, tickets + 2);
+  } else if (g.rx) {
+    ac_xwalk_smem<TM><<<g.x, kXWarps * 32, 0, st>>>(s, T, g.xc, px, res, tickets + 2);
+  }
   return cudaGetLastError();
 }
 

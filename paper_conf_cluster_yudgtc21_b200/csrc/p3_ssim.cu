@@ -123,20 +123,23 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
     vbits |= (v ? 1u : 0u) << k;
     off[k] = v ? (int)(gy * f.nx + gx) : 0;
   }
-  // Prefetch of plane z (x, y) and of the y sample of the plane leaving the z-window (z - WZ),
-  // which is re-read from L2 instead of being kept in the register ring.
-  auto load = [&](int64_t z, float2 (&dst)[KC], float (&yold)[KC]) {
-    if (z < zend) {
-      const float* X = f.xp(z);
-      const float* Y = f.yp(z);
-      const bool has_old = z - zb >= WZ;
-      const float* Yo = has_old ? f.yp(z - WZ) : Y;
+  // Prefetch of plane zb + n (x, y) and of the y sample of the plane leaving the z-window
+  // (zb + n - WZ), which is re-read from L2 instead of being kept in the register ring.  Both
+  // streams advance through plane cursors (pointer increments, no per-plane address math).
+  const int nsteps = (int)(zend - zb);
+  SegCursor cin, cold;
+  if (nsteps > 0) { cin.init(f, zb); cold.init(f, zb); }
+  auto load = [&](int n, float2 (&dst)[KC], float (&yold)[KC]) {
+    if (n < nsteps) {
+      const bool has_old = n >= WZ;
 #pragma unroll
       for (int k = 0; k < KC; k++) {
         const bool v = (vbits >> k) & 1u;
-        dst[k] = v ? make_float2(__ldg(X + off[k]), __ldg(Y + off[k])) : make_float2(0.f, 0.f);
-        yold[k] = (v && has_old) ? __ldg(Yo + off[k]) : 0.f;
+        dst[k] = v ? make_float2(__ldg(cin.x + off[k]), __ldg(cin.y + off[k])) : make_float2(0.f, 0.f);
+        yold[k] = (v && has_old) ? __ldg(cold.y + off[k]) : 0.f;
       }
+      cin.advance(f, zb + n + 1);
+      if (has_old) cold.advance(f, zb + n + 1 - WZ);
     }
   };
 
@@ -151,21 +154,30 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
   }
   float2 nxt[KC];                                        // prefetched next plane
   float nyo[KC];                                         // ... and its leaving y sample
-  load(zb, nxt, nyo);
+  load(0, nxt, nyo);
 
   double ssum = 0, scnt = 0;
   const bool range_global = p.range_mode != 0;
-  for (int64_t zz = zb; zz < zend; zz += WZ) {
+  // origin-grid membership: x and y are fixed per thread, z advances one plane per step
+  const int64_t gxl = x0 + lane;
+  const bool xok = lane < TX && gxl <= f.nx - WX && (gxl % p.sx) == 0;
+  bool gok[G];
+#pragma unroll
+  for (int g = 0; g < G; g++) {
+    const int64_t gy = y0 + warp * G + g;
+    gok[g] = xok && gy <= f.ny - WY && (gy % p.sy) == 0;
+  }
+  int zph = (int)(zb % p.sz);                            // phase of origin plane zb
+  for (int s0 = 0; s0 < nsteps; s0 += WZ) {
 #pragma unroll
     for (int s = 0; s < WZ; s++) {
-      const int64_t zi = zz + s;
-      if (zi >= zend) break;                             // block-uniform
-      const int step = (int)(zi - zb);                   // == s (mod WZ)
+      const int step = s0 + s;                           // == s (mod WZ)
+      if (step >= nsteps) break;                         // block-uniform
       float2 v[KC];
       float yo[KC];
 #pragma unroll
       for (int k = 0; k < KC; k++) { v[k] = nxt[k]; yo[k] = nyo[k]; }
-      load(zi + 1, nxt, nyo);
+      load(step + 1, nxt, nyo);
       const int buf = step & 1;
       double* Zd = reinterpret_cast<double*>(smem_raw + buf * Gm::buf_bytes);
       float* Zm = reinterpret_cast<float*>(Zd + 4 * ZS);
@@ -197,10 +209,8 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
       }
       if (step < WZ - 1) continue;                       // no complete z-window yet
       __syncthreads();
-      const int64_t oz = zi - WZ + 1;
-      const bool zok = (oz % p.sz) == 0;
-      const int64_t gxl = x0 + lane;
-      const bool xok = lane < TX && gxl <= f.nx - WX && (gxl % p.sx) == 0;
+      const bool zok = zph == 0;                         // origin plane zb + step - WZ + 1
+      zph = zph + 1 == p.sz ? 0 : zph + 1;
       // ---- (b) y-pass over WY rows, (c) x-pass with shuffles, mix ------------------------
       // ---- (b) y-pass: the G origin rows of this warp (running sums over WY rows) ------------
       double h[G][4];
@@ -254,8 +264,7 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
       }
 #pragma unroll
       for (int g = 0; g < G; g++) {
-        const int64_t gy = y0 + warp * G + g;
-        const bool ok = xok && zok && gy <= f.ny - WY && (gy % p.sy) == 0;
+        const bool ok = zok && gok[g];
         // computed by every lane (no divergence); invalid lanes are masked out of the sums
         const double mua = S[g][0] * invM, mue = S[g][1] * invM;
         const double mux = K + mua, muy = mux + mue;
@@ -269,7 +278,10 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
         const double ssim = (A * B) * fast_rcp((A + mue * mue) * (B + see));
         ssum += ok ? ssim : 0.0;
         scnt += ok ? 1.0 : 0.0;
-        if (dbg && ok) dbg[((oz / p.sz) * p.nwy + gy / p.sy) * p.nwx + (x0 + lane) / p.sx] = ssim;
+        if (dbg && ok) {
+          const int64_t oz = zb + step - WZ + 1, gy = y0 + warp * G + g;
+          dbg[((oz / p.sz) * p.nwy + gy / p.sy) * p.nwx + (x0 + lane) / p.sx] = ssim;
+        }
       }
     }
   }
