@@ -181,15 +181,15 @@ struct SegCursor {
   const float* x;
   const float* y;
   int left;
-  __device__ __forceinline__ void init(const Field3& f, int64_t z0) {
-    x = f.xp(z0);
-    y = f.yp(z0);
+  __device__ __forceinline__ void init(const Field3& f, int64_t z0, int64_t off = 0) {
+    x = f.xp(z0) + off;
+    y = f.yp(z0) + off;
     const int64_t last = f.nseg == 1 ? f.zs[1] : (f.nseg == 2 ? f.zs[2] : f.zs[3]);   // static indices
     const int64_t e = (f.nseg > 1 && z0 < f.zs[1]) ? f.zs[1] : ((f.nseg > 2 && z0 < f.zs[2]) ? f.zs[2] : last);
     left = (int)(e - z0 < INT32_MAX ? e - z0 : INT32_MAX);
   }
-  __device__ __forceinline__ void advance(const Field3& f, int64_t znext) {
-    if (--left <= 0) init(f, znext);
+  __device__ __forceinline__ void advance(const Field3& f, int64_t znext, int64_t off = 0) {
+    if (--left <= 0) init(f, znext, off);
     else { x += f.ny * f.nx; y += f.ny * f.nx; }
   }
 };

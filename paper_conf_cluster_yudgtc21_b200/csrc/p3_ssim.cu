@@ -173,11 +173,10 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
     for (int s = 0; s < WZ; s++) {
       const int step = s0 + s;                           // == s (mod WZ)
       if (step >= nsteps) break;                         // block-uniform
-      float2 v[KC];
-      float yo[KC];
-#pragma unroll
-      for (int k = 0; k < KC; k++) { v[k] = nxt[k]; yo[k] = nyo[k]; }
-      load(step + 1, nxt, nyo);
+      // the prefetched plane is consumed by the z-walk below, then the next one is requested
+      // into the same registers (no copies; its latency hides behind the y / x passes)
+      const float2 (&v)[KC] = nxt;
+      const float (&yo)[KC] = nyo;
       const int buf = step & 1;
       double* Zd = reinterpret_cast<double*>(smem_raw + buf * Gm::buf_bytes);
       float* Zm = reinterpret_cast<float*>(Zd + 4 * ZS);
@@ -207,6 +206,7 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
           Zm[ZS + c] = mx;
         }
       }
+      load(step + 1, nxt, nyo);
       if (step < WZ - 1) continue;                       // no complete z-window yet
       __syncthreads();
       const bool zok = zph == 0;                         // origin plane zb + step - WZ + 1
