@@ -350,3 +350,46 @@ def test_sampled_windows_large(czc, orc, cfg, dims):
         worst = max(worst, abs(d[tuple(o)] - orc.ssim_window(xn, yn, o, [8, 8, 8])))
     print(f"{cfg} worst sampled window error {worst:.3e}")
     assert worst < 1e-6
+
+
+def test_misaligned_3d_views(czc, orc):
+    """3-D fields whose base pointers are 4-byte (not 16-byte) aligned: the in-plane AC tile
+    kernel and the z-walk take their scalar staging paths, everything else must not care."""
+    x, y = synth.make_pair(synth.config("C2", dims=(21, 36, 64)))
+    n = x.numel()
+    for off in (1, 2):
+        bx = torch.zeros(n + 8); by = torch.zeros(n + 8)
+        bx[off:off + n] = x.ravel(); by[off:off + n] = y.ravel()
+        xd = bx.cuda()[off:off + n].view(21, 36, 64)
+        yd = by.cuda()[off:off + n].view(21, 36, 64)
+        with czc.Assessor(ndim=3, ssim_window=6, ac_max_lag=10) as a:
+            g = a.assess(xd, yd, czc.M_ALL)
+        xn, yn = x.numpy(), y.numpy()
+        o = {}
+        o.update(orc.p1(xn, yn)); o.update(orc.deriv(xn, yn))
+        o["ac"], o["ac_count"] = orc.autocorr(xn, yn, 10)
+        o["ssim"], o["n_windows"] = orc.ssim(xn, yn, [6, 6, 6], [1, 1, 1], 0)
+        full_check(g, o)
+
+
+@pytest.mark.parametrize("kind", ["negated", "scaled"])
+def test_sign_flip_and_scaled_recon(czc, orc, kind):
+    """Reconstructions far from the original (opposite sign, 2.5x): every float difference is
+    inexact in fp32 and many error magnitudes exceed the values."""
+    x, y = synth.make_pair(synth.config("C1", dims=(19, 37, 72)))
+    xn = x.numpy()
+    yn = (-xn + 1e-3 * y.numpy()).astype(np.float32) if kind == "negated" else (2.5 * xn).astype(np.float32)
+    g, o = run_both(czc, orc, xn, yn, window=5)
+    full_check(g, o)
+
+
+@pytest.mark.parametrize("dims,lag", [((12, 74, 138), 10), ((11, 32, 64), 10), ((13, 42, 74), 10),
+                                      ((20, 50, 90), 16), ((15, 33, 65), 3)])
+def test_plane_tile_edges(czc, orc, dims, lag):
+    """In-plane AC tiles (64 x 32 + lag halo): fields that end exactly at a tile, at a tile plus
+    its halo, one past it, and the 16-lag template."""
+    x, y = synth.make_pair(synth.config("C2", dims=dims))
+    g, o = run_both(czc, orc, x.numpy(), y.numpy(), window=4, lag=lag)
+    errors = []
+    check_ac(g["ac"], g["ac_count"], o["ac"], o["ac_count"], errors)
+    report(errors)
