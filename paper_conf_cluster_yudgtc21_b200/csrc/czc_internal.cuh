@@ -3,6 +3,7 @@
 // Partial-result records, the order-fixed (deterministic) cross-block finish, and small device
 // helpers.  Citations "Lnnn" are PAPER.md lines; DESIGN.md §5 describes the kernels.
 #pragma once
+#include <atomic>
 
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -280,6 +281,20 @@ __device__ __forceinline__ double fast_rcp(double v) {
   r = fma(r, e, r);
   e = fma(-v, r, 1.0);
   return fma(r, e, r);
+}
+
+// Opt a kernel into > 48 KB of dynamic shared memory once per device (the attribute persists);
+// keeps host API calls out of the per-call launch sequence.
+template <auto KERN>
+inline cudaError_t set_smem_once(int bytes) {
+  static std::atomic<unsigned long long> done{0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const unsigned long long bit = 1ull << (dev & 63);
+  if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
+  const cudaError_t e = cudaFuncSetAttribute(KERN, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+  if (e == cudaSuccess) done.fetch_or(bit, std::memory_order_release);
+  return e;
 }
 
 // ---- TMA bulk copies + mbarriers (sm_90+ PTX; UBLKCP / SYNCS in SASS) -------------------------

@@ -13,6 +13,13 @@ namespace czc {
 
 // Per-thread accumulator: sums about the thread's first element (kx, ky, ke).  The element count
 // is implicit (counted per vector), so no per-element work is spent on it.
+// rcp.approx.ftz.f64 + one Newton step (relative error < 1e-12 for |v| in the float range)
+__device__ __forceinline__ double rcp_newton1(double v) {
+  double r;
+  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(v));
+  return fma(r, fma(-v, r, 1.0), r);
+}
+
 struct P1Acc {
   double kx, ky, ke;
   double sa, sb, sc, saa, sbb, sab, scc, sae;
@@ -33,14 +40,15 @@ __device__ __forceinline__ void acc_init(P1Acc& a, float kxf, float kyf) {
 
 
 // One element: e = recon - orig in double (reading R1; same rounding as the oracle).  Point-wise
-// relative error |e|/|x| (reading R3): its SUM uses q~ = |e| * rcp(|x|) (relative error <= 4u,
-// far inside the 1e-9 tolerance of pwr_mean); its extrema must be the IEEE quotient, bit-exact
-// with the oracle, so the correctly rounded division runs only for candidates: an element can
-// raise the maximum only if q~ > thr_hi = pmax (1 - 1e-12) (q~ >= Q (1 - 4u) and pmax <= RN(Q)
-// for a larger true quotient Q), and lower the minimum only if q~ < thr_lo = pmin (1 + 1e-12);
-// a zero minimum admits no further candidate (thr_lo = 0), a zero maximum admits only q~ > 0.
-// Returns whether this element is a candidate; the caller resolves candidates per vector so the
-// hot loop has one rarely-taken branch per 4 elements.
+// relative error |e|/|x| (reading R3): its SUM uses q~ = |e| * r, r = rcp.approx(|x|) refined by
+// one Newton step (relative error of q~ < 1e-12: measured max 8.6e-13 for r, profiles/
+// r01_rcp_probe.txt; far inside the 1e-9 tolerance of pwr_mean); its extrema must be the IEEE
+// quotient, bit-exact with the oracle, so the correctly rounded division runs only for
+// candidates: an element can raise the maximum only if q~ > thr_hi = pmax (1 - 1e-10) (q~ >=
+// Q (1 - 1e-12) and pmax <= RN(Q) for a larger true quotient Q), and lower the minimum only if
+// q~ < thr_lo = pmin (1 + 1e-10); a zero minimum admits no further candidate (thr_lo = 0), a zero
+// maximum admits only q~ > 0.  Returns whether this element is a candidate; candidates are
+// resolved per vector, warp-uniformly (see acc_vec).
 __device__ __forceinline__ bool acc_elem(P1Acc& a, float xf, float yf, double& ae_out, double& ax_out) {
   const double x = xf, y = yf;
   const double e = y - x;
@@ -58,7 +66,7 @@ __device__ __forceinline__ bool acc_elem(P1Acc& a, float xf, float yf, double& a
   a.xmax = fmaxf(a.xmax, xf);
   const bool nz = xf != 0.0f;
   const double ax = nz ? fabs(x) : 1.0;
-  const double qa = nz ? ae * fast_rcp(ax) : 0.0;
+  const double qa = nz ? ae * rcp_newton1(ax) : 0.0;
   a.spwr += qa;
   a.npwr += nz ? 1u : 0u;
   ae_out = ae;
@@ -68,8 +76,8 @@ __device__ __forceinline__ bool acc_elem(P1Acc& a, float xf, float yf, double& a
 
 __device__ __forceinline__ void acc_resolve(P1Acc& a, double ae, double ax) {
   const double q = ae / ax;                          // IEEE, correctly rounded
-  if (q > a.pmax) { a.pmax = q; a.pthr_hi = q * (1.0 - 1e-12); }
-  if (q < a.pmin) { a.pmin = q; a.pthr_lo = q * (1.0 + 1e-12); }   // q = 0 -> thr_lo = 0
+  if (q > a.pmax) { a.pmax = q; a.pthr_hi = q * (1.0 - 1e-10); }
+  if (q < a.pmin) { a.pmin = q; a.pthr_lo = q * (1.0 + 1e-10); }   // q = 0 -> thr_lo = 0
 }
 
 __device__ __forceinline__ void acc_vec(P1Acc& a, float4 xv, float4 yv) {
@@ -78,11 +86,26 @@ __device__ __forceinline__ void acc_vec(P1Acc& a, float4 xv, float4 yv) {
   const bool c1 = acc_elem(a, xv.y, yv.y, ae1, ax1);
   const bool c2 = acc_elem(a, xv.z, yv.z, ae2, ax2);
   const bool c3 = acc_elem(a, xv.w, yv.w, ae3, ax3);
-  if (c0 | c1 | c2 | c3) {                            // rare after the first few vectors
+  // Warp-uniform resolve; in a full warp the lanes then share their extrema (a lane may report
+  // the warp's maximum / minimum: merging takes max / min, so the result is unchanged), which
+  // makes later candidates ~32x rarer than with per-lane thresholds.
+  const unsigned m = __activemask();
+  if (__any_sync(m, c0 | c1 | c2 | c3)) {
     if (c0) acc_resolve(a, ae0, ax0);
     if (c1) acc_resolve(a, ae1, ax1);
     if (c2) acc_resolve(a, ae2, ax2);
     if (c3) acc_resolve(a, ae3, ax3);
+    if (m == 0xffffffffu) {
+      double mx = a.pmax, mn = a.pmin;
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) {
+        const double ox = __shfl_xor_sync(m, mx, off), on = __shfl_xor_sync(m, mn, off);
+        mx = ox > mx ? ox : mx;
+        mn = on < mn ? on : mn;
+      }
+      if (mx > a.pmax) { a.pmax = mx; a.pthr_hi = mx * (1.0 - 1e-10); }
+      if (mn < a.pmin) { a.pmin = mn; a.pthr_lo = mn * (1.0 + 1e-10); }
+    }
   }
 }
 

@@ -778,7 +778,7 @@ static cudaError_t launch_ac_t(const Field3& s, int T, double* parts, DevResults
   if (e != cudaSuccess) return e;
   if (g.rz && vec) {
     constexpr int wsm = (int)sizeof(BulkWalkSmem<TM>);
-    if ((e = cudaFuncSetAttribute(ac_zwalk_tma<TM>, cudaFuncAttributeMaxDynamicSharedMemorySize, wsm)) != cudaSuccess) return e;
+    if ((e = set_smem_once<ac_zwalk_tma<TM>>(wsm)) != cudaSuccess) return e;
     ac_zwalk_tma<TM><<<g.zt, kWalkThreads, wsm, st>>>(s, T, g.zc, pz, res, tickets + 0);
   } else if (g.rz) {
     ac_zwalk<TM><<<g.z, dim3(kTX, kTY), 0, st>>>(s, T, g.zc, pz, res, tickets + 0);
@@ -788,7 +788,7 @@ static cudaError_t launch_ac_t(const Field3& s, int T, double* parts, DevResults
     // 16-byte staging needs aligned rows; tile-relative offsets are 32-bit
     const bool pvec = vec && (int64_t)(kPlTY + TM) * s.nx < ((int64_t)1 << 31);
     auto kern = pvec ? ac_plane<TM, true> : ac_plane<TM, false>;
-    if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, psm)) != cudaSuccess) return e;
+    if ((e = pvec ? set_smem_once<ac_plane<TM, true>>(psm) : set_smem_once<ac_plane<TM, false>>(psm)) != cudaSuccess) return e;
     kern<<<g.pl, kPlThreads, psm, st>>>(s, pp, res, tickets + 1);
   } else if (g.rx && vec) {
     ac_xwalk_vec<TM><<<g.xvec, 256, 0, st>>>(s, T, g.xc, px, res, tickets + 2);

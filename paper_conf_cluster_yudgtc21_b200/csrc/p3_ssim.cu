@@ -309,7 +309,7 @@ static cudaError_t launch_t(const Field3& f, const SsimParams& p, double* parts,
             (unsigned)cdiv(noz, p.zchunk));
   if (nblocks_out) { *nblocks_out = (int64_t)grid.x * grid.y * grid.z; return cudaSuccess; }
   if (f.ny * f.nx >= (int64_t)1 << 31) return cudaErrorInvalidValue;   // 32-bit in-plane offsets
-  cudaError_t e = cudaFuncSetAttribute(p3_kernel<WX, WY, WZ, G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Gm::smem);
+  cudaError_t e = set_smem_once<p3_kernel<WX, WY, WZ, G>>((int)Gm::smem);
   if (e != cudaSuccess) return e;
   p3_kernel<WX, WY, WZ, G><<<grid, kP3Threads, Gm::smem, st>>>(f, p, parts, res, ticket, dbg);
   return cudaGetLastError();

@@ -19,7 +19,7 @@ with czc.Assessor(ndim=x.dim(), ssim_window=w, timing=True) as a:
             a.assess(xd, yd, mask)
         ts = []
         for _ in range(5):
-            flush.zero_()
+            flush.zero_(); flush.sum()
             r = a.assess(xd, yd, mask)
             ts.append(r["kernel_ms"])
         best = [min(t[i] for t in ts) for i in range(5)]
