@@ -193,6 +193,11 @@ struct SegCursor {
     if (--left <= 0) init(f, znext, off);
     else { x += f.ny * f.nx; y += f.ny * f.nx; }
   }
+  // same with the plane stride (ny * nx) precomputed by the caller
+  __device__ __forceinline__ void advance_by(const Field3& f, int64_t znext, int64_t off, int64_t plane) {
+    if (--left <= 0) init(f, znext, off);
+    else { x += plane; y += plane; }
+  }
 };
 #endif
 

@@ -172,6 +172,127 @@ deriv_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __res
   if (tid == 0) *ticket = 0;
 }
 
+// 3-D variant with two points per thread: threads (32, 4) cover a 32 x 8 tile, thread (tx, ty)
+// owns rows ty and ty + 4.  The 25 accumulators are shared by both points (half the registers
+// per point) and the two independent stencils double each warp's instruction-level parallelism.
+template <int PTS>
+__global__ void __launch_bounds__(kTX * kTY / PTS, 3)
+deriv3_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+              unsigned int* __restrict__ ticket) {
+  constexpr int RY = kTY / PTS;                    // thread rows
+  constexpr int kHalo = 2 * (kTX + 2) + 2 * kTY;
+  static_assert(kHalo <= kTX * RY, "halo larger than the block");
+  __shared__ double2 pl[2][kTY + 2][kTX + 2];
+  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * kTX + tx;
+  const int64_t gx = (int64_t)blockIdx.x * kTX + tx, gy0 = (int64_t)blockIdx.y * kTY + ty;
+  int64_t zlo = 1, zhi = s.nz - 1;
+  if (zlo < s.zown0) zlo = s.zown0;
+  if (zhi > s.zown1) zhi = s.zown1;
+  const int64_t zb = zlo + (int64_t)blockIdx.z * zchunk;
+  int64_t ze = zb + zchunk;
+  if (ze > zhi) ze = zhi;
+
+  double acc[kDerivSlots];
+#pragma unroll
+  for (int k = 0; k < kDerivSlots; k++) acc[k] = op_identity(deriv_op(k));
+
+  bool own[PTS], inxy[PTS];
+#pragma unroll
+  for (int p = 0; p < PTS; p++) {
+    const int64_t gy = gy0 + p * RY;
+    own[p] = gx < s.nx && gy < s.ny;
+    inxy[p] = own[p] && gy >= 1 && gy < s.ny - 1 && gx >= 1 && gx < s.nx - 1;
+  }
+  const int64_t col = own[0] ? gy0 * s.nx + gx : 0;  // point p: col + p * RY * nx
+  const int64_t rstep = (int64_t)RY * s.nx;
+  int hr = 0, hc = 0;
+  if (tid < 2 * (kTX + 2)) { hr = tid < kTX + 2 ? 0 : kTY + 1; hc = tid % (kTX + 2); }
+  else if (tid < kHalo) { const int t = tid - 2 * (kTX + 2); hr = 1 + t % kTY; hc = t < kTY ? 0 : kTX + 1; }
+  const int64_t hy = (int64_t)blockIdx.y * kTY + hr - 1, hx = (int64_t)blockIdx.x * kTX + hc - 1;
+  const bool hown = tid < kHalo && hy >= 0 && hy < s.ny && hx >= 0 && hx < s.nx;
+  const int64_t hcol = hown ? hy * s.nx + hx : 0;
+
+  double xm[PTS], x0[PTS], ym[PTS], y0[PTS];
+  float nxv[PTS], nyv[PTS];
+  float nhx = 0.f, nhy = 0.f;
+  SegCursor cown, chalo;                          // own column (row 0) at z+2, halo cell at z+1
+  const int64_t plane = s.ny * s.nx;
+#pragma unroll
+  for (int p = 0; p < PTS; p++) { xm[p] = x0[p] = ym[p] = y0[p] = 0; nxv[p] = nyv[p] = 0.f; }
+  if (zb < ze) {
+#pragma unroll
+    for (int p = 0; p < PTS; p++) {
+      if (own[p]) {
+        const int64_t c = col + p * rstep;
+        x0[p] = s.xp(zb)[c]; y0[p] = s.yp(zb)[c];
+        xm[p] = s.xp(zb - 1)[c]; ym[p] = s.yp(zb - 1)[c];
+        nxv[p] = s.xp(zb + 1)[c]; nyv[p] = s.yp(zb + 1)[c];
+      }
+    }
+    if (own[0] && zb + 2 <= s.nz - 1) cown.init(s, zb + 2, col);
+    if (hown) {
+      nhx = s.xp(zb)[hcol]; nhy = s.yp(zb)[hcol];
+      if (zb + 1 < ze) chalo.init(s, zb + 1, hcol);
+    }
+  }
+  // shared-memory slots of this thread (both buffers): centres of its PTS points, its halo cell
+  double2* cbase[2];
+  double2* hslot[2];
+#pragma unroll
+  for (int b = 0; b < 2; b++) {
+    cbase[b] = &pl[b][ty + 1][tx + 1];
+    hslot[b] = &pl[b][hr][hc];
+  }
+  const int n = ze > zb ? (int)(ze - zb) : 0;
+  for (int i = 0; i < n; i++) {
+    const int buf = i & 1;
+    double xp[PTS], yp[PTS];
+#pragma unroll
+    for (int p = 0; p < PTS; p++) { xp[p] = (double)nxv[p]; yp[p] = (double)nyv[p]; }
+    const float hxv = nhx, hyv = nhy;
+    if (i + 1 < n) {
+#pragma unroll
+      for (int p = 0; p < PTS; p++)
+        if (own[p]) { nxv[p] = __ldg(cown.x + p * rstep); nyv[p] = __ldg(cown.y + p * rstep); }
+      if (own[0]) cown.advance_by(s, zb + i + 3, col, plane);
+      if (hown) { nhx = __ldg(chalo.x); nhy = __ldg(chalo.y); chalo.advance_by(s, zb + i + 2, hcol, plane); }
+    }
+    double2* cb = buf ? cbase[1] : cbase[0];
+#pragma unroll
+    for (int p = 0; p < PTS; p++) cb[p * RY * (kTX + 2)] = make_double2(x0[p], y0[p]);
+    if (tid < kHalo) *(buf ? hslot[1] : hslot[0]) = make_double2(hxv, hyv);
+    __syncthreads();
+#pragma unroll
+    for (int p = 0; p < PTS; p++) {
+      if (inxy[p]) {
+        const int r = ty + p * RY + 1;
+        const double2 yn = pl[buf][r + 1][tx + 1], ys = pl[buf][r - 1][tx + 1];
+        const double2 xe = pl[buf][r][tx + 2], xw = pl[buf][r][tx];
+        double Fx[CZC_NDERIV], Fy[CZC_NDERIV];
+        deriv_fields<true, true>(x0[p], xp[p], xm[p], yn.x, ys.x, xe.x, xw.x, Fx);
+        deriv_fields<true, true>(y0[p], yp[p], ym[p], yn.y, ys.y, xe.y, xw.y, Fy);
+#pragma unroll
+        for (int fi = 0; fi < CZC_NDERIV; fi++) {
+          const double d = Fy[fi] - Fx[fi];
+          acc[fi * kDerivStats + 0] = dmax(acc[fi * kDerivStats + 0], fabs(d));
+          acc[fi * kDerivStats + 1] += fabs(d);
+          acc[fi * kDerivStats + 2] = fma(d, d, acc[fi * kDerivStats + 2]);
+          acc[fi * kDerivStats + 3] = dmin(acc[fi * kDerivStats + 3], Fx[fi]);
+          acc[fi * kDerivStats + 4] = dmax(acc[fi * kDerivStats + 4], Fx[fi]);
+        }
+      }
+    }
+#pragma unroll
+    for (int p = 0; p < PTS; p++) { xm[p] = x0[p]; x0[p] = xp[p]; ym[p] = y0[p]; y0[p] = yp[p]; }
+  }
+  __syncthreads();
+  const unsigned bid = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
+  block_reduce_slots<kDerivSlots>(acc, DerivOp{}, parts + (size_t)bid * kDerivSlots);
+  if (!last_block_arrive(ticket)) return;
+  finish_slots<kDerivSlots>(parts, gridDim.x * gridDim.y * gridDim.z, DerivOp{}, res->rec.deriv);
+  if (tid == 0) *ticket = 0;
+}
+
 // ================================================================================================
 // Autocorrelation line walks
 // ================================================================================================
@@ -725,7 +846,8 @@ cudaError_t launch_deriv(const Field3& s0, int zchunk, double* parts, DevResults
   const Field3 s = deriv_view(s0);
   int zc;
   const dim3 grid = deriv_grid(s, zchunk, &zc);
-  if (s.ny > 1) deriv_kernel<true, true, kTX, kTY><<<grid, dim3(kTX, kTY), 0, st>>>(s, zc, parts, res, ticket);
+  if (s.ny > 1 && s.nz > 2) deriv3_kernel<2><<<grid, dim3(kTX, kTY / 2), 0, st>>>(s, zc, parts, res, ticket);
+  else if (s.ny > 1) deriv_kernel<true, true, kTX, kTY><<<grid, dim3(kTX, kTY), 0, st>>>(s, zc, parts, res, ticket);
   else if (s.nz > 1) deriv_kernel<true, false, 256, 1><<<grid, dim3(256, 1), 0, st>>>(s, zc, parts, res, ticket);
   else deriv_kernel<false, false, 256, 1><<<grid, dim3(256, 1), 0, st>>>(s, zc, parts, res, ticket);
   return cudaGetLastError();
