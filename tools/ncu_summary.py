@@ -119,7 +119,7 @@ def main():
         if ks:
             k = ks[0]
             import os
-            out = {"kernel_pattern": pat, "kernel": k["kernel"], "source": reps,
+            out = {"kernel_pattern": pat, "kernel": k["kernel"], "source": [prefix + ".json"], "reports": reps,
                    "dram_bytes_per_launch": k["dram_read_bytes"] + k["dram_write_bytes"],
                    "dram_read_bytes": k["dram_read_bytes"], "dram_write_bytes": k["dram_write_bytes"],
                    "duration_us_cold": k["duration_us"]}
