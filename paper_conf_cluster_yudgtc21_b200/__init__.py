@@ -19,7 +19,8 @@ from typing import Dict, Optional, Sequence
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libczc.so")
+# CZC_LIB overrides the library path (development A/B timing only: tools/ab_time.py)
+LIB_PATH = os.environ.get("CZC_LIB") or os.path.join(_HERE, "libczc.so")
 
 M_P1, M_DERIV, M_AUTOCORR, M_SSIM = 1, 2, 4, 8
 M_ALL = 0xF

@@ -278,6 +278,14 @@ __device__ void finish_slots(const double* parts, int nblocks, OpOf op_of, doubl
 }
 
 
+// rcp.approx.ftz.f64 + one Newton step (relative error < 1e-12 for |v| in the float range;
+// measured max 8.6e-13, profiles/r01_rcp_probe.txt))
+__device__ __forceinline__ double rcp_newton1(double v) {
+  double r;
+  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(v));
+  return fma(r, fma(-v, r, 1.0), r);
+}
+
 // 1/v for finite normal v > 0: rcp.approx (MUFU.RCP64H) + two Newton steps, |rel err| <= 2u.
 __device__ __forceinline__ double fast_rcp(double v) {
   double r;

@@ -13,12 +13,6 @@ namespace czc {
 
 // Per-thread accumulator: sums about the thread's first element (kx, ky, ke).  The element count
 // is implicit (counted per vector), so no per-element work is spent on it.
-// rcp.approx.ftz.f64 + one Newton step (relative error < 1e-12 for |v| in the float range)
-__device__ __forceinline__ double rcp_newton1(double v) {
-  double r;
-  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(v));
-  return fma(r, fma(-v, r, 1.0), r);
-}
 
 struct P1Acc {
   double kx, ky, ke;
