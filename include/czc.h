@@ -37,8 +37,9 @@
 extern "C" {
 #endif
 
-#define CZC_ABI_VERSION 1
+#define CZC_ABI_VERSION 2
 #define CZC_MAX_LAG 16           /* largest supported autocorrelation lag (paper uses <= 10, L345) */
+#define CZC_PDF_MAX_BINS 256     /* largest number of error-PDF bins                              */
 
 typedef enum czc_status {
   CZC_OK = 0,
@@ -59,7 +60,10 @@ enum {
   CZC_M_DERIV = 1u << 1,         /* Category II: Der1/Der2/Grad/Div/Lap errors (L120-L129)      */
   CZC_M_AUTOCORR = 1u << 2,      /* Category II: error autocorrelation, Eq. 2 (L131-L135)        */
   CZC_M_SSIM = 1u << 3,          /* Category III: SSIM (L139-L146)                               */
-  CZC_M_ALL = 0xFu
+  CZC_M_PDF = 1u << 4,           /* Category I: error PDF and pwr-error PDF (Table I): one */
+                                 /* extra pass over the pair after P1 (bins span P1's extrema)  */
+  CZC_M_ALL = 0xFu,              /* the four pattern groups of the north_star (bench.py's step) */
+  CZC_M_FULL = 0x1Fu             /* every metric group, PDFs included                           */
 };
 
 /* Indices of czc_result.deriv[] */
@@ -84,6 +88,7 @@ typedef struct czc_config {
                                  /* into that many slabs and runs the exact multi-GPU path (halo */
                                  /* buffers, owned ranges, rank-ordered combine) with device     */
                                  /* copies in place of NCCL; 0/1 = off.  Requires nranks <= 1.   */
+  int pdf_bins;                  /* CZC_M_PDF: bins per PDF, 1..CZC_PDF_MAX_BINS; 0 -> 100       */
 } czc_config;
 
 /* Field shape.  Single GPU: z0 = 0 and nz_local = dims[0] (or 0 meaning dims[0]).
@@ -125,6 +130,16 @@ typedef struct czc_result {
   double ssim;
   uint64_t n_ssim_exact;         /* windows whose fast-path error bound failed and were          */
                                  /* recomputed by the exact per-window path                      */
+  /* ---- PDFs (Table I Category I "Error PDF", "Pwr error PDF"; reading R24) ------ */
+  /* pdf_bins equal-width bins over [lo, lo + pdf_bins * width]: the error e over [err_min,        */
+  /* err_max] (all N elements), the point-wise relative error |e|/|x| over [pwr_min, pwr_max]      */
+  /* (elements with x != 0).  Bin of v: floor((v - lo) / width) in IEEE double, the top edge       */
+  /* clamped into the last bin; width 0 (all values equal) puts everything in bin 0.  Counts are   */
+  /* exact integers; the density of bin b is count[b] / (total * width).                          */
+  int32_t pdf_bins, _pad1;
+  double err_pdf_lo, err_pdf_width, pwr_pdf_lo, pwr_pdf_width;
+  uint64_t err_pdf[CZC_PDF_MAX_BINS];
+  uint64_t pwr_pdf[CZC_PDF_MAX_BINS];
   /* ---- timing (cfg.timing) ------------------------------------------------------------------- */
   float kernel_ms[6];            /* device ms on the context stream: P1, P2 derivatives, P2      */
                                  /* autocorrelation, P3 SSIM, whole call, (reserved = 0)         */

@@ -13,6 +13,8 @@ implements.  Pinning status of every function:
   autocorr  pinned  (checkerboard (-1)^tau; single-axis cosine; constant error -> NaN)
   ssim      pinned  (zero error = 1; constant-field closed form; global-range mode equals the
                      scipy uniform_filter formulation of scikit-image's SSIM; numpy brute force)
+  pdf       pinned  (constructed values at bin centres: exact per-bin counts; numpy.histogram on
+                     edge-free data; constant error -> one bin; totals = n, n_pwr; top edge clamp)
 """
 from __future__ import annotations
 
@@ -72,6 +74,9 @@ def _load():
         lib.czco_ssim_window.restype = ctypes.c_double
         lib.czco_ssim.argtypes = [P, P, ctypes.c_int, I64P, I64P, I64P, ctypes.c_int,
                                   ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_uint64)]
+        DP = ctypes.POINTER(ctypes.c_double)
+        UP = ctypes.POINTER(ctypes.c_uint64)
+        lib.czco_pdf.argtypes = [P, P, ctypes.c_uint64, ctypes.c_int, DP, DP, UP, DP, DP, UP, UP]
         lib.czco_threads.restype = ctypes.c_int
         _lib = lib
     return _lib
@@ -154,6 +159,23 @@ def ssim(x, y, window, step=None, range_mode: int = 0, dims=None):
     if rc:
         raise ValueError(f"czco_ssim failed ({rc})")
     return out.value, int(nw.value)
+
+
+def pdf(x, y, nbins: int = 100) -> Dict:
+    """Error PDF and pwr-error PDF counts (czco_pdf): keys err_pdf_lo/width, err_pdf (counts),
+    pwr_pdf_lo/width, pwr_pdf, n_pwr."""
+    x, y = _f32(x), _f32(y)
+    d = [ctypes.c_double() for _ in range(4)]
+    ec = (ctypes.c_uint64 * nbins)()
+    pc = (ctypes.c_uint64 * nbins)()
+    npw = ctypes.c_uint64()
+    rc = _load().czco_pdf(x.ctypes.data, y.ctypes.data, x.size, nbins, ctypes.byref(d[0]), ctypes.byref(d[1]),
+                          ec, ctypes.byref(d[2]), ctypes.byref(d[3]), pc, ctypes.byref(npw))
+    if rc:
+        raise ValueError(f"czco_pdf failed ({rc})")
+    return {"err_pdf_lo": d[0].value, "err_pdf_width": d[1].value, "err_pdf": np.array(ec[:], dtype=np.uint64),
+            "pwr_pdf_lo": d[2].value, "pwr_pdf_width": d[3].value, "pwr_pdf": np.array(pc[:], dtype=np.uint64),
+            "n_pwr": int(npw.value)}
 
 
 def assess(x, y, window=None, step=None, max_lag: int = 10, range_mode: int = 0) -> Dict[str, float]:

@@ -393,3 +393,49 @@ int czco_ssim(const float* x, const float* y, int ndim, const int64_t* dims, con
   *ssim = (double)(tot / (ld)total);
   return 0;
 }
+
+/* ======================================================================================
+ * Error PDF / pwr-error PDF (Table I Category I, L107).  The paper names the two metrics but
+ * defines no binning; reading R24: equal-width bins over the value range of the data.
+ * Pass 1 finds the ranges (the same extrema as czco_p1), pass 2 bins every value.
+ * ====================================================================================== */
+static int pdf_bin(double v, double lo, double w, int nbins) {
+  if (!(w > 0) || isinf(w)) return 0;
+  const double q = (v - lo) / w;              /* IEEE quotient, no contraction (R21) */
+  int b = (int)floor(q);
+  if (b >= nbins) b = nbins - 1;
+  if (b < 0) b = 0;
+  return b;
+}
+
+int czco_pdf(const float* x, const float* y, uint64_t n, int nbins, double* err_lo, double* err_w,
+             uint64_t* err_counts, double* pwr_lo, double* pwr_w, uint64_t* pwr_counts, uint64_t* n_pwr) {
+  if (!x || !y || n == 0 || nbins < 1 || !err_counts || !pwr_counts) return 1;
+  double emin = INFINITY, emax = -INFINITY, pmin = INFINITY, pmax = -INFINITY;
+  uint64_t np = 0;
+  for (uint64_t i = 0; i < n; i++) {
+    const double e = err_of(x, y, (int64_t)i);
+    if (e < emin) emin = e;
+    if (e > emax) emax = e;
+    if (x[i] != 0.0f) {
+      const double q = fabs(e) / fabs((double)x[i]);
+      if (q < pmin) pmin = q;
+      if (q > pmax) pmax = q;
+      np++;
+    }
+  }
+  const double ew = (emax - emin) / (double)nbins;
+  const double pw = np ? (pmax - pmin) / (double)nbins : NAN;
+  for (int b = 0; b < nbins; b++) err_counts[b] = pwr_counts[b] = 0;
+  for (uint64_t i = 0; i < n; i++) {
+    const double e = err_of(x, y, (int64_t)i);
+    err_counts[pdf_bin(e, emin, ew, nbins)]++;
+    if (x[i] != 0.0f) pwr_counts[pdf_bin(fabs(e) / fabs((double)x[i]), pmin, pw, nbins)]++;
+  }
+  *err_lo = emin;
+  *err_w = ew;
+  *pwr_lo = np ? pmin : NAN;
+  *pwr_w = pw;
+  *n_pwr = np;
+  return 0;
+}

@@ -61,6 +61,15 @@ double czco_ssim_window(const float* x, const float* y, int ndim, const int64_t*
 int czco_ssim(const float* x, const float* y, int ndim, const int64_t* dims, const int64_t* window,
               const int64_t* step, int range_mode, double* ssim, uint64_t* n_windows);
 
+/* Error PDF and pwr-error PDF (Table I Category I, L107: "Error PDF", "Pwr error PDF"; the paper
+ * gives no bin rule — reading R24): nbins equal-width bins over [min, max] of the
+ * values (the error e = y - x over all n elements; |e|/|x| over x != 0), bin of v =
+ * floor((v - lo) / w) with w = (max - min) / nbins, the top edge clamped into the last bin, w == 0
+ * -> bin 0.  Outputs: lo, w and counts[nbins] of each; *n_pwr = number of x != 0 (if 0, the pwr
+ * lo / w are NaN and its counts 0).  Returns 0 on success. */
+int czco_pdf(const float* x, const float* y, uint64_t n, int nbins, double* err_lo, double* err_w,
+             uint64_t* err_counts, double* pwr_lo, double* pwr_w, uint64_t* pwr_counts, uint64_t* n_pwr);
+
 /* Number of OpenMP threads the oracle uses (bench.py reports it as "cores"). */
 int czco_threads(void);
 

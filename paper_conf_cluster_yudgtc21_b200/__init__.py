@@ -22,9 +22,11 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 # CZC_LIB overrides the library path (development A/B timing only: tools/ab_time.py)
 LIB_PATH = os.environ.get("CZC_LIB") or os.path.join(_HERE, "libczc.so")
 
-M_P1, M_DERIV, M_AUTOCORR, M_SSIM = 1, 2, 4, 8
-M_ALL = 0xF
+M_P1, M_DERIV, M_AUTOCORR, M_SSIM, M_PDF = 1, 2, 4, 8, 16
+M_ALL = 0xF          # the four pattern groups (bench.py's step)
+M_FULL = 0x1F        # + the error / pwr-error PDFs (Table I Category I)
 MAX_LAG = 16
+PDF_MAX_BINS = 256
 DERIV_FIELDS = ("der1", "der2", "grad", "div", "lap")
 DERIV_STATS = ("maxabs", "mae", "mse", "rmse", "f_min", "f_max", "psnr")
 STATUS = {0: "ok", 1: "invalid argument", 2: "invalid shape", 3: "unsupported dtype", 4: "CUDA error",
@@ -42,7 +44,7 @@ class Config(ctypes.Structure):
                 ("ssim_window", ctypes.c_int * 3), ("ssim_step", ctypes.c_int * 3),
                 ("ssim_range_mode", ctypes.c_int), ("ac_max_lag", ctypes.c_int), ("timing", ctypes.c_int),
                 ("rank", ctypes.c_int), ("nranks", ctypes.c_int), ("nccl_uid", ctypes.c_void_p),
-                ("debug_wssim", ctypes.c_void_p), ("loopback_slabs", ctypes.c_int)]
+                ("debug_wssim", ctypes.c_void_p), ("loopback_slabs", ctypes.c_int), ("pdf_bins", ctypes.c_int)]
 
 
 class Shape(ctypes.Structure):
@@ -68,7 +70,12 @@ class Result(ctypes.Structure):
                    ("ac", ctypes.c_double * (MAX_LAG + 1)), ("ac_count", ctypes.c_uint64 * (MAX_LAG + 1)),
                    ("ssim_window", ctypes.c_int32 * 3), ("ssim_step", ctypes.c_int32 * 3),
                    ("n_windows", ctypes.c_uint64), ("ssim", ctypes.c_double),
-                   ("n_ssim_exact", ctypes.c_uint64), ("kernel_ms", ctypes.c_float * 6)])
+                   ("n_ssim_exact", ctypes.c_uint64),
+                   ("pdf_bins", ctypes.c_int32), ("_pad1", ctypes.c_int32),
+                   ("err_pdf_lo", ctypes.c_double), ("err_pdf_width", ctypes.c_double),
+                   ("pwr_pdf_lo", ctypes.c_double), ("pwr_pdf_width", ctypes.c_double),
+                   ("err_pdf", ctypes.c_uint64 * PDF_MAX_BINS), ("pwr_pdf", ctypes.c_uint64 * PDF_MAX_BINS),
+                   ("kernel_ms", ctypes.c_float * 6)])
 
 
 def _load():
@@ -133,7 +140,7 @@ def _per_axis(v, ndim) -> Sequence[int]:
 def make_config(ndim: int = 3, device: int = -1, stream: Optional[int] = None, ssim_window=8, ssim_step=1,
                 ssim_range_mode: int = 0, ac_max_lag: int = 10, timing: bool = False, rank: int = 0,
                 nranks: int = 1, nccl_uid: Optional[bytes] = None, debug_wssim: Optional[int] = None,
-                loopback_slabs: int = 0) -> Config:
+                loopback_slabs: int = 0, pdf_bins: int = 0) -> Config:
     c = Config()
     c.device = device
     c.stream = stream
@@ -151,6 +158,7 @@ def make_config(ndim: int = 3, device: int = -1, stream: Optional[int] = None, s
         c.nccl_uid = ctypes.cast(c._uid, ctypes.c_void_p)
     c.debug_wssim = debug_wssim
     c.loopback_slabs = loopback_slabs
+    c.pdf_bins = pdf_bins
     return c
 
 
@@ -194,6 +202,12 @@ def result_dict(r: Result) -> Dict:
     out["n_windows"] = r.n_windows
     out["ssim"] = r.ssim
     out["n_ssim_exact"] = r.n_ssim_exact
+    nb = max(r.pdf_bins, 0)
+    out["pdf_bins"] = nb
+    for k in ("err_pdf_lo", "err_pdf_width", "pwr_pdf_lo", "pwr_pdf_width"):
+        out[k] = getattr(r, k)
+    out["err_pdf"] = np.array(r.err_pdf[:nb], dtype=np.uint64)
+    out["pwr_pdf"] = np.array(r.pwr_pdf[:nb], dtype=np.uint64)
     out["kernel_ms"] = list(r.kernel_ms)
     return out
 

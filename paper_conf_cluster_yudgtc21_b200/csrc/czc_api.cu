@@ -22,6 +22,8 @@ namespace czc {
 cudaError_t launch_p1(const float* x, const float* y, int64_t n, int grid_cap, P1State* parts,
                       DevResults* res, unsigned int* ticket, cudaStream_t st);
 cudaError_t launch_p1_combine(const P1State* states, int count, DevResults* res, cudaStream_t st);
+cudaError_t launch_pdf(const float* x, const float* y, int64_t n, int nb, int grid_cap, DevResults* res,
+                       cudaStream_t st);
 int p1_max_blocks_per_sm();
 int64_t deriv_blocks(const Field3& s, int zchunk);
 int64_t ac_blocks(const Field3& s, int T);
@@ -102,6 +104,7 @@ static czc_status validate_config(const czc_config& c) {
   if (c.nranks > 1 && (c.rank < 0 || c.rank >= c.nranks || !c.nccl_uid)) return CZC_ERR_INVALID;
   if (c.nccl_uid && (c.nranks < 1 || c.rank < 0 || c.rank >= c.nranks)) return CZC_ERR_INVALID;
   if (c.loopback_slabs < 0 || (c.loopback_slabs > 1 && (c.nranks > 1 || c.nccl_uid))) return CZC_ERR_INVALID;
+  if (c.pdf_bins < 0 || c.pdf_bins > CZC_PDF_MAX_BINS) return CZC_ERR_INVALID;
   return CZC_OK;
 }
 
@@ -201,7 +204,8 @@ struct Plan {
   int win3[3] = {1, 1, 1};
   int kind = 0;                   // 3, 2, 1 (active axes of the SSIM window)
   int T = 10;
-  bool run_p1 = false, run_deriv = false, run_ac = false, run_ssim = false;
+  int nb = 100;                   // PDF bins
+  bool run_p1 = false, run_deriv = false, run_ac = false, run_ssim = false, run_pdf = false;
   int32_t win_in[3] = {0, 0, 0}, step_in[3] = {0, 0, 0};  // reported per input axis
 };
 
@@ -222,7 +226,9 @@ czc_status make_plan(const czc_config& c, int ndim, const int64_t* dims, uint64_
   P.run_ssim = (mask & CZC_M_SSIM) != 0;
   P.run_deriv = (mask & CZC_M_DERIV) != 0;
   P.run_ac = (mask & CZC_M_AUTOCORR) != 0;
-  P.run_p1 = (mask & (CZC_M_P1 | CZC_M_AUTOCORR)) != 0 || (P.run_ssim && c.ssim_range_mode == 1);
+  P.run_pdf = (mask & CZC_M_PDF) != 0;
+  P.nb = c.pdf_bins ? c.pdf_bins : 100;
+  P.run_p1 = (mask & (CZC_M_P1 | CZC_M_AUTOCORR | CZC_M_PDF)) != 0 || (P.run_ssim && c.ssim_range_mode == 1);
   for (int i = 0; i < ndim; i++) {
     const int w = c.ssim_window[i] ? c.ssim_window[i] : 8;
     const int s = c.ssim_step[i] ? c.ssim_step[i] : 1;
@@ -295,6 +301,9 @@ void combine_and_finish(const Plan& P, const Record* recs, int nrec, uint64_t ma
     for (int w = 0; w < kAcWalks; w++)
       for (int k = 0; k < kAcSlots; k++) R.ac[w][k] += recs[r].ac[w][k];
     for (int k = 0; k < kSsimSlots; k++) R.ssim[k] += recs[r].ssim[k];
+    if (P.run_pdf)
+      for (int h = 0; h < 2; h++)
+        for (int b = 0; b < P.nb; b++) R.pdf[h][b] += recs[r].pdf[h][b];
   }
   uint64_t done = 0;
   if (P.run_p1 && (mask & CZC_M_P1)) { finish_p1(R.p1, out); done |= CZC_M_P1; }
@@ -345,6 +354,18 @@ void combine_and_finish(const Plan& P, const Record* recs, int nrec, uint64_t ma
     out->ssim = R.ssim[1] > 0 ? R.ssim[0] / R.ssim[1] : NAN;
     out->n_ssim_exact = (uint64_t)R.ssim[2];
     done |= CZC_M_SSIM;
+  }
+  if (P.run_pdf) {
+    // the ranges are the global P1 extrema, computed exactly as on the device (pdf_range)
+    const PdfRange re = pdf_range(R.p1.emin, R.p1.emax, P.nb);
+    const PdfRange rp = pdf_range(R.p1.pmin, R.p1.pmax, P.nb);
+    out->pdf_bins = P.nb;
+    out->err_pdf_lo = re.lo;
+    out->err_pdf_width = re.w;
+    out->pwr_pdf_lo = R.p1.npwr > 0 ? rp.lo : NAN;
+    out->pwr_pdf_width = R.p1.npwr > 0 ? rp.w : NAN;
+    for (int b = 0; b < P.nb; b++) { out->err_pdf[b] = R.pdf[0][b]; out->pwr_pdf[b] = R.pdf[1][b]; }
+    done |= CZC_M_PDF;
   }
   out->computed_mask = done;
 }
@@ -465,10 +486,12 @@ static czc_status assess_single(czc_ctx* ctx, const Plan& P, const float* x, con
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
   czc_status st = p1_local(ctx, P, x, y, F.nz * F.ny * F.nx);
   if (st != CZC_OK) return st;
+  if (P.run_pdf) CZC_CUDA(ctx, launch_pdf(x, y, F.nz * F.ny * F.nx, P.nb, ctx->p1_grid_cap, ctx->dres, s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
   if ((st = run_p23(ctx, P, F, sp)) != CZC_OK) return st;
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
-  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, &ctx->dres->rec, sizeof(Record), cudaMemcpyDeviceToHost, s));
+  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, &ctx->dres->rec, P.run_pdf ? sizeof(Record) : kRecordNoPdf,
+                                cudaMemcpyDeviceToHost, s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[5], s));
   CZC_CUDA(ctx, cudaStreamSynchronize(s));
   combine_and_finish(P, ctx->hrec, 1, mask, out);
@@ -559,6 +582,8 @@ static czc_status assess_loopback(czc_ctx* ctx, const Plan& P, const float* x, c
       CZC_CUDA(ctx, cudaMemcpyAsync(xhi, x + (z0 + nzl) * plane, hhi * pb, cudaMemcpyDeviceToDevice, s));
       CZC_CUDA(ctx, cudaMemcpyAsync(yhi, y + (z0 + nzl) * plane, hhi * pb, cudaMemcpyDeviceToDevice, s));
     }
+    if (P.run_pdf)
+      CZC_CUDA(ctx, launch_pdf(x + z0 * plane, y + z0 * plane, nzl * plane, P.nb, ctx->p1_grid_cap, ctx->dres, s));
     if ((st = run_p23(ctx, P, F, sp)) != CZC_OK) return st;
     CZC_CUDA(ctx, cudaMemcpyAsync(drec[k].deriv, ctx->dres->rec.deriv,
                                   sizeof(Record) - offsetof(Record, deriv), cudaMemcpyDeviceToDevice, s));
@@ -629,6 +654,7 @@ static czc_status assess_ranks(czc_ctx* ctx, const Plan& P, const float* x, cons
     if (!comm_allgather(ctx->comm, &ctx->dres->rec.p1, ctx->dstates, sizeof(P1State), s, &ctx->last_error)) return CZC_ERR_COMM;
     CZC_CUDA(ctx, launch_p1_combine((const P1State*)ctx->dstates, nranks, ctx->dres, s));
   }
+  if (P.run_pdf) CZC_CUDA(ctx, launch_pdf(x, y, nzl * plane, P.nb, ctx->p1_grid_cap, ctx->dres, s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
   if ((st = run_p23(ctx, P, F, sp)) != CZC_OK) return st;
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
@@ -752,6 +778,10 @@ static czc_status assess_host_pipelined(czc_ctx* ctx, const Plan& P, const float
   }
   for (int j = waited + 1; j < K; j++) CZC_CUDA(ctx, cudaStreamWaitEvent(s, ctx->copy_ev[0][j], 0));
   if (P.run_p1) CZC_CUDA(ctx, launch_p1_combine(dst, K, ctx->dres, s));
+  if (P.run_pdf) {
+    CZC_CUDA(ctx, launch_pdf(x, y, nz * plane, P.nb, ctx->p1_grid_cap, ctx->dres, s));
+    CZC_CUDA(ctx, cudaMemcpyAsync(drec[0].pdf, ctx->dres->rec.pdf, sizeof(drec[0].pdf), cudaMemcpyDeviceToDevice, s));
+  }
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
   if (P.run_ac) {

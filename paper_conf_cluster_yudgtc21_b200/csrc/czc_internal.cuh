@@ -7,6 +7,7 @@
 
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stddef.h>
 #include <string.h>
 
 #include "../../include/czc.h"
@@ -118,7 +119,26 @@ struct Record {
   double deriv[kDerivSlots];
   double ac[kAcWalks][kAcSlots];
   double ssim[kSsimSlots];
+  unsigned long long pdf[2][CZC_PDF_MAX_BINS];   // error / pwr-error PDF counts (CZC_M_PDF); last
 };
+// bytes of a Record that carry results when no PDF was requested (the D2H copy stops there)
+constexpr size_t kRecordNoPdf = offsetof(Record, pdf);
+
+// PDF bin of v (reading R24; the oracle implements the same definition): equal-width bins of
+// width w = (hi - lo) / nb starting at lo, b = floor((v - lo) / w) in IEEE double with the top
+// edge clamped into the last bin; w == 0 (all values equal) or a non-finite w gives bin 0.
+struct PdfRange {
+  double lo, w, rw;                  // rw = 1 / w (IEEE), for the fast path
+  int nb;
+};
+__host__ __device__ inline PdfRange pdf_range(double lo, double hi, int nb) {
+  PdfRange r;
+  r.lo = lo;
+  r.nb = nb;
+  r.w = (hi - lo) / (double)nb;
+  r.rw = r.w > 0 && r.w < dinf() ? 1.0 / r.w : 0.0;
+  return r;
+}
 
 // Device-side results of one launch sequence.  The kernels write `rec`; the AC and SSIM kernels
 // read `p1g`, the GLOBAL P1 state (single GPU: a copy of rec.p1; slab mode: the rank-ordered

@@ -250,6 +250,95 @@ cudaError_t launch_p1(const float* x, const float* y, int64_t n, int grid_cap, P
   return cudaGetLastError();
 }
 
+// ------------------------------------------------------------------------------------------------
+// Error PDF / pwr-error PDF (Table I Category I, L107; reading R24).  One pass after P1: the bins
+// span the GLOBAL extrema found by P1 (res->p1g), so the counts need no second scan.  Every block
+// keeps a shared-memory histogram of 32-bit counters and folds it into the 64-bit device counts
+// with one global atomicAdd per non-empty bin (integer sums: order-independent, deterministic).
+// Bin index: fast path q = (v - lo) * (1/w); when q lies within a relative 1e-10 of a bin edge,
+// the IEEE quotient (v - lo) / w decides (|q - RN((v - lo) / w)| <= ~2 ulp of q), so every count
+// is bit-exact with the oracle's floor((v - lo) / w).  The pwr value is |e| * rcp(|x|) (relative
+// error < 1e-12, see acc_elem); near an edge the IEEE |e| / |x| is formed first.
+// ------------------------------------------------------------------------------------------------
+__device__ __forceinline__ int pdf_clamp(double q, int nb) {
+  const int b = (int)floor(q);
+  return b >= nb ? nb - 1 : (b < 0 ? 0 : b);
+}
+__device__ __forceinline__ bool pdf_near_edge(double q, double tol) {
+  const double f = floor(q);
+  return q - f < tol || f + 1.0 - q < tol;
+}
+__device__ __forceinline__ int pdf_bin_err(double e, const PdfRange& r) {
+  if (!(r.rw > 0)) return 0;
+  const double q = (e - r.lo) * r.rw;                 // e >= lo
+  if (pdf_near_edge(q, 1e-10 * (q + 1.0))) return pdf_clamp((e - r.lo) / r.w, r.nb);
+  return pdf_clamp(q, r.nb);
+}
+__device__ __forceinline__ int pdf_bin_pwr(double ae, double ax, const PdfRange& r) {
+  if (!(r.rw > 0)) return 0;
+  const double qa = ae * rcp_newton1(ax);
+  const double t = (qa - r.lo) * r.rw;
+  if (pdf_near_edge(t, 1e-10 * (fabs(qa) * r.rw + 1.0))) return pdf_clamp((ae / ax - r.lo) / r.w, r.nb);
+  return pdf_clamp(t, r.nb);
+}
+
+template <bool VEC>
+__global__ void __launch_bounds__(kP1Threads)
+pdf_kernel(const float* __restrict__ x, const float* __restrict__ y, int64_t n, int64_t head, int nb,
+           DevResults* __restrict__ res) {
+  __shared__ unsigned int h[2][CZC_PDF_MAX_BINS];
+  for (int i = threadIdx.x; i < 2 * CZC_PDF_MAX_BINS; i += blockDim.x) (&h[0][0])[i] = 0u;
+  __syncthreads();
+  const P1State& g = res->p1g;
+  const PdfRange re = pdf_range(g.emin, g.emax, nb);
+  const PdfRange rp = pdf_range(g.pmin, g.pmax, nb);
+  auto elem = [&](float xf, float yf) {
+    const double xd = xf, e = (double)yf - xd;
+    atomicAdd(&h[0][pdf_bin_err(e, re)], 1u);
+    if (xf != 0.0f) atomicAdd(&h[1][pdf_bin_pwr(fabs(e), fabs(xd), rp)], 1u);
+  };
+  const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
+  if (VEC) {
+    const int64_t nvec = (n - head) / 4, tail0 = head + 4 * nvec;
+    const float4* x4 = reinterpret_cast<const float4*>(x + head);
+    const float4* y4 = reinterpret_cast<const float4*>(y + head);
+    for (int64_t v = gtid; v < nvec; v += gsz) {
+      const float4 a = ld_stream_f4(x4 + v), b = ld_stream_f4(y4 + v);
+      elem(a.x, b.x); elem(a.y, b.y); elem(a.z, b.z); elem(a.w, b.w);
+    }
+    if (gtid < head) elem(x[gtid], y[gtid]);
+    if (gtid < n - tail0) elem(x[tail0 + gtid], y[tail0 + gtid]);
+  } else {
+    for (int64_t i = gtid; i < n; i += gsz) elem(x[i], y[i]);
+  }
+  __syncthreads();
+  unsigned long long* out = &res->rec.pdf[0][0];
+  for (int i = threadIdx.x; i < nb; i += blockDim.x) {
+    if (h[0][i]) atomicAdd(out + i, (unsigned long long)h[0][i]);
+    if (h[1][i]) atomicAdd(out + CZC_PDF_MAX_BINS + i, (unsigned long long)h[1][i]);
+  }
+}
+
+// Zeroes the counts, then histograms x[0, n), y[0, n) into res->rec.pdf (needs res->p1g).
+cudaError_t launch_pdf(const float* x, const float* y, int64_t n, int nb, int grid_cap, DevResults* res,
+                       cudaStream_t st) {
+  cudaError_t e = cudaMemsetAsync(res->rec.pdf, 0, sizeof(res->rec.pdf), st);
+  if (e != cudaSuccess) return e;
+  const uintptr_t ax = reinterpret_cast<uintptr_t>(x), ay = reinterpret_cast<uintptr_t>(y);
+  const bool vec = (ax % 16) == (ay % 16) && (ax % 4) == 0;
+  int64_t head = 0;
+  if (vec) head = (int64_t)(((16 - ax % 16) % 16) / 4);
+  if (head > n) head = n;
+  const int64_t work = vec ? ((n - head) / 4 + 8) : n;
+  int64_t blocks = (work + kP1Threads - 1) / kP1Threads;
+  if (blocks > grid_cap) blocks = grid_cap;
+  if (blocks < 1) blocks = 1;
+  if (vec) pdf_kernel<true><<<(unsigned)blocks, kP1Threads, 0, st>>>(x, y, n, head, nb, res);
+  else pdf_kernel<false><<<(unsigned)blocks, kP1Threads, 0, st>>>(x, y, n, head, nb, res);
+  return cudaGetLastError();
+}
+
 // Slab mode: merge the allgathered per-rank states in rank order (every rank runs the same code
 // on the same bytes, so all ranks hold identical results).
 __global__ void p1_combine_kernel(const P1State* __restrict__ states, int count, DevResults* __restrict__ res) {

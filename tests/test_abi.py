@@ -33,11 +33,11 @@ def test_exports_every_declared_symbol(czc):
 
 
 def test_struct_layout_and_version(czc):
-    assert czc.lib.czc_abi_version() == 1
+    assert czc.lib.czc_abi_version() == 2
     for what, st in ((0, czc.Config), (1, czc.Shape), (2, czc.Result)):
         assert czc.lib.czc_sizeof(what) == ctypes.sizeof(st)
     assert czc.lib.czc_sizeof(7) == 0
-    assert 0 < czc.lib.czc_sizeof(3) < 4096
+    assert 0 < czc.lib.czc_sizeof(3) < 8192
     assert czc.lib.czc_has_nccl() in (0, 1)
 
 
@@ -54,6 +54,8 @@ def test_validation_without_gpu(czc):
     bad = czc.make_config(ac_max_lag=czc.MAX_LAG + 1)
     assert czc.lib.czc_init(ctypes.byref(h), ctypes.byref(bad)) == 1
     bad = czc.make_config(ssim_range_mode=3)
+    assert czc.lib.czc_init(ctypes.byref(h), ctypes.byref(bad)) == 1
+    bad = czc.make_config(pdf_bins=czc.PDF_MAX_BINS + 1)
     assert czc.lib.czc_init(ctypes.byref(h), ctypes.byref(bad)) == 1
     bad = czc.make_config(nranks=2, rank=0)                           # no NCCL uid
     assert czc.lib.czc_init(ctypes.byref(h), ctypes.byref(bad)) == 1

@@ -26,7 +26,28 @@ def _czc():
 
 
 # Record layout (mirrors czc_internal.cuh `Record`): P1State {n, mx, my, me, m2x, m2y, cxy, m2e, sae,
-# emin, emax, pmin, pmax, spwr, npwr : double; xmin, xmax : float}, deriv[25], ac[3][16], ssim[3].
+# emin, emax, pmin, pmax, spwr, npwr : double; xmin, xmax : float}, deriv[25], ac[3][16], ssim[3],
+# pdf[2][256] (uint64 counts of the error / pwr-error PDFs, binned over the GLOBAL ranges).
+PDF_MAX = 256
+
+
+def pdf_counts(x, y, xg, yg, nb):
+    """Counts of this slab's values in the bins of the whole field (reading R24's bin rule)."""
+    def bins(v, lo, hi):
+        w = (hi - lo) / nb
+        if not (w > 0):
+            return np.zeros(v.shape, dtype=np.int64)
+        b = np.floor((v - lo) / w).astype(np.int64)
+        return np.clip(b, 0, nb - 1)
+    e = y.astype(np.float64).ravel() - x.astype(np.float64).ravel()
+    eg = yg.astype(np.float64).ravel() - xg.astype(np.float64).ravel()
+    nzg = xg.ravel() != 0
+    qg = np.abs(eg[nzg]) / np.abs(xg.astype(np.float64).ravel()[nzg])
+    nz = x.ravel() != 0
+    q = np.abs(e[nz]) / np.abs(x.astype(np.float64).ravel()[nz])
+    ce = np.bincount(bins(e, eg.min(), eg.max()), minlength=PDF_MAX)
+    cp = np.bincount(bins(q, qg.min(), qg.max()), minlength=PDF_MAX) if q.size else np.zeros(PDF_MAX, np.int64)
+    return struct.pack(f"<{2 * PDF_MAX}Q", *[int(v) for v in ce], *[int(v) for v in cp])
 def p1_state(x, y):
     xd, yd = x.astype(np.float64).ravel(), y.astype(np.float64).ravel()
     e = yd - xd
@@ -59,7 +80,7 @@ def deriv_fields(f):
     return [out["der1"], out["der2"], np.sqrt(out["g2"]), out["div"], out["lap"]]
 
 
-def record(x, y, z0, z1, w, T=10):
+def record(x, y, z0, z1, w, T=10, nb=0):
     """The record of slab [z0, z1) computed with numpy from the whole field (ownership rules)."""
     nz = x.shape[0]
     rec = p1_state(x[z0:z1], y[z0:z1])
@@ -96,6 +117,7 @@ def record(x, y, z0, z1, w, T=10):
                 s += oracle.ssim_window(x, y, [oz, oy, ox], [w, w, w])
                 cnt += 1
     rec += struct.pack("<3d", s, float(cnt), 0.0)
+    rec += pdf_counts(x[z0:z1], y[z0:z1], x, y, nb) if nb else bytes(16 * PDF_MAX)
     return rec
 
 
@@ -134,6 +156,24 @@ def test_combine_matches_oracle(orc, cuts):
     cfg = czc.make_config(ndim=3, ssim_window=w, ac_max_lag=10)
     g = czc.czc_combine(recs, len(cuts) - 1, xn.shape, cfg)
     compare(g, oracle_all(xn, yn, w))
+
+
+def test_combine_pdf_counts(orc):
+    """Per-slab PDF counts over the global ranges, summed in slab order, equal the oracle's."""
+    czc = _czc()
+    import oracle
+    x, y = synth.make_pair(synth.config("C2q", dims=(10, 9, 12)))
+    xn, yn = x.numpy(), y.numpy()
+    w, nb = 3, 37
+    cuts = (0, 4, 10)
+    recs = b"".join(record(xn, yn, a, b, w, nb=nb) for a, b in zip(cuts[:-1], cuts[1:]))
+    cfg = czc.make_config(ndim=3, ssim_window=w, ac_max_lag=10, pdf_bins=nb)
+    g = czc.czc_combine(recs, len(cuts) - 1, xn.shape, cfg, czc.M_FULL)
+    o = oracle.pdf(xn, yn, nb)
+    assert g["computed_mask"] == czc.M_FULL and g["pdf_bins"] == nb
+    assert np.array_equal(g["err_pdf"], o["err_pdf"]) and np.array_equal(g["pwr_pdf"], o["pwr_pdf"])
+    for k in ("err_pdf_lo", "err_pdf_width", "pwr_pdf_lo", "pwr_pdf_width"):
+        assert g[k] == o[k], k
 
 
 def _worker(rank, world, port, out_q):

@@ -393,3 +393,59 @@ def test_plane_tile_edges(czc, orc, dims, lag):
     errors = []
     check_ac(g["ac"], g["ac_count"], o["ac"], o["ac_count"], errors)
     report(errors)
+
+
+# ---------------------------------------------------------------- error PDF / pwr-error PDF (f1)
+def pdf_check(g, o, nb):
+    """Counts are bit-exact (the bin rule is the same IEEE arithmetic on both sides, R24)."""
+    assert g["pdf_bins"] == nb
+    assert np.array_equal(g["err_pdf"], o["err_pdf"]), (g["err_pdf"] - o["err_pdf"].astype(np.int64))
+    assert np.array_equal(g["pwr_pdf"], o["pwr_pdf"]), (g["pwr_pdf"] - o["pwr_pdf"].astype(np.int64))
+    for k in ("err_pdf_lo", "err_pdf_width", "pwr_pdf_lo", "pwr_pdf_width"):
+        assert g[k] == o[k] or (math.isnan(g[k]) and math.isnan(o[k])), (k, g[k], o[k])
+
+
+@pytest.mark.parametrize("cfg,dims,nb", [("C1", (30, 41, 53), 100), ("C2", (20, 90, 130), 256),
+                                         ("C2q", (17, 60, 77), 64), ("C3", (25, 33, 47), 7),
+                                         ("C4", (180, 360), 1), ("C1", (1001,), 13)])
+def test_pdf_counts(czc, orc, cfg, dims, nb):
+    x, y = synth.make_pair(synth.config(cfg, dims=dims))
+    xn, yn = x.numpy(), y.numpy()
+    with czc.Assessor(ndim=xn.ndim, pdf_bins=nb) as a:
+        g = a.assess(torch.from_numpy(xn).cuda(), torch.from_numpy(yn).cuda(), czc.M_PDF | czc.M_P1)
+    assert g["computed_mask"] == czc.M_PDF | czc.M_P1
+    pdf_check(g, orc.pdf(xn, yn, nb), nb)
+
+
+def test_pdf_edge_values_and_degenerate(czc, orc):
+    """Errors exactly on bin edges (dyadic construction), a constant error and misaligned views."""
+    k = np.repeat(np.arange(17), np.arange(1, 18))
+    x = np.ones(k.size, np.float32)
+    y = (1.0 + k / 16.0).astype(np.float32)
+    for xs, ys in ((x, y), (x, x + np.float32(2.0 ** -10))):
+        with czc.Assessor(ndim=1, pdf_bins=4) as a:
+            g = a.assess(torch.from_numpy(xs).cuda(), torch.from_numpy(ys).cuda(), czc.M_PDF)
+        pdf_check(g, orc.pdf(xs, ys, 4), 4)
+    xa, ya = synth.make_pair(synth.config("C2q", dims=(9, 40, 51)))
+    xd, yd = xa.cuda().reshape(-1), ya.cuda().reshape(-1)
+    for off in (1, 3):
+        xv, yv = xd[off:].contiguous(), yd[off:].clone()
+        xv = xd[off:]                                        # misaligned view (scalar prologue)
+        yv = yd[off:]
+        with czc.Assessor(ndim=1, pdf_bins=50) as a:
+            g = a.assess(xv, yv, czc.M_PDF)
+        pdf_check(g, orc.pdf(xv.cpu().numpy(), yv.cpu().numpy(), 50), 50)
+
+
+def test_pdf_slab_and_host_paths(czc, orc):
+    """Loopback slab mode and the pipelined host path give the single-GPU counts."""
+    x, y = synth.make_pair(synth.config("C2", dims=(40, 50, 60)))
+    xn, yn = x.numpy(), y.numpy()
+    o = orc.pdf(xn, yn, 100)
+    for kw in ({"loopback_slabs": 3}, {}):
+        with czc.Assessor(ndim=3, pdf_bins=100, **kw) as a:
+            g = a.assess(torch.from_numpy(xn).cuda(), torch.from_numpy(yn).cuda(), czc.M_FULL)
+            h = a.assess_host(xn, yn, czc.M_FULL)
+        pdf_check(g, o, 100)
+        pdf_check(h, o, 100)
+        assert g["computed_mask"] == czc.M_FULL

@@ -319,3 +319,64 @@ class TestSSIM:
         x = dyadic_field((5, 5, 5))
         s, nw = orc.ssim(x, x, [6, 6, 6])
         assert nw == 0 and math.isnan(s)
+
+
+# ----------------------------------------------------------------------------------------- PDF
+class TestPdf:
+    """Error PDF / pwr-error PDF (Table I Category I, L107), bin rule of reading R24."""
+
+    def test_constructed_bin_counts(self, orc):
+        """e = k/16, k = 0..16 with multiplicity m_k, x = 1: lo = 0, w = 1/4, bin = floor(k/4) with
+        k = 16 clamped into the last bin -> counts are sums of m_k by hand (closed form)."""
+        m = np.arange(1, 18)                               # multiplicities 1..17
+        k = np.repeat(np.arange(17), m)
+        x = np.ones(k.size, np.float32)
+        y = (1.0 + k / 16.0).astype(np.float32)            # exact in float32
+        r = orc.pdf(x, y, 4)
+        assert r["err_pdf_lo"] == 0.0 and r["err_pdf_width"] == 0.25
+        want = [m[0:4].sum(), m[4:8].sum(), m[8:12].sum(), m[12:17].sum()]
+        assert r["err_pdf"].tolist() == want
+        # pwr = |e| / 1 = e: the same bins
+        assert r["pwr_pdf"].tolist() == want and r["n_pwr"] == k.size
+
+    def test_constant_error_single_bin(self, orc):
+        """Dyadic constant offset: every error equal -> width 0, all counts in bin 0."""
+        x = dyadic_field((5, 6, 7)).ravel()
+        x[x == 0] = 2.0 ** -12
+        y = x + np.float32(2.0 ** -10)
+        r = orc.pdf(x, y, 10)
+        assert r["err_pdf_width"] == 0.0 and r["err_pdf"][0] == x.size and r["err_pdf"][1:].sum() == 0
+
+    def test_numpy_histogram_edge_free(self, orc):
+        """numpy.histogram implements equal-width bins independently; on data with no value
+        within 1e-6 of a bin edge the counts must agree exactly."""
+        x = (1.0 + rng.random(20000)).astype(np.float32)
+        y = (x + rng.uniform(-1e-3, 1e-3, x.size)).astype(np.float32)
+        e = y.astype(np.float64) - x.astype(np.float64)
+        nb = 50
+        lo, hi = e.min(), e.max()
+        t = (e - lo) / ((hi - lo) / nb)
+        keep = (np.abs(t - np.round(t)) > 1e-6) | (e == lo) | (e == hi)
+        r = orc.pdf(x[keep], y[keep], nb)
+        want, edges = np.histogram(e[keep], bins=nb, range=(lo, hi))
+        assert r["err_pdf"].tolist() == want.tolist()
+        assert r["err_pdf_lo"] == lo and r["err_pdf_width"] == (hi - lo) / nb
+
+    def test_totals_and_zero_originals(self, orc):
+        """Counts total n (error PDF) and n_pwr = #{x != 0} (pwr PDF, reading R3)."""
+        x, y = synth.make_pair(synth.config("C2q", dims=(6, 20, 30)))
+        xn, yn = x.numpy().ravel(), y.numpy().ravel()
+        r = orc.pdf(xn, yn, 33)
+        assert int(r["err_pdf"].sum()) == xn.size
+        assert r["n_pwr"] == int((xn != 0).sum()) == int(r["pwr_pdf"].sum())
+        assert r["err_pdf"][0] > 0 and r["err_pdf"][-1] > 0    # the extrema fill the end bins
+        q = np.abs(yn.astype(np.float64) - xn)[xn != 0] / np.abs(xn[xn != 0].astype(np.float64))
+        assert r["pwr_pdf_lo"] == q.min() and r["pwr_pdf_width"] == (q.max() - q.min()) / 33
+
+    def test_no_nonzero_original(self, orc):
+        """All x == 0: no pwr values -> pwr range NaN, counts 0 (reading R3)."""
+        x = np.zeros(100, np.float32)
+        y = rng.uniform(-1, 1, 100).astype(np.float32)
+        r = orc.pdf(x, y, 8)
+        assert r["n_pwr"] == 0 and math.isnan(r["pwr_pdf_lo"]) and r["pwr_pdf"].sum() == 0
+        assert int(r["err_pdf"].sum()) == 100
