@@ -207,6 +207,7 @@ def run_ours(args, rank, world, local):
         torch.cuda.synchronize(dev)
 
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)   # 256 MB > L2
+    clean = torch.zeros(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)   # read-only after this
     for _ in range(args.warmup):
         a.assess(xd, yd, czc.M_ALL, **kw)
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
@@ -218,8 +219,9 @@ def run_ours(args, rank, world, local):
     t_wall = time.perf_counter()
     for i in range(args.steps):
         flush.zero_()                                   # L2 flush between timed steps (not timed):
-        flush.sum()                                     # write 256 MB, then read it back so the
-                                                        # dirty lines drain before the step starts
+        clean.sum()                                     # write 256 MB, then read ANOTHER 256 MB so
+                                                        # the dirty lines are written back before the
+                                                        # step starts and L2 holds only clean lines
         ev[i][0].record(stream)
         r = a.assess(xd, yd, czc.M_ALL, **kw)
         ev[i][1].record(stream)
@@ -253,6 +255,10 @@ def run_ours(args, rank, world, local):
     # end-to-end through the public host-buffer entry point (H2D + kernels + D2H inside)
     e2e = None
     if not args.no_e2e:
+        # czc_assess_host pipelines K = min(8, nz / halo) z-chunks (halo = max(1, T, W - 1) = 10)
+        # and copies back one record prefix per chunk (czc_sizeof(4) bytes each)
+        K = min(8, nz_local // 10) if world == 1 else world
+        d2h_host = int(czc.get_lib().czc_sizeof(4)) * (K if K >= 2 else 1)
         xp = xh.pin_memory()
         yp = yh.pin_memory()
         for _ in range(2):
@@ -273,7 +279,7 @@ def run_ours(args, rank, world, local):
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             e_tot = float(t.item())
         e2e = {"value": round(world * nbytes_rank * nsteps_e2e / (e_tot * 1e-3) / 1e9, 3), "unit": UNIT,
-               "h2d_bytes_per_step": nbytes_rank, "d2h_bytes_per_step": int(czc.get_lib().czc_sizeof(3)),
+               "h2d_bytes_per_step": nbytes_rank, "d2h_bytes_per_step": d2h_host,
                "ms_per_step": round(e_tot / nsteps_e2e, 4)}
 
     cpu = None
@@ -292,7 +298,8 @@ def run_ours(args, rank, world, local):
                                    f"float32 pair, abs eb {spec.eb:g}, full metric set (P1, derivatives, "
                                    f"AC lags 1..10, SSIM 8^3 step 1)",
                        "per_rank_planes": nz_local, "parallelism": f"slab{world}",
-                       "l2": "flushed between timed steps (256 MB write + read-back, outside the step events)"},
+                       "l2": "flushed between timed steps (256 MB write + 256 MB read of another buffer, "
+                                 "outside the step events); the pair (200 MB) is also larger than L2"},
             "per_pattern_ms": {k: round(v, 4) for k, v in shares.items()},
             "per_pattern_gbs": {k: round(alg_bytes / (v * 1e-3) / 1e9, 2) for k, v in shares.items() if v > 0},
             "roofline": {"bound": "hbm", "kernel": dom, "achieved": round(achieved, 2), "peak": peak,

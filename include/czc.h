@@ -189,7 +189,9 @@ int czc_abi_version(void);
 int czc_has_nccl(void);
 
 /* sizeof(czc_config) (what = 0), sizeof(czc_shape) (1), sizeof(czc_result) (2), size of one
- * partial record = bytes copied device->host per single-GPU czc_assess call (3); 0 otherwise.  Lets bindings verify their struct mirrors
+ * partial record (3: what czc_combine consumes per slab), bytes of a record copied device->host
+ * when no PDF is requested (4: one record per single-GPU czc_assess call, one per slab / z-chunk
+ * in slab mode and czc_assess_host); 0 otherwise.  Lets bindings verify their struct mirrors
  * against the compiled library. */
 uint64_t czc_sizeof(int what);
 

@@ -82,7 +82,7 @@ extern "C" int czc_abi_version(void) { return CZC_ABI_VERSION; }
 extern "C" int czc_has_nccl(void) { return comm_available(); }
 extern "C" uint64_t czc_sizeof(int what) {
   return what == 0 ? sizeof(czc_config) : what == 1 ? sizeof(czc_shape) : what == 2 ? sizeof(czc_result)
-       : what == 3 ? sizeof(Record) : 0;
+       : what == 3 ? sizeof(Record) : what == 4 ? kRecordNoPdf : 0;
 }
 
 static czc_status cuda_fail(czc_ctx* ctx, cudaError_t e, const char* where) {
@@ -458,6 +458,14 @@ static czc_status run_p23(czc_ctx* ctx, const Plan& P, const Field3& F, const Ss
   return CZC_OK;
 }
 
+// D2H copy of n consecutive records; without PDFs only the first kRecordNoPdf bytes of each
+// (one strided copy).
+static cudaError_t copy_records(Record* h, const Record* d, int n, bool pdf, cudaStream_t s) {
+  if (pdf) return cudaMemcpyAsync(h, d, (size_t)n * sizeof(Record), cudaMemcpyDeviceToHost, s);
+  return cudaMemcpy2DAsync(h, sizeof(Record), d, sizeof(Record), kRecordNoPdf, (size_t)n,
+                           cudaMemcpyDeviceToHost, s);
+}
+
 static czc_status p1_local(czc_ctx* ctx, const Plan& P, const float* x, const float* y, int64_t n) {
   if (!P.run_p1) return CZC_OK;
   czc_status st = ensure_buf(ctx, &ctx->parts, &ctx->parts_cap, (size_t)ctx->p1_grid_cap * sizeof(P1State));
@@ -490,8 +498,7 @@ static czc_status assess_single(czc_ctx* ctx, const Plan& P, const float* x, con
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
   if ((st = run_p23(ctx, P, F, sp)) != CZC_OK) return st;
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
-  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, &ctx->dres->rec, P.run_pdf ? sizeof(Record) : kRecordNoPdf,
-                                cudaMemcpyDeviceToHost, s));
+  CZC_CUDA(ctx, copy_records(ctx->hrec, &ctx->dres->rec, 1, P.run_pdf, s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[5], s));
   CZC_CUDA(ctx, cudaStreamSynchronize(s));
   combine_and_finish(P, ctx->hrec, 1, mask, out);
@@ -589,7 +596,7 @@ static czc_status assess_loopback(czc_ctx* ctx, const Plan& P, const float* x, c
                                   sizeof(Record) - offsetof(Record, deriv), cudaMemcpyDeviceToDevice, s));
   }
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
-  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, drec, (size_t)K * sizeof(Record), cudaMemcpyDeviceToHost, s));
+  CZC_CUDA(ctx, copy_records(ctx->hrec, drec, K, P.run_pdf, s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[5], s));
   CZC_CUDA(ctx, cudaStreamSynchronize(s));
   combine_and_finish(P, ctx->hrec, K, mask, out);
@@ -660,7 +667,7 @@ static czc_status assess_ranks(czc_ctx* ctx, const Plan& P, const float* x, cons
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
   // second small allgather: every rank's record, combined in rank order on the host
   if (!comm_allgather(ctx->comm, &ctx->dres->rec, ctx->dgather, sizeof(Record), s, &ctx->last_error)) return CZC_ERR_COMM;
-  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, ctx->dgather, (size_t)nranks * sizeof(Record), cudaMemcpyDeviceToHost, s));
+  CZC_CUDA(ctx, copy_records(ctx->hrec, (const Record*)ctx->dgather, nranks, P.run_pdf, s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[5], s));
   CZC_CUDA(ctx, cudaStreamSynchronize(s));
   combine_and_finish(P, ctx->hrec, nranks, mask, out);
@@ -794,7 +801,7 @@ static czc_status assess_host_pipelined(czc_ctx* ctx, const Plan& P, const float
   }
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
-  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->hrec, drec, (size_t)K * sizeof(Record), cudaMemcpyDeviceToHost, s));
+  CZC_CUDA(ctx, copy_records(ctx->hrec, drec, K, P.run_pdf, s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[5], s));
   CZC_CUDA(ctx, cudaStreamSynchronize(s));
   combine_and_finish(P, ctx->hrec, K, mask, out);
