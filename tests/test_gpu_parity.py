@@ -449,3 +449,93 @@ def test_pdf_slab_and_host_paths(czc, orc):
         pdf_check(g, o, 100)
         pdf_check(h, o, 100)
         assert g["computed_mask"] == czc.M_FULL
+
+
+# ------------------------------------------------------------ BASELINE full sizes, maximum size
+def _sampled_ssim(orc, xn, yn, d, win, count, seed):
+    rng = np.random.default_rng(seed)
+    nw = d.shape
+    worst = 0.0
+    for _ in range(count):
+        o = [int(rng.integers(0, k)) for k in nw]
+        worst = max(worst, abs(d[tuple(o)] - orc.ssim_window(xn, yn, o, win)))
+    return worst
+
+
+def test_full_size_cesm_2d(czc, orc):
+    """BASELINE configs[3]: 1800 x 3600 2-D field, 8 x 8 windows, lags 1..10: P1 / derivatives /
+    AC against the oracle over the whole field, SSIM on 400 sampled windows + the exact mean."""
+    spec = synth.CONFIGS["C4"]
+    x, y = synth.make_pair(spec)
+    xn, yn = x.numpy(), y.numpy()
+    nw = [n - 8 + 1 for n in xn.shape]
+    dbg = torch.empty(nw, dtype=torch.float64, device="cuda")
+    with czc.Assessor(ndim=2, ssim_window=8, debug_wssim=dbg.data_ptr()) as a:
+        g = a.assess(x.cuda(), y.cuda())
+    errors = []
+    check_p1(g, orc.p1(xn, yn), errors)
+    check_deriv(g, orc.deriv(xn, yn), errors)
+    ac, cnt = orc.autocorr(xn, yn, 10)
+    check_ac(g["ac"], g["ac_count"], ac, cnt, errors)
+    report(errors)
+    d = dbg.cpu().numpy()
+    assert g["n_windows"] == np.prod(nw) and abs(d.mean() - g["ssim"]) < 1e-12
+    assert _sampled_ssim(orc, xn, yn, d, [8, 8], 400, 21) < 1e-6
+
+
+def test_full_size_nyx(czc, orc):
+    """BASELINE configs[2]: 512^3 log-normal pair (1.07 GB), full metric set in the bench launch
+    configuration: P1, derivatives and AC against the oracle over all 134M elements, SSIM on 300
+    sampled windows + the exact mean of the per-window values."""
+    spec = synth.CONFIGS["C3"]
+    x, y = synth.make_pair(spec)
+    xn, yn = x.numpy(), y.numpy()
+    nw = [n - 8 + 1 for n in xn.shape]
+    dbg = torch.empty(nw, dtype=torch.float64, device="cuda")
+    with czc.Assessor(ssim_window=8, debug_wssim=dbg.data_ptr()) as a:
+        g = a.assess(x.cuda(), y.cuda())
+    errors = []
+    check_p1(g, orc.p1(xn, yn), errors)
+    check_deriv(g, orc.deriv(xn, yn), errors)
+    ac, cnt = orc.autocorr(xn, yn, 10)
+    check_ac(g["ac"], g["ac_count"], ac, cnt, errors)
+    report(errors)
+    d = dbg.cpu().numpy()
+    assert g["n_windows"] == np.prod(nw) and abs(d.mean() - g["ssim"]) < 1e-11
+    del dbg
+    assert _sampled_ssim(orc, xn, yn, d, [8, 8, 8], 300, 31) < 1e-6
+
+
+def test_maximum_size_closed_forms(czc):
+    """BASELINE configs[4] size on ONE GPU: a 2048^3 pair (68.7 GB, 8.6e9 elements) with
+    x = v constant and y = v + c (c = 2^-10 exact): every metric has a closed form — e = c,
+    MSE = c^2, R = 0 (PSNR = -inf, reading R4), dF = 0, sigma_e^2 = 0 (AC NaN, R12), and every
+    window has L = 0 -> 1 (R15): SSIM = A / (A + c^2) with A = 2 v (v + c) + 1e-4.  Exercises
+    64-bit element counts, 2^31+ element offsets, the largest grids and the PDF pass."""
+    n = 2048
+    free, _ = torch.cuda.mem_get_info()
+    if free < 2 * n ** 3 * 4 + (4 << 30):
+        pytest.skip(f"needs ~70 GB free device memory, have {free / 2**30:.0f} GiB")
+    v, c = 280.0, 2.0 ** -10
+    x = torch.full((n, n, n), v, dtype=torch.float32, device="cuda")
+    y = torch.full((n, n, n), v + c, dtype=torch.float32, device="cuda")
+    with czc.Assessor(ssim_window=8, pdf_bins=16) as a:
+        g = a.assess(x, y, czc.M_FULL)
+    del x, y
+    torch.cuda.empty_cache()
+    N = n ** 3
+    assert g["computed_mask"] == czc.M_FULL and g["n"] == N
+    assert g["x_min"] == v and g["x_max"] == v and g["value_range"] == 0.0
+    assert g["err_min"] == c and g["err_max"] == c and g["err_maxabs"] == c
+    assert g["mse"] == c * c and g["rmse"] == c and g["psnr"] == -math.inf
+    assert abs(g["err_mean"] - c) <= 1e-15 and g["err_var"] <= 1e-20
+    assert g["n_pwr"] == N and g["pwr_min"] == c / v and g["pwr_max"] == c / v
+    assert math.isnan(g["pearson"])
+    assert g["n_interior"] == (n - 2) ** 3
+    for f in ("der1", "der2", "grad", "div", "lap"):
+        assert g[f + "_maxabs"] == 0 and g[f + "_mse"] == 0 and g[f + "_psnr"] == math.inf, f
+    assert g["ac_count"][10] == (n - 10) ** 3 and all(math.isnan(t) for t in g["ac"][1:])
+    A = 2 * v * (v + c) + 1e-4
+    assert g["n_windows"] == (n - 7) ** 3
+    assert abs(g["ssim"] - A / (A + c * c)) < 1e-12
+    assert g["err_pdf"][0] == N and g["err_pdf_width"] == 0.0 and g["pwr_pdf"][0] == N
