@@ -176,7 +176,7 @@ deriv_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __res
 // owns rows ty and ty + 4.  The 25 accumulators are shared by both points (half the registers
 // per point) and the two independent stencils double each warp's instruction-level parallelism.
 template <int PTS>
-__global__ void __launch_bounds__(kTX * kTY / PTS, 5)
+__global__ void __launch_bounds__(kTX * kTY / PTS, 4)
 deriv3_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
               unsigned int* __restrict__ ticket) {
   constexpr int RY = kTY / PTS;                    // thread rows
