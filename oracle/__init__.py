@@ -78,15 +78,30 @@ def _load():
         UP = ctypes.POINTER(ctypes.c_uint64)
         lib.czco_pdf.argtypes = [P, P, ctypes.c_uint64, ctypes.c_int, DP, DP, UP, DP, DP, UP, UP]
         lib.czco_threads.restype = ctypes.c_int
+        for name in ("czco_p1", "czco_deriv", "czco_autocorr", "czco_ssim_window", "czco_ssim", "czco_pdf"):
+            f32, f64 = getattr(lib, name), getattr(lib, name + "_f64")
+            f64.argtypes = f32.argtypes
+            f64.restype = f32.restype
         _lib = lib
     return _lib
 
 
-def _f32(a) -> np.ndarray:
+def _np(a) -> np.ndarray:
     if hasattr(a, "detach"):
         a = a.detach().cpu().numpy()
-    a = np.ascontiguousarray(a, dtype=np.float32)
-    return a
+    return np.asarray(a)
+
+
+def _pair(x, y):
+    """The pair as C-contiguous arrays of one element type: float64 if either input is float64
+    (NEXT row f3), else float32 (the paper's precision)."""
+    x, y = _np(x), _np(y)
+    dt = np.float64 if np.float64 in (x.dtype, y.dtype) else np.float32
+    return np.ascontiguousarray(x, dtype=dt), np.ascontiguousarray(y, dtype=dt)
+
+
+def _fn(name: str, x: np.ndarray):
+    return getattr(_load(), name + ("_f64" if x.dtype == np.float64 else ""))
 
 
 def _dims(a: np.ndarray, dims=None):
@@ -103,19 +118,19 @@ def threads() -> int:
 
 
 def p1(x, y) -> Dict[str, float]:
-    x, y = _f32(x), _f32(y)
+    x, y = _pair(x, y)
     r = _P1()
-    rc = _load().czco_p1(x.ctypes.data, y.ctypes.data, x.size, ctypes.byref(r))
+    rc = _fn("czco_p1", x)(x.ctypes.data, y.ctypes.data, x.size, ctypes.byref(r))
     if rc:
         raise ValueError(f"czco_p1 failed ({rc})")
     return {k: getattr(r, k) for k, _ in _P1._fields_}
 
 
 def deriv(x, y, dims=None) -> Dict[str, float]:
-    x, y = _f32(x), _f32(y)
+    x, y = _pair(x, y)
     nd, d = _dims(x, dims)
     r = _Deriv()
-    rc = _load().czco_deriv(x.ctypes.data, y.ctypes.data, nd, d, ctypes.byref(r))
+    rc = _fn("czco_deriv", x)(x.ctypes.data, y.ctypes.data, nd, d, ctypes.byref(r))
     if rc:
         raise ValueError(f"czco_deriv failed ({rc})")
     out = {"n_interior": r.n_interior}
@@ -127,32 +142,32 @@ def deriv(x, y, dims=None) -> Dict[str, float]:
 
 def autocorr(x, y, max_lag: int = 10, dims=None):
     """Returns (ac[0..max_lag], count[0..max_lag])."""
-    x, y = _f32(x), _f32(y)
+    x, y = _pair(x, y)
     nd, d = _dims(x, dims)
     ac = (ctypes.c_double * (max_lag + 1))()
     cnt = (ctypes.c_uint64 * (max_lag + 1))()
-    rc = _load().czco_autocorr(x.ctypes.data, y.ctypes.data, nd, d, max_lag, ac, cnt)
+    rc = _fn("czco_autocorr", x)(x.ctypes.data, y.ctypes.data, nd, d, max_lag, ac, cnt)
     if rc:
         raise ValueError(f"czco_autocorr failed ({rc})")
     return np.array(ac[:], dtype=np.float64), np.array(cnt[:], dtype=np.uint64)
 
 
 def ssim_window(x, y, origin, window, range_mode: int = 0, global_range: float = 0.0, dims=None) -> float:
-    x, y = _f32(x), _f32(y)
+    x, y = _pair(x, y)
     nd, d = _dims(x, dims)
-    return float(_load().czco_ssim_window(x.ctypes.data, y.ctypes.data, nd, d, _i64(origin),
+    return float(_fn("czco_ssim_window", x)(x.ctypes.data, y.ctypes.data, nd, d, _i64(origin),
                                           _i64(window), range_mode, global_range))
 
 
 def ssim(x, y, window, step=None, range_mode: int = 0, dims=None):
     """Returns (ssim, n_windows).  window/step: one value per axis (slowest-first)."""
-    x, y = _f32(x), _f32(y)
+    x, y = _pair(x, y)
     nd, d = _dims(x, dims)
     if step is None:
         step = [1] * nd
     out = ctypes.c_double()
     nw = ctypes.c_uint64()
-    rc = _load().czco_ssim(x.ctypes.data, y.ctypes.data, nd, d, _i64(window), _i64(step), range_mode,
+    rc = _fn("czco_ssim", x)(x.ctypes.data, y.ctypes.data, nd, d, _i64(window), _i64(step), range_mode,
                            ctypes.byref(out), ctypes.byref(nw))
     if rc == 3:
         return float("nan"), 0
@@ -164,12 +179,12 @@ def ssim(x, y, window, step=None, range_mode: int = 0, dims=None):
 def pdf(x, y, nbins: int = 100) -> Dict:
     """Error PDF and pwr-error PDF counts (czco_pdf): keys err_pdf_lo/width, err_pdf (counts),
     pwr_pdf_lo/width, pwr_pdf, n_pwr."""
-    x, y = _f32(x), _f32(y)
+    x, y = _pair(x, y)
     d = [ctypes.c_double() for _ in range(4)]
     ec = (ctypes.c_uint64 * nbins)()
     pc = (ctypes.c_uint64 * nbins)()
     npw = ctypes.c_uint64()
-    rc = _load().czco_pdf(x.ctypes.data, y.ctypes.data, x.size, nbins, ctypes.byref(d[0]), ctypes.byref(d[1]),
+    rc = _fn("czco_pdf", x)(x.ctypes.data, y.ctypes.data, x.size, nbins, ctypes.byref(d[0]), ctypes.byref(d[1]),
                           ec, ctypes.byref(d[2]), ctypes.byref(d[3]), pc, ctypes.byref(npw))
     if rc:
         raise ValueError(f"czco_pdf failed ({rc})")
@@ -180,7 +195,7 @@ def pdf(x, y, nbins: int = 100) -> Dict:
 
 def assess(x, y, window=None, step=None, max_lag: int = 10, range_mode: int = 0) -> Dict[str, float]:
     """All oracle metrics in one flat dict keyed like the CUDA binding's result."""
-    x, y = _f32(x), _f32(y)
+    x, y = _pair(x, y)
     nd = x.ndim
     out = dict(p1(x, y))
     out.update(deriv(x, y))

@@ -37,9 +37,21 @@ static int shape3(int ndim, const int64_t* dims, int64_t n3[3]) {
   return 1;
 }
 
+/* An input field: float32 (the paper's precision, L330) or float64 (NEXT row f3).  Every sample
+ * is read as a double (float -> double is exact), so one definition serves both element types. */
+typedef struct {
+  const void* p;
+  int f64;
+} fld_t;
+static inline fld_t fld32(const float* p) { fld_t f = {p, 0}; return f; }
+static inline fld_t fld64(const double* p) { fld_t f = {p, 1}; return f; }
+static inline double V(fld_t f, int64_t i) {
+  return f.f64 ? ((const double*)f.p)[i] : (double)((const float*)f.p)[i];
+}
+
 /* e = recon - orig (reading R1), computed as (double)y - (double)x. */
-static inline double err_of(const float* x, const float* y, int64_t i) {
-  return (double)y[i] - (double)x[i];
+static inline double err_of(fld_t x, fld_t y, int64_t i) {
+  return V(y, i) - V(x, i);
 }
 
 /* ======================================================================================
@@ -47,17 +59,17 @@ static inline double err_of(const float* x, const float* y, int64_t i) {
  * MSE, RMSE, NRMSE, SNR, PSNR; plus north_star's range, max relative error and Pearson.
  * Definitions: SURVEY.md §8(c) C-P1 and readings R1-R6.
  * ====================================================================================== */
-int czco_p1(const float* x, const float* y, uint64_t n, czco_p1_t* r) {
-  if (!x || !y || !r || n == 0) return 1;
+static int p1_impl(fld_t x, fld_t y, uint64_t n, czco_p1_t* r) {
+  if (!x.p || !y.p || !r || n == 0) return 1;
   memset(r, 0, sizeof(*r));
   /* pass 1: extrema, plain sums */
-  float xmin = x[0], xmax = x[0];
+  double xmin = V(x, 0), xmax = xmin;
   double emin = err_of(x, y, 0), emax = emin, emaxabs = fabs(emin);
   double pmin = INFINITY, pmax = -INFINITY;
   uint64_t npwr = 0;
   ld sx = 0, sy = 0, se = 0, sae = 0, spwr = 0;
   for (uint64_t i = 0; i < n; i++) {
-    float xi = x[i];
+    const double xi = V(x, (int64_t)i);
     double e = err_of(x, y, (int64_t)i);
     if (xi < xmin) xmin = xi;
     if (xi > xmax) xmax = xi;
@@ -65,11 +77,11 @@ int czco_p1(const float* x, const float* y, uint64_t n, czco_p1_t* r) {
     if (e > emax) emax = e;
     if (fabs(e) > emaxabs) emaxabs = fabs(e);
     sx += (ld)xi;
-    sy += (ld)y[i];
+    sy += (ld)V(y, (int64_t)i);
     se += (ld)e;
     sae += (ld)fabs(e);
-    if (xi != 0.0f) {                      /* point-wise relative error, x = 0 excluded (R3) */
-      double q = fabs(e) / fabs((double)xi);
+    if (xi != 0.0) {                       /* point-wise relative error, x = 0 excluded (R3) */
+      double q = fabs(e) / fabs(xi);
       if (q < pmin) pmin = q;
       if (q > pmax) pmax = q;
       spwr += (ld)q;
@@ -81,7 +93,7 @@ int czco_p1(const float* x, const float* y, uint64_t n, czco_p1_t* r) {
   /* pass 2: centred second moments */
   ld sxx = 0, syy = 0, sxy = 0, svar = 0, se2 = 0;
   for (uint64_t i = 0; i < n; i++) {
-    ld dx = (ld)x[i] - mx, dy = (ld)y[i] - my;
+    ld dx = (ld)V(x, (int64_t)i) - mx, dy = (ld)V(y, (int64_t)i) - my;
     ld e = (ld)err_of(x, y, (int64_t)i);
     sxx += dx * dx;
     syy += dy * dy;
@@ -92,7 +104,7 @@ int czco_p1(const float* x, const float* y, uint64_t n, czco_p1_t* r) {
   r->n = n;
   r->x_min = xmin;
   r->x_max = xmax;
-  r->value_range = (double)xmax - (double)xmin;      /* R4: range of the original */
+  r->value_range = xmax - xmin;                      /* R4: range of the original */
   r->err_min = emin;
   r->err_max = emax;
   r->err_maxabs = emaxabs;
@@ -118,6 +130,10 @@ int czco_p1(const float* x, const float* y, uint64_t n, czco_p1_t* r) {
   r->err_var = (double)(svar / N);                   /* R6: population variance */
   return 0;
 }
+int czco_p1(const float* x, const float* y, uint64_t n, czco_p1_t* r) { return p1_impl(fld32(x), fld32(y), n, r); }
+int czco_p1_f64(const double* x, const double* y, uint64_t n, czco_p1_t* r) {
+  return p1_impl(fld64(x), fld64(y), n, r);
+}
 
 /* ======================================================================================
  * Pattern 2 — stencil metrics.  Eq. (1): Der = sum_a |f(p+e_a) - f(p-e_a)|;  "the
@@ -125,15 +141,15 @@ int czco_p1(const float* x, const float* y, uint64_t n, czco_p1_t* r) {
  * Alg. 2: central differences /2 and their L2 norm (Grad).  Readings R7, R9, R11:
  * interior points only (1-point border on every active axis), compact second difference.
  * ====================================================================================== */
-static void deriv_point(const float* f, const int64_t n3[3], const int act[3], int64_t z, int64_t yy,
+static void deriv_point(fld_t f, const int64_t n3[3], const int act[3], int64_t z, int64_t yy,
                         int64_t xx, double F[CZCO_NF]) {
   const int64_t st[3] = {n3[1] * n3[2], n3[2], 1};
   const int64_t c = z * st[0] + yy * st[1] + xx;
-  const double f0 = (double)f[c];
+  const double f0 = V(f, c);
   double der1 = 0, der2 = 0, g2 = 0, div = 0, lap = 0;
   for (int a = 0; a < 3; a++) {
     if (!act[a]) continue;
-    const double fp = (double)f[c + st[a]], fm = (double)f[c - st[a]];
+    const double fp = V(f, c + st[a]), fm = V(f, c - st[a]);
     const double delta = fp - fm;               /* first difference f(p+1) - f(p-1)      */
     const double D = delta / 2.0;               /* central derivative (Alg. 2)  */
     const double lap_a = fp - 2.0 * f0 + fm;    /* second difference f(p+1)-2f(p)+f(p-1)  */
@@ -150,9 +166,9 @@ static void deriv_point(const float* f, const int64_t n3[3], const int act[3], i
   F[CZCO_LAP] = lap;
 }
 
-int czco_deriv(const float* x, const float* y, int ndim, const int64_t* dims, czco_deriv_t* r) {
+static int deriv_impl(fld_t x, fld_t y, int ndim, const int64_t* dims, czco_deriv_t* r) {
   int64_t n3[3];
-  if (!x || !y || !r || !shape3(ndim, dims, n3)) return 1;
+  if (!x.p || !y.p || !r || !shape3(ndim, dims, n3)) return 1;
   memset(r, 0, sizeof(*r));
   int act[3], any = 0;
   int64_t lo[3], hi[3];
@@ -224,6 +240,12 @@ int czco_deriv(const float* x, const float* y, int ndim, const int64_t* dims, cz
   free(pext);
   return 0;
 }
+int czco_deriv(const float* x, const float* y, int ndim, const int64_t* dims, czco_deriv_t* r) {
+  return deriv_impl(fld32(x), fld32(y), ndim, dims, r);
+}
+int czco_deriv_f64(const double* x, const double* y, int ndim, const int64_t* dims, czco_deriv_t* r) {
+  return deriv_impl(fld64(x), fld64(y), ndim, dims, r);
+}
 
 /* ======================================================================================
  * Error autocorrelation, Eq. (2):
@@ -231,10 +253,10 @@ int czco_deriv(const float* x, const float* y, int ndim, const int64_t* dims, cz
  * R_tau = { p : p_a <= n_a - 1 - tau on every active axis },  ne = prod_a (n_a - tau).
  * mu, sigma^2: mean and (population) variance of e over all N elements (R13).  1/3 -> 1/D (R12).
  * ====================================================================================== */
-int czco_autocorr(const float* x, const float* y, int ndim, const int64_t* dims, int max_lag,
-                  double* ac, uint64_t* count) {
+static int autocorr_impl(fld_t x, fld_t y, int ndim, const int64_t* dims, int max_lag,
+                         double* ac, uint64_t* count) {
   int64_t n3[3];
-  if (!x || !y || !ac || !count || max_lag < 0 || !shape3(ndim, dims, n3)) return 1;
+  if (!x.p || !y.p || !ac || !count || max_lag < 0 || !shape3(ndim, dims, n3)) return 1;
   const int64_t N = n3[0] * n3[1] * n3[2];
   const int64_t st[3] = {n3[1] * n3[2], n3[2], 1};
   int act[3], D = 0;
@@ -288,6 +310,14 @@ int czco_autocorr(const float* x, const float* y, int ndim, const int64_t* dims,
   }
   return 0;
 }
+int czco_autocorr(const float* x, const float* y, int ndim, const int64_t* dims, int max_lag,
+                  double* ac, uint64_t* count) {
+  return autocorr_impl(fld32(x), fld32(y), ndim, dims, max_lag, ac, count);
+}
+int czco_autocorr_f64(const double* x, const double* y, int ndim, const int64_t* dims, int max_lag,
+                      double* ac, uint64_t* count) {
+  return autocorr_impl(fld64(x), fld64(y), ndim, dims, max_lag, ac, count);
+}
 
 /* ======================================================================================
  * SSIM, L139-L146: a w^D window slides with a fixed step over both fields; per window the
@@ -296,20 +326,21 @@ int czco_autocorr(const float* x, const float* y, int ndim, const int64_t* dims,
  * only (o_a + w_a <= n_a, R17).  Dynamic range L = max - min of the ORIGINAL window (R15;
  * range_mode 1: the caller's global range), L := 1 when L == 0.
  * ====================================================================================== */
-static double ssim_window3(const float* x, const float* y, const int64_t n3[3], const int64_t o[3],
+static double ssim_window3(fld_t x, fld_t y, const int64_t n3[3], const int64_t o[3],
                            const int64_t w[3], int range_mode, double global_range) {
   const int64_t st[3] = {n3[1] * n3[2], n3[2], 1};
   const ld M = (ld)(w[0] * w[1] * w[2]);
   ld sx = 0, sy = 0;
-  float xmin = x[o[0] * st[0] + o[1] * st[1] + o[2]], xmax = xmin;
+  double xmin = V(x, o[0] * st[0] + o[1] * st[1] + o[2]), xmax = xmin;
   for (int64_t k = 0; k < w[0]; k++)
     for (int64_t j = 0; j < w[1]; j++)
       for (int64_t i = 0; i < w[2]; i++) {
         const int64_t p = (o[0] + k) * st[0] + (o[1] + j) * st[1] + o[2] + i;
-        sx += (ld)x[p];
-        sy += (ld)y[p];
-        if (x[p] < xmin) xmin = x[p];
-        if (x[p] > xmax) xmax = x[p];
+        const double xp = V(x, p);
+        sx += (ld)xp;
+        sy += (ld)V(y, p);
+        if (xp < xmin) xmin = xp;
+        if (xp > xmax) xmax = xp;
       }
   const ld mx = sx / M, my = sy / M;
   ld vx = 0, vy = 0, cxy = 0;
@@ -317,7 +348,7 @@ static double ssim_window3(const float* x, const float* y, const int64_t n3[3], 
     for (int64_t j = 0; j < w[1]; j++)
       for (int64_t i = 0; i < w[2]; i++) {
         const int64_t p = (o[0] + k) * st[0] + (o[1] + j) * st[1] + o[2] + i;
-        const ld dx = (ld)x[p] - mx, dy = (ld)y[p] - my;
+        const ld dx = (ld)V(x, p) - mx, dy = (ld)V(y, p) - my;
         vx += dx * dx;
         vy += dy * dy;
         cxy += dx * dy;
@@ -339,11 +370,11 @@ static int window3(int ndim, const int64_t* v, int64_t out[3], int64_t fill) {
   return 1;
 }
 
-double czco_ssim_window(const float* x, const float* y, int ndim, const int64_t* dims,
-                        const int64_t* origin, const int64_t* window, int range_mode,
-                        double global_range) {
+static double ssim_window_impl(fld_t x, fld_t y, int ndim, const int64_t* dims,
+                               const int64_t* origin, const int64_t* window, int range_mode,
+                               double global_range) {
   int64_t n3[3], o[3], w[3];
-  if (!x || !y || !shape3(ndim, dims, n3)) return NAN;
+  if (!x.p || !y.p || !shape3(ndim, dims, n3)) return NAN;
   window3(ndim, origin, o, 0);
   window3(ndim, window, w, 1);
   for (int a = 0; a < 3; a++) {
@@ -352,19 +383,33 @@ double czco_ssim_window(const float* x, const float* y, int ndim, const int64_t*
   }
   return ssim_window3(x, y, n3, o, w, range_mode, global_range);
 }
+double czco_ssim_window(const float* x, const float* y, int ndim, const int64_t* dims,
+                        const int64_t* origin, const int64_t* window, int range_mode,
+                        double global_range) {
+  return ssim_window_impl(fld32(x), fld32(y), ndim, dims, origin, window, range_mode, global_range);
+}
+double czco_ssim_window_f64(const double* x, const double* y, int ndim, const int64_t* dims,
+                            const int64_t* origin, const int64_t* window, int range_mode,
+                            double global_range) {
+  return ssim_window_impl(fld64(x), fld64(y), ndim, dims, origin, window, range_mode, global_range);
+}
 
-int czco_ssim(const float* x, const float* y, int ndim, const int64_t* dims, const int64_t* window,
-              const int64_t* step, int range_mode, double* ssim, uint64_t* n_windows) {
+static int ssim_impl(fld_t x, fld_t y, int ndim, const int64_t* dims, const int64_t* window,
+                     const int64_t* step, int range_mode, double* ssim, uint64_t* n_windows) {
   int64_t n3[3], w[3], s[3], nw[3];
-  if (!x || !y || !ssim || !n_windows || !shape3(ndim, dims, n3)) return 1;
+  if (!x.p || !y.p || !ssim || !n_windows || !shape3(ndim, dims, n3)) return 1;
   window3(ndim, window, w, 1);
   window3(ndim, step, s, 1);
   double grange = 0;
   if (range_mode) {
     const int64_t N = n3[0] * n3[1] * n3[2];
-    float mn = x[0], mxv = x[0];
-    for (int64_t i = 0; i < N; i++) { if (x[i] < mn) mn = x[i]; if (x[i] > mxv) mxv = x[i]; }
-    grange = (double)mxv - (double)mn;
+    double mn = V(x, 0), mxv = mn;
+    for (int64_t i = 0; i < N; i++) {
+      const double v = V(x, i);
+      if (v < mn) mn = v;
+      if (v > mxv) mxv = v;
+    }
+    grange = mxv - mn;
   }
   for (int a = 0; a < 3; a++) {
     if (n3[a] == 1) { w[a] = 1; s[a] = 1; }
@@ -393,6 +438,14 @@ int czco_ssim(const float* x, const float* y, int ndim, const int64_t* dims, con
   *ssim = (double)(tot / (ld)total);
   return 0;
 }
+int czco_ssim(const float* x, const float* y, int ndim, const int64_t* dims, const int64_t* window,
+              const int64_t* step, int range_mode, double* ssim, uint64_t* n_windows) {
+  return ssim_impl(fld32(x), fld32(y), ndim, dims, window, step, range_mode, ssim, n_windows);
+}
+int czco_ssim_f64(const double* x, const double* y, int ndim, const int64_t* dims, const int64_t* window,
+                  const int64_t* step, int range_mode, double* ssim, uint64_t* n_windows) {
+  return ssim_impl(fld64(x), fld64(y), ndim, dims, window, step, range_mode, ssim, n_windows);
+}
 
 /* ======================================================================================
  * Error PDF / pwr-error PDF (Table I Category I, L107).  The paper names the two metrics but
@@ -408,17 +461,18 @@ static int pdf_bin(double v, double lo, double w, int nbins) {
   return b;
 }
 
-int czco_pdf(const float* x, const float* y, uint64_t n, int nbins, double* err_lo, double* err_w,
-             uint64_t* err_counts, double* pwr_lo, double* pwr_w, uint64_t* pwr_counts, uint64_t* n_pwr) {
-  if (!x || !y || n == 0 || nbins < 1 || !err_counts || !pwr_counts) return 1;
+static int pdf_impl(fld_t x, fld_t y, uint64_t n, int nbins, double* err_lo, double* err_w,
+                    uint64_t* err_counts, double* pwr_lo, double* pwr_w, uint64_t* pwr_counts, uint64_t* n_pwr) {
+  if (!x.p || !y.p || n == 0 || nbins < 1 || !err_counts || !pwr_counts) return 1;
   double emin = INFINITY, emax = -INFINITY, pmin = INFINITY, pmax = -INFINITY;
   uint64_t np = 0;
   for (uint64_t i = 0; i < n; i++) {
     const double e = err_of(x, y, (int64_t)i);
     if (e < emin) emin = e;
     if (e > emax) emax = e;
-    if (x[i] != 0.0f) {
-      const double q = fabs(e) / fabs((double)x[i]);
+    const double xi = V(x, (int64_t)i);
+    if (xi != 0.0) {
+      const double q = fabs(e) / fabs(xi);
       if (q < pmin) pmin = q;
       if (q > pmax) pmax = q;
       np++;
@@ -430,7 +484,8 @@ int czco_pdf(const float* x, const float* y, uint64_t n, int nbins, double* err_
   for (uint64_t i = 0; i < n; i++) {
     const double e = err_of(x, y, (int64_t)i);
     err_counts[pdf_bin(e, emin, ew, nbins)]++;
-    if (x[i] != 0.0f) pwr_counts[pdf_bin(fabs(e) / fabs((double)x[i]), pmin, pw, nbins)]++;
+    const double xi = V(x, (int64_t)i);
+    if (xi != 0.0) pwr_counts[pdf_bin(fabs(e) / fabs(xi), pmin, pw, nbins)]++;
   }
   *err_lo = emin;
   *err_w = ew;
@@ -438,4 +493,12 @@ int czco_pdf(const float* x, const float* y, uint64_t n, int nbins, double* err_
   *pwr_w = pw;
   *n_pwr = np;
   return 0;
+}
+int czco_pdf(const float* x, const float* y, uint64_t n, int nbins, double* err_lo, double* err_w,
+             uint64_t* err_counts, double* pwr_lo, double* pwr_w, uint64_t* pwr_counts, uint64_t* n_pwr) {
+  return pdf_impl(fld32(x), fld32(y), n, nbins, err_lo, err_w, err_counts, pwr_lo, pwr_w, pwr_counts, n_pwr);
+}
+int czco_pdf_f64(const double* x, const double* y, uint64_t n, int nbins, double* err_lo, double* err_w,
+                 uint64_t* err_counts, double* pwr_lo, double* pwr_w, uint64_t* pwr_counts, uint64_t* n_pwr) {
+  return pdf_impl(fld64(x), fld64(y), n, nbins, err_lo, err_w, err_counts, pwr_lo, pwr_w, pwr_counts, n_pwr);
 }

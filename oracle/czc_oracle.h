@@ -70,6 +70,21 @@ int czco_ssim(const float* x, const float* y, int ndim, const int64_t* dims, con
 int czco_pdf(const float* x, const float* y, uint64_t n, int nbins, double* err_lo, double* err_w,
              uint64_t* err_counts, double* pwr_lo, double* pwr_w, uint64_t* pwr_counts, uint64_t* n_pwr);
 
+/* float64 inputs (NEXT row f3; the paper evaluates single precision only, L330): the same
+ * definitions, every sample read as a double.  For float-representable data they return exactly
+ * what the float32 entry points return. */
+int czco_p1_f64(const double* x, const double* y, uint64_t n, czco_p1_t* out);
+int czco_deriv_f64(const double* x, const double* y, int ndim, const int64_t* dims, czco_deriv_t* out);
+int czco_autocorr_f64(const double* x, const double* y, int ndim, const int64_t* dims, int max_lag,
+                      double* ac, uint64_t* count);
+double czco_ssim_window_f64(const double* x, const double* y, int ndim, const int64_t* dims,
+                            const int64_t* origin, const int64_t* window, int range_mode,
+                            double global_range);
+int czco_ssim_f64(const double* x, const double* y, int ndim, const int64_t* dims, const int64_t* window,
+                  const int64_t* step, int range_mode, double* ssim, uint64_t* n_windows);
+int czco_pdf_f64(const double* x, const double* y, uint64_t n, int nbins, double* err_lo, double* err_w,
+                 uint64_t* err_counts, double* pwr_lo, double* pwr_w, uint64_t* pwr_counts, uint64_t* n_pwr);
+
 /* Number of OpenMP threads the oracle uses (bench.py reports it as "cores"). */
 int czco_threads(void);
 

@@ -380,3 +380,70 @@ class TestPdf:
         r = orc.pdf(x, y, 8)
         assert r["n_pwr"] == 0 and math.isnan(r["pwr_pdf_lo"]) and r["pwr_pdf"].sum() == 0
         assert int(r["err_pdf"].sum()) == 100
+
+
+# ------------------------------------------------------------------- float64 inputs (NEXT f3)
+class TestFloat64:
+    """The float64 entry points (NEXT row f3, L92 / L330): pinned by (1) the invariant that
+    float-representable data gives bit-identical results through both element types (every
+    sample is read as a double either way), (2) closed forms whose inputs float32 cannot hold,
+    (3) numpy on data with full 53-bit mantissas."""
+
+    def test_float_data_identical_through_f64(self, orc):
+        x, y = synth.make_pair(synth.config("C1", dims=(12, 14, 16)))
+        xn, yn = x.numpy(), y.numpy()
+        xd, yd = xn.astype(np.float64), yn.astype(np.float64)
+        assert orc.p1(xn, yn) == orc.p1(xd, yd)
+        assert orc.deriv(xn, yn) == orc.deriv(xd, yd)
+        a32, c32 = orc.autocorr(xn, yn, 5)
+        a64, c64 = orc.autocorr(xd, yd, 5)
+        assert np.array_equal(a32, a64) and np.array_equal(c32, c64)
+        assert orc.ssim(xn, yn, [5, 5, 5], [2, 3, 1]) == orc.ssim(xd, yd, [5, 5, 5], [2, 3, 1])
+        p32, p64 = orc.pdf(xn, yn, 17), orc.pdf(xd, yd, 17)
+        for k in p32:
+            assert np.array_equal(p32[k], p64[k]), k
+
+    def test_sub_float_offset_closed_form(self, orc):
+        """x on a 2^-40 grid (|x| < 2^-12, not float32-representable), e == c = 2^-45 exactly:
+        MSE = c^2, PSNR = 20 log10(R / c), every window's SSIM has the closed form of a constant
+        offset, Der/Div/Lap errors are 0 (a constant offset has no derivative), AC undefined."""
+        x = rng.integers(-(2 ** 28), 2 ** 28, size=(9, 10, 11)).astype(np.float64) * 2.0 ** -40
+        assert np.any(x.astype(np.float32).astype(np.float64) != x)
+        c = 2.0 ** -45
+        y = x + c
+        assert np.all(y - x == c)
+        r = orc.p1(x, y)
+        R = float(x.max() - x.min())
+        assert r["mse"] == c * c and r["err_min"] == c == r["err_max"] and r["err_var"] == 0.0
+        assert abs(r["psnr"] - 20 * math.log10(R / c)) < 1e-12
+        d = orc.deriv(x, y)
+        for f in ("der1", "der2", "div", "lap"):
+            assert d[f + "_maxabs"] == 0.0, f
+        ac, _ = orc.autocorr(x, y, 3)
+        assert all(math.isnan(v) for v in ac[1:])
+        # SSIM of one window with y = x + c: (2 mx (mx + c) + C1) (2 vx + C2) /
+        # ((mx^2 + (mx + c)^2 + C1) (2 vx + C2)) = (2 mx (mx + c) + C1) / (mx^2 + (mx + c)^2 + C1)
+        o, w = (1, 2, 3), (4, 4, 4)
+        win = x[1:5, 2:6, 3:7]
+        mx, L = win.mean(), float(win.max() - win.min())
+        C1 = (0.01 * L) ** 2
+        want = (2 * mx * (mx + c) + C1) / (mx * mx + (mx + c) ** 2 + C1)
+        assert abs(orc.ssim_window(x, y, o, w) - want) < 1e-12
+
+    def test_numpy_brute_force_full_mantissa(self, orc):
+        x = rng.standard_normal((6, 7, 9)) * 1e3 + 1e4
+        y = x + rng.standard_normal(x.shape) * 1e-7
+        e = y - x
+        r = orc.p1(x, y)
+        assert r["err_min"] == e.min() and r["err_max"] == e.max() and r["x_min"] == x.min()
+        q = np.abs(e) / np.abs(x)
+        assert r["pwr_max"] == q.max() and r["pwr_min"] == q.min()
+        assert abs(r["mse"] / np.mean(e * e) - 1) < 1e-12
+        assert abs(r["pearson"] - np.corrcoef(x.ravel(), y.ravel())[0, 1]) < 1e-12
+        d = orc.deriv(x, y)
+        gx = [np.gradient(x, axis=a)[1:-1, 1:-1, 1:-1] for a in range(3)]
+        gy = [np.gradient(y, axis=a)[1:-1, 1:-1, 1:-1] for a in range(3)]
+        grad = np.sqrt(sum(g * g for g in gy)) - np.sqrt(sum(g * g for g in gx))
+        assert abs(d["grad_mae"] - np.mean(np.abs(grad))) < 1e-9 * np.mean(np.abs(grad)) + 1e-15
+        s, nw = orc.ssim(x, y, [3, 3, 3])
+        assert nw == 4 * 5 * 7 and 0.0 < s <= 1.0
