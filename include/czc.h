@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define CZC_ABI_VERSION 2
+#define CZC_ABI_VERSION 3
 #define CZC_MAX_LAG 16           /* largest supported autocorrelation lag (paper uses <= 10, L345) */
 #define CZC_PDF_MAX_BINS 256     /* largest number of error-PDF bins                              */
 
@@ -45,14 +45,18 @@ typedef enum czc_status {
   CZC_OK = 0,
   CZC_ERR_INVALID = 1,           /* NULL pointer, bad config value                              */
   CZC_ERR_SHAPE = 2,             /* ndim/dims invalid, SSIM window larger than the field, ...  */
-  CZC_ERR_DTYPE = 3,             /* dtype not supported (hot path: float32 only)                */
+  CZC_ERR_DTYPE = 3,             /* dtype not one of czc_dtype                                  */
   CZC_ERR_CUDA = 4,              /* a CUDA runtime call or kernel launch failed                 */
   CZC_ERR_NOMEM = 5,             /* device or host allocation failed                            */
   CZC_ERR_COMM = 6,              /* NCCL failure (multi-GPU slab mode)                          */
   CZC_ERR_UNSUPPORTED = 7        /* feature not built / requested combination not supported     */
 } czc_status;
 
-typedef enum czc_dtype { CZC_F32 = 0, CZC_F64 = 1 /* not in the hot path: CZC_ERR_DTYPE */ } czc_dtype;
+/* Element type of BOTH fields.  CZC_F32 is the paper's precision (L330: "all the data are
+ * single-precision"); CZC_F64 is NEXT row f3 ("easily extended", L92): the same kernels with a
+ * double element type (every accumulator is FP64 either way; e = y - x is rounded to double, as
+ * in the oracle, reading R1), 16 bytes per element pair instead of 8. */
+typedef enum czc_dtype { CZC_F32 = 0, CZC_F64 = 1 } czc_dtype;
 
 /* metric_mask bits — one per pattern group (Table I categories, L107). */
 enum {
@@ -71,7 +75,9 @@ enum { CZC_DER1 = 0, CZC_DER2 = 1, CZC_GRAD = 2, CZC_DIV = 3, CZC_LAP = 4, CZC_N
 
 typedef struct czc_config {
   int device;                    /* CUDA device ordinal the context binds to; -1 = current       */
-  void* stream;                  /* cudaStream_t to run on; NULL = a stream owned by the context */
+  void* stream;                  /* cudaStream_t to run on; NULL = a BLOCKING stream owned by the */
+                                 /* context (ordered after the caller's legacy-default-stream    */
+                                 /* work, e.g. PyTorch's default stream, handle 0)               */
   int ssim_window[3];            /* window extent per input axis (index i <-> dims[i]); 0 -> 8   */
   int ssim_step[3];              /* window step per input axis; 0 -> 1 (L352: w = 8, step 1)     */
   int ssim_range_mode;           /* 0: L = max - min of the original window (reading R15)        */
@@ -154,7 +160,8 @@ czc_status czc_init(czc_ctx** ctx, const czc_config* cfg);
 
 /* Assess a field pair resident in DEVICE memory.
  *   orig, recon : caller-owned device pointers to shape->nz_local * dims[1] * dims[2] elements of
- *                 `dtype` (read-only; any alignment, 16-byte alignment takes the vector path).
+ *                 `dtype` (read-only; element-aligned; 16-byte alignment takes the vector path).
+ *   dtype       : CZC_F32 or CZC_F64 (both fields), else CZC_ERR_DTYPE.
  *   metric_mask : OR of CZC_M_* bits; groups run in the order P1 -> P2 -> P3 (AC needs P1's
  *                 mean and variance of the error, Alg. 2).
  *   out         : caller-owned host struct, filled before return.

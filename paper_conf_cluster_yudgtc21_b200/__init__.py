@@ -7,7 +7,7 @@ There is NO CPU fallback: if libczc.so is missing or cannot be loaded, the first
 or attribute `lib`) raises ImportError.
 
     import paper_conf_cluster_yudgtc21_b200 as czc
-    r = czc.assess(orig, recon)                # orig/recon: CUDA float32 tensors, same shape
+    r = czc.assess(orig, recon)                # orig/recon: CUDA float32 (or float64) tensors
     r["psnr"], r["ssim"], r["ac"], r["der1_mae"] ...
 """
 from __future__ import annotations
@@ -23,6 +23,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("CZC_LIB") or os.path.join(_HERE, "libczc.so")
 
 M_P1, M_DERIV, M_AUTOCORR, M_SSIM, M_PDF = 1, 2, 4, 8, 16
+F32, F64 = 0, 1      # czc_dtype
 M_ALL = 0xF          # the four pattern groups (bench.py's step)
 M_FULL = 0x1F        # + the error / pwr-error PDFs (Table I Category I)
 MAX_LAG = 16
@@ -212,12 +213,13 @@ def result_dict(r: Result) -> Dict:
     return out
 
 
-def czc_assess(ctx: int, orig_ptr: int, recon_ptr: int, shape: Shape, mask: int = M_ALL, host: bool = False) -> Dict:
+def czc_assess(ctx: int, orig_ptr: int, recon_ptr: int, shape: Shape, mask: int = M_ALL, host: bool = False,
+               dtype: int = F32) -> Dict:
     """czc_assess / czc_assess_host with raw pointers; returns the result as a dict."""
     r = Result()
     lib = get_lib()
     fn = lib.czc_assess_host if host else lib.czc_assess
-    rc = fn(ctx, orig_ptr, recon_ptr, ctypes.byref(shape), 0, mask, ctypes.byref(r))
+    rc = fn(ctx, orig_ptr, recon_ptr, ctypes.byref(shape), dtype, mask, ctypes.byref(r))
     if rc:
         raise CzcError(rc, lib.czc_last_error(ctx).decode(errors="replace"))
     return result_dict(r)
@@ -249,28 +251,32 @@ class Assessor:
         self.ctx = czc_init(self.cfg)
 
     def assess(self, orig, recon, mask: int = M_ALL, dims=None, z0: int = 0) -> Dict:
-        """orig/recon: CUDA float32 C-contiguous tensors (slab mode: this rank's planes, with the
-        GLOBAL dims passed in `dims` and the first plane index in `z0`)."""
+        """orig/recon: CUDA C-contiguous tensors, both float32 or both float64 (slab mode: this
+        rank's planes, with the GLOBAL dims passed in `dims` and the first plane index in `z0`)."""
         import torch
+        dts = {torch.float32: F32, torch.float64: F64}
         for t in (orig, recon):
-            if not (t.is_cuda and t.dtype == torch.float32 and t.is_contiguous()):
-                raise TypeError("orig/recon must be contiguous float32 CUDA tensors")
+            if not (t.is_cuda and t.dtype in dts and t.is_contiguous()):
+                raise TypeError("orig/recon must be contiguous float32 or float64 CUDA tensors")
+        if orig.dtype != recon.dtype:
+            raise TypeError("orig and recon must have the same dtype")
         if orig.shape != recon.shape:
             raise ValueError("orig and recon must have the same shape")
         gdims = list(orig.shape) if dims is None else list(dims)
         shape = make_shape(gdims, z0, orig.shape[0] if dims is not None else 0)
-        return czc_assess(self.ctx, orig.data_ptr(), recon.data_ptr(), shape, mask)
+        return czc_assess(self.ctx, orig.data_ptr(), recon.data_ptr(), shape, mask, dtype=dts[orig.dtype])
 
     def assess_host(self, orig, recon, mask: int = M_ALL, dims=None, z0: int = 0) -> Dict:
         """Same, from HOST buffers (numpy arrays or CPU tensors, ideally pinned): the library copies
         them to the device on its stream inside the call."""
         o = orig if isinstance(orig, np.ndarray) else orig.numpy()
         r_ = recon if isinstance(recon, np.ndarray) else recon.numpy()
-        if o.dtype != np.float32 or r_.dtype != np.float32 or not o.flags.c_contiguous or not r_.flags.c_contiguous:
-            raise TypeError("orig/recon must be C-contiguous float32")
+        dts = {np.dtype(np.float32): F32, np.dtype(np.float64): F64}
+        if o.dtype not in dts or r_.dtype != o.dtype or not o.flags.c_contiguous or not r_.flags.c_contiguous:
+            raise TypeError("orig/recon must be C-contiguous, both float32 or both float64")
         gdims = list(o.shape) if dims is None else list(dims)
         shape = make_shape(gdims, z0, o.shape[0] if dims is not None else 0)
-        return czc_assess(self.ctx, o.ctypes.data, r_.ctypes.data, shape, mask, host=True)
+        return czc_assess(self.ctx, o.ctypes.data, r_.ctypes.data, shape, mask, host=True, dtype=dts[o.dtype])
 
     def close(self):
         if getattr(self, "ctx", None):
@@ -291,6 +297,6 @@ class Assessor:
 
 
 def assess(orig, recon, mask: int = M_ALL, **cfg) -> Dict:
-    """One-shot assessment of two CUDA float32 tensors (creates and frees a context)."""
+    """One-shot assessment of two CUDA float32 / float64 tensors (creates and frees a context)."""
     with Assessor(ndim=orig.dim(), **cfg) as a:
         return a.assess(orig, recon, mask)

@@ -19,19 +19,27 @@
 #include "czc_internal.cuh"
 
 namespace czc {
-cudaError_t launch_p1(const float* x, const float* y, int64_t n, int grid_cap, P1State* parts,
+// Launchers, instantiated for E = float and E = double in their .cu files.
+template <typename E>
+cudaError_t launch_p1(const E* x, const E* y, int64_t n, int grid_cap, P1State* parts,
                       DevResults* res, unsigned int* ticket, cudaStream_t st);
 cudaError_t launch_p1_combine(const P1State* states, int count, DevResults* res, cudaStream_t st);
-cudaError_t launch_pdf(const float* x, const float* y, int64_t n, int nb, int grid_cap, DevResults* res,
+template <typename E>
+cudaError_t launch_pdf(const E* x, const E* y, int64_t n, int nb, int grid_cap, DevResults* res,
                        cudaStream_t st);
 int p1_max_blocks_per_sm();
-int64_t deriv_blocks(const Field3& s, int zchunk);
-int64_t ac_blocks(const Field3& s, int T);
-cudaError_t launch_deriv(const Field3& s, int zchunk, double* parts, DevResults* res,
+template <typename E>
+int64_t deriv_blocks(const Field3<E>& s, int zchunk);
+template <typename E>
+int64_t ac_blocks(const Field3<E>& s, int T);
+template <typename E>
+cudaError_t launch_deriv(const Field3<E>& s, int zchunk, double* parts, DevResults* res,
                          unsigned int* ticket, cudaStream_t st);
-cudaError_t launch_ac(const Field3& s, int T, int zchunk, double* parts, DevResults* res,
+template <typename E>
+cudaError_t launch_ac(const Field3<E>& s, int T, int zchunk, double* parts, DevResults* res,
                       unsigned int* ticket, cudaStream_t st);
-cudaError_t launch_ssim(int kind, int W, const Field3& f, const SsimParams& p,
+template <typename E>
+cudaError_t launch_ssim(int kind, int W, const Field3<E>& f, const SsimParams& p,
                         double* parts, DevResults* res, unsigned int* ticket, double* dbg,
                         cudaStream_t st, int64_t* nblocks_out);
 }  // namespace czc
@@ -52,7 +60,7 @@ struct czc_ctx {
   unsigned int* tickets = nullptr; // device
   void* parts = nullptr;           // per-block partial records
   size_t parts_cap = 0;
-  float* din[2] = {nullptr, nullptr};   // staging for czc_assess_host
+  void* din[2] = {nullptr, nullptr};    // staging for czc_assess_host
   size_t din_cap = 0;
   cudaEvent_t ev[6] = {};   // P1 start, P1 end, deriv end, AC end, SSIM end, call end
   std::string last_error;
@@ -61,7 +69,7 @@ struct czc_ctx {
   void* dgather_in = nullptr;      // device, 64 B
   void* dgather = nullptr;         // device, max_records * sizeof(Record)
   void* dstates = nullptr;         // device, max_records * sizeof(P1State)
-  float* halo = nullptr;           // device halo planes (x lo, y lo, x hi, y hi)
+  void* halo = nullptr;            // device halo planes (x lo, y lo, x hi, y hi)
   size_t halo_cap = 0;
   int max_records = 1;
   // pipelined host path
@@ -137,7 +145,9 @@ extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
     if (c.stream) {
       ctx->stream = (cudaStream_t)c.stream;
     } else {
-      e = cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking);
+      // a BLOCKING stream: it is ordered after work the caller queued on the legacy default
+      // stream (e.g. the kernels that produced the fields), as a NULL stream argument implies
+      e = cudaStreamCreateWithFlags(&ctx->stream, cudaStreamDefault);
       if (e != cudaSuccess) { st = cuda_fail(ctx, e, "cudaStreamCreate"); break; }
       ctx->own_stream = true;
     }
@@ -145,7 +155,8 @@ extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
     if ((e = cudaMalloc(&ctx->dres, sizeof(DevResults))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(res)"); break; }
     if ((e = cudaMallocHost(&ctx->hrec, rb)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMallocHost"); break; }
     if ((e = cudaMalloc(&ctx->tickets, TICKET_N * sizeof(unsigned int))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(tickets)"); break; }
-    if ((e = cudaMemset(ctx->tickets, 0, TICKET_N * sizeof(unsigned int))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMemset"); break; }
+    if ((e = cudaMemsetAsync(ctx->tickets, 0, TICKET_N * sizeof(unsigned int), ctx->stream)) != cudaSuccess ||
+        (e = cudaStreamSynchronize(ctx->stream)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMemset"); break; }
     for (int i = 0; i < 6 && st == CZC_OK; i++)
       if ((e = cudaEventCreate(&ctx->ev[i])) != cudaSuccess) st = cuda_fail(ctx, e, "cudaEventCreate");
     if (st != CZC_OK) break;
@@ -391,8 +402,12 @@ extern "C" czc_status czc_combine(const void* records, int nrecords, const czc_s
 // ------------------------------------------------------------------------------------------------
 // Device execution
 // ------------------------------------------------------------------------------------------------
+// Grow a context buffer.  Work already queued on the context stream may still use the old
+// buffer (e.g. P1's partials when the P2/P3 scratch grows), so the stream is drained before the
+// free: cudaFree does not order itself after work on a non-blocking stream.
 static czc_status ensure_buf(czc_ctx* ctx, void** p, size_t* cap, size_t bytes) {
   if (bytes <= *cap) return CZC_OK;
+  if (*p) CZC_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
   cudaFree(*p);
   *p = nullptr;
   *cap = 0;
@@ -426,7 +441,8 @@ int64_t halo_depth(const Plan& P) {
 }  // namespace
 
 // Scratch for the largest launch over the given field view.
-static czc_status ensure_scratch(czc_ctx* ctx, const Plan& P, const Field3& F, const SsimParams& sp) {
+template <typename E>
+static czc_status ensure_scratch(czc_ctx* ctx, const Plan& P, const Field3<E>& F, const SsimParams& sp) {
   size_t need = (size_t)ctx->p1_grid_cap * sizeof(P1State);
   if (P.run_deriv) need = std::max(need, (size_t)deriv_blocks(F, kZchunkDeriv) * kDerivSlots * sizeof(double));
   if (P.run_ac) need = std::max(need, (size_t)ac_blocks(F, P.T) * kAcSlots * sizeof(double));
@@ -442,7 +458,8 @@ static czc_status ensure_scratch(czc_ctx* ctx, const Plan& P, const Field3& F, c
 }
 
 // P2 + P3 over one field view (the owned planes of F); results land in dres->rec.
-static czc_status run_p23(czc_ctx* ctx, const Plan& P, const Field3& F, const SsimParams& sp) {
+template <typename E>
+static czc_status run_p23(czc_ctx* ctx, const Plan& P, const Field3<E>& F, const SsimParams& sp) {
   const cudaStream_t s = ctx->stream;
   czc_status st = ensure_scratch(ctx, P, F, sp);
   if (st != CZC_OK) return st;
@@ -466,7 +483,8 @@ static cudaError_t copy_records(Record* h, const Record* d, int n, bool pdf, cud
                            cudaMemcpyDeviceToHost, s);
 }
 
-static czc_status p1_local(czc_ctx* ctx, const Plan& P, const float* x, const float* y, int64_t n) {
+template <typename E>
+static czc_status p1_local(czc_ctx* ctx, const Plan& P, const E* x, const E* y, int64_t n) {
   if (!P.run_p1) return CZC_OK;
   czc_status st = ensure_buf(ctx, &ctx->parts, &ctx->parts_cap, (size_t)ctx->p1_grid_cap * sizeof(P1State));
   if (st != CZC_OK) return st;
@@ -482,11 +500,12 @@ static void finish_timing(czc_ctx* ctx, czc_result* out) {
 }
 
 // Single GPU, whole field resident.
-static czc_status assess_single(czc_ctx* ctx, const Plan& P, const float* x, const float* y, czc_result* out,
+template <typename E>
+static czc_status assess_single(czc_ctx* ctx, const Plan& P, const E* x, const E* y, czc_result* out,
                                 uint64_t mask) {
   const cudaStream_t s = ctx->stream;
   const bool timing = ctx->cfg.timing != 0;
-  Field3 F{};
+  Field3<E> F{};
   F.nz = P.g3[0]; F.ny = P.g3[1]; F.nx = P.g3[2];
   F.zown0 = 0; F.zown1 = F.nz;
   F.nseg = 1; F.xs[0] = x; F.ys[0] = y; F.zs[0] = 0; F.zs[1] = F.nz;
@@ -508,14 +527,15 @@ static czc_status assess_single(czc_ctx* ctx, const Plan& P, const float* x, con
 
 // Field view of one slab [z0, z0 + nzl) whose halo planes live in ctx->halo (lo: hlo planes,
 // hi: hhi planes; filled by NCCL receives or, in loopback mode, device copies).
-static Field3 slab_field(czc_ctx* ctx, const Plan& P, const float* x, const float* y, int64_t z0, int64_t nzl,
-                         int64_t hlo, int64_t hhi, float** xlo, float** ylo, float** xhi, float** yhi) {
+template <typename E>
+static Field3<E> slab_field(czc_ctx* ctx, const Plan& P, const E* x, const E* y, int64_t z0, int64_t nzl,
+                            int64_t hlo, int64_t hhi, E** xlo, E** ylo, E** xhi, E** yhi) {
   const int64_t plane = P.g3[1] * P.g3[2];
-  *xlo = ctx->halo;
+  *xlo = static_cast<E*>(ctx->halo);
   *ylo = *xlo + hlo * plane;
   *xhi = *ylo + hlo * plane;
   *yhi = *xhi + hhi * plane;
-  Field3 F{};
+  Field3<E> F{};
   F.nz = P.g3[0]; F.ny = P.g3[1]; F.nx = P.g3[2];
   F.zown0 = z0; F.zown1 = z0 + nzl;
   int k = 0;
@@ -541,7 +561,8 @@ static bool slabs_ok(const std::vector<std::pair<int64_t, int64_t>>& tab, int64_
 // Loopback: the multi-GPU algorithm on one GPU.  Slab k owns planes [z0_k, z0_k + n_k); its
 // halos are device-copied into ctx->halo (the buffers NCCL receives into); P1 states are merged
 // in slab order on the device before P2; per-slab records are combined in slab order on the host.
-static czc_status assess_loopback(czc_ctx* ctx, const Plan& P, const float* x, const float* y, czc_result* out,
+template <typename E>
+static czc_status assess_loopback(czc_ctx* ctx, const Plan& P, const E* x, const E* y, czc_result* out,
                                   uint64_t mask) {
   const cudaStream_t s = ctx->stream;
   const bool timing = ctx->cfg.timing != 0;
@@ -559,7 +580,7 @@ static czc_status assess_loopback(czc_ctx* ctx, const Plan& P, const float* x, c
   Record* drec = (Record*)ctx->dgather;
   P1State* dst = (P1State*)ctx->dstates;
   // one halo allocation for all slabs (a reallocation between slabs would synchronise the device)
-  czc_status st0 = ensure_buf(ctx, (void**)&ctx->halo, &ctx->halo_cap, 2 * (size_t)(1 + H) * plane * sizeof(float) + 16);
+  czc_status st0 = ensure_buf(ctx, &ctx->halo, &ctx->halo_cap, 2 * (size_t)(1 + H) * plane * sizeof(E) + 16);
   if (st0 != CZC_OK) return st0;
   CZC_CUDA(ctx, cudaMemsetAsync(drec, 0, (size_t)K * sizeof(Record), s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
@@ -578,9 +599,9 @@ static czc_status assess_loopback(czc_ctx* ctx, const Plan& P, const float* x, c
     const int64_t hlo = (P.run_deriv && z0 > 0) ? 1 : 0;
     const int64_t hhi = std::min(H, nz - (z0 + nzl));
     czc_status st;
-    float *xlo, *ylo, *xhi, *yhi;
-    const Field3 F = slab_field(ctx, P, x + z0 * plane, y + z0 * plane, z0, nzl, hlo, hhi, &xlo, &ylo, &xhi, &yhi);
-    const size_t pb = (size_t)plane * sizeof(float);
+    E *xlo, *ylo, *xhi, *yhi;
+    const Field3<E> F = slab_field(ctx, P, x + z0 * plane, y + z0 * plane, z0, nzl, hlo, hhi, &xlo, &ylo, &xhi, &yhi);
+    const size_t pb = (size_t)plane * sizeof(E);
     if (hlo) {
       CZC_CUDA(ctx, cudaMemcpyAsync(xlo, x + (z0 - 1) * plane, pb, cudaMemcpyDeviceToDevice, s));
       CZC_CUDA(ctx, cudaMemcpyAsync(ylo, y + (z0 - 1) * plane, pb, cudaMemcpyDeviceToDevice, s));
@@ -605,7 +626,8 @@ static czc_status assess_loopback(czc_ctx* ctx, const Plan& P, const float* x, c
 }
 
 // NCCL slab mode: this rank holds planes [z0, z0 + nzl) of the global field.
-static czc_status assess_ranks(czc_ctx* ctx, const Plan& P, const float* x, const float* y, const czc_shape* shape,
+template <typename E>
+static czc_status assess_ranks(czc_ctx* ctx, const Plan& P, const E* x, const E* y, const czc_shape* shape,
                                czc_result* out, uint64_t mask) {
   const cudaStream_t s = ctx->stream;
   const bool timing = ctx->cfg.timing != 0;
@@ -631,11 +653,11 @@ static czc_status assess_ranks(czc_ctx* ctx, const Plan& P, const float* x, cons
   const int64_t hhi = std::min(H, nz - (z0 + nzl));
   const int64_t prev_hhi = rank > 0 ? std::min(H, nz - z0) : 0;
   const bool next_lo = P.run_deriv && rank + 1 < nranks;
-  const size_t pb = (size_t)plane * sizeof(float);
-  czc_status st = ensure_buf(ctx, (void**)&ctx->halo, &ctx->halo_cap, 2 * (size_t)(hlo + hhi) * pb + 16);
+  const size_t pb = (size_t)plane * sizeof(E);
+  czc_status st = ensure_buf(ctx, &ctx->halo, &ctx->halo_cap, 2 * (size_t)(hlo + hhi) * pb + 16);
   if (st != CZC_OK) return st;
-  float *xlo, *ylo, *xhi, *yhi;
-  const Field3 F = slab_field(ctx, P, x, y, z0, nzl, hlo, hhi, &xlo, &ylo, &xhi, &yhi);
+  E *xlo, *ylo, *xhi, *yhi;
+  const Field3<E> F = slab_field(ctx, P, x, y, z0, nzl, hlo, hhi, &xlo, &ylo, &xhi, &yhi);
   if (!comm_group_begin(&ctx->last_error)) return CZC_ERR_COMM;
   bool ok = true;
   if (rank > 0 && prev_hhi > 0) {
@@ -680,11 +702,19 @@ static czc_status check_common(czc_ctx* ctx, const void* orig, const void* recon
   if (!out) return CZC_ERR_INVALID;
   memset(out, 0, sizeof(*out));
   if (!ctx || !orig || !recon || !shape) return CZC_ERR_INVALID;
-  if (dtype != CZC_F32) {
-    ctx->last_error = "only float32 fields are supported on the hot path";
+  if (dtype != CZC_F32 && dtype != CZC_F64) {
+    ctx->last_error = "dtype must be CZC_F32 or CZC_F64";
     return CZC_ERR_DTYPE;
   }
   return CZC_OK;
+}
+
+template <typename E>
+static czc_status assess_dispatch(czc_ctx* ctx, const Plan& P, const E* x, const E* y, const czc_shape* shape,
+                                  czc_result* out, uint64_t mask) {
+  if (ctx->comm) return assess_ranks(ctx, P, x, y, shape, out, mask);
+  if (ctx->cfg.loopback_slabs > 1) return assess_loopback(ctx, P, x, y, out, mask);
+  return assess_single(ctx, P, x, y, out, mask);
 }
 
 extern "C" czc_status czc_assess(czc_ctx* ctx, const void* orig, const void* recon, const czc_shape* shape,
@@ -702,12 +732,10 @@ extern "C" czc_status czc_assess(czc_ctx* ctx, const void* orig, const void* rec
     } else if (!ctx->comm && (shape->z0 != 0 || nzl != shape->dims[0])) {
       ctx->last_error = "a slab shape needs nranks > 1";
       st = CZC_ERR_SHAPE;
-    } else if (ctx->comm) {
-      st = assess_ranks(ctx, P, (const float*)orig, (const float*)recon, shape, out, metric_mask);
-    } else if (ctx->cfg.loopback_slabs > 1) {
-      st = assess_loopback(ctx, P, (const float*)orig, (const float*)recon, out, metric_mask);
+    } else if (dtype == CZC_F64) {
+      st = assess_dispatch(ctx, P, (const double*)orig, (const double*)recon, shape, out, metric_mask);
     } else {
-      st = assess_single(ctx, P, (const float*)orig, (const float*)recon, out, metric_mask);
+      st = assess_dispatch(ctx, P, (const float*)orig, (const float*)recon, shape, out, metric_mask);
     }
   }
   if (st != CZC_OK) out->computed_mask = 0;
@@ -719,14 +747,15 @@ extern "C" czc_status czc_assess(czc_ctx* ctx, const void* orig, const void* rec
 // chunk k and the halo planes above it have arrived (records per chunk, owned ranges as in slab
 // mode); the autocorrelation, which needs the global mean / variance of the error, runs once the
 // whole field is resident.  Same combine as slab mode.
-static czc_status assess_host_pipelined(czc_ctx* ctx, const Plan& P, const float* hx, const float* hy,
+template <typename E>
+static czc_status assess_host_pipelined(czc_ctx* ctx, const Plan& P, const E* hx, const E* hy,
                                         czc_result* out, uint64_t mask, int K) {
   const cudaStream_t s = ctx->stream;
   const bool timing = ctx->cfg.timing != 0;
   const int64_t nz = P.g3[0], plane = P.g3[1] * P.g3[2];
-  const size_t pb = (size_t)plane * sizeof(float);
-  float* x = ctx->din[0];
-  float* y = ctx->din[1];
+  const size_t pb = (size_t)plane * sizeof(E);
+  E* x = static_cast<E*>(ctx->din[0]);
+  E* y = static_cast<E*>(ctx->din[1]);
   if (!ctx->copy_stream[0]) {
     for (int c = 0; c < 2; c++) {
       CZC_CUDA(ctx, cudaStreamCreateWithFlags(&ctx->copy_stream[c], cudaStreamNonBlocking));
@@ -753,7 +782,7 @@ static czc_status assess_host_pipelined(czc_ctx* ctx, const Plan& P, const float
     while (j + 1 < K && b[j + 1] < std::min(nz, b[k + 1] + H)) j++;
     return j;
   };
-  Field3 F{};
+  Field3<E> F{};
   F.nz = nz; F.ny = P.g3[1]; F.nx = P.g3[2];
   F.nseg = 1; F.xs[0] = x; F.ys[0] = y; F.zs[0] = 0; F.zs[1] = nz;
   const SsimParams sp = ssim_params(P, ctx->cfg);
@@ -820,7 +849,7 @@ extern "C" czc_status czc_assess_host(czc_ctx* ctx, const void* orig, const void
     n *= (i == 0 && shape->nz_local > 0) ? shape->nz_local : shape->dims[i];
   }
   if (cudaSetDevice(ctx->device) != cudaSuccess) return cuda_fail(ctx, cudaGetLastError(), "cudaSetDevice");
-  const size_t bytes = (size_t)n * sizeof(float);
+  const size_t bytes = (size_t)n * (dtype == CZC_F64 ? sizeof(double) : sizeof(float));
   if (bytes > ctx->din_cap) {
     cudaFree(ctx->din[0]);
     cudaFree(ctx->din[1]);
@@ -840,7 +869,9 @@ extern "C" czc_status czc_assess_host(czc_ctx* ctx, const void* orig, const void
     const int64_t H = std::max<int64_t>(halo_depth(P), 1);
     const int K = (int)std::min<int64_t>(std::min<int64_t>(8, kMaxHostChunks), P.g3[0] / H);
     if (K >= 2) {
-      st = assess_host_pipelined(ctx, P, (const float*)orig, (const float*)recon, out, metric_mask, K);
+      st = dtype == CZC_F64
+               ? assess_host_pipelined(ctx, P, (const double*)orig, (const double*)recon, out, metric_mask, K)
+               : assess_host_pipelined(ctx, P, (const float*)orig, (const float*)recon, out, metric_mask, K);
       if (st != CZC_OK) out->computed_mask = 0;
       return st;
     }

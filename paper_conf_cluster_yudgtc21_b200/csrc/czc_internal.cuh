@@ -56,7 +56,7 @@ struct P1State {
   double emin, emax;          // extrema of e (exact doubles)
   double pmin, pmax, spwr;    // point-wise relative error |e|/|x| over x != 0
   double npwr;                // count of x != 0
-  float xmin, xmax;           // extrema of x (exact)
+  double xmin, xmax;          // extrema of x (exact: float32 and float64 samples are doubles)
 };
 constexpr int kP1Words = sizeof(P1State) / 4;
 static_assert(sizeof(P1State) % 8 == 0, "P1State must be a whole number of doubles");
@@ -65,7 +65,7 @@ __host__ __device__ inline void p1_empty(P1State& s) {
   s.n = 0; s.mx = s.my = s.me = 0; s.m2x = s.m2y = s.cxy = s.m2e = 0; s.sae = 0;
   s.emin = dinf(); s.emax = -dinf();
   s.pmin = dinf(); s.pmax = -dinf(); s.spwr = 0; s.npwr = 0;
-  s.xmin = finf(); s.xmax = -finf();
+  s.xmin = dinf(); s.xmax = -dinf();
 }
 
 __host__ __device__ inline void p1_merge(P1State& a, const P1State& b) {
@@ -151,25 +151,27 @@ struct DevResults {
 // A 3-D field view for the stencil / window kernels: global extents, the planes this launch
 // owns (stencil points / window origins), and up to three z-segments of plane storage (in slab
 // mode: the lower halo, the local slab and the upper halo received from the neighbour ranks).
+// T is the element type of the pair: float (the paper's precision, L330) or double (NEXT f3).
+template <typename T>
 struct Field3 {
   int64_t nz, ny, nx;        // GLOBAL extents (3-D view, inactive axes squeezed)
   int64_t zown0, zown1;      // owned planes [zown0, zown1)
   int nseg;                  // 1..3
-  const float* xs[3];
-  const float* ys[3];
+  const T* xs[3];
+  const T* ys[3];
   int64_t zs[4];             // segment i holds global planes [zs[i], zs[i+1])
 #if defined(__CUDACC__)
   // Plane pointers.  Segment selection uses static indices only (a dynamic index into the
   // by-value kernel parameter would force a local-memory copy of the struct).
-  __device__ __forceinline__ const float* xp(int64_t z) const {
+  __device__ __forceinline__ const T* xp(int64_t z) const {
     const bool s1 = nseg > 1 && z >= zs[1], s2 = nseg > 2 && z >= zs[2];
-    const float* b = s2 ? xs[2] : (s1 ? xs[1] : xs[0]);
+    const T* b = s2 ? xs[2] : (s1 ? xs[1] : xs[0]);
     const int64_t z0 = s2 ? zs[2] : (s1 ? zs[1] : zs[0]);
     return b + (z - z0) * (ny * nx);
   }
-  __device__ __forceinline__ const float* yp(int64_t z) const {
+  __device__ __forceinline__ const T* yp(int64_t z) const {
     const bool s1 = nseg > 1 && z >= zs[1], s2 = nseg > 2 && z >= zs[2];
-    const float* b = s2 ? ys[2] : (s1 ? ys[1] : ys[0]);
+    const T* b = s2 ? ys[2] : (s1 ? ys[1] : ys[0]);
     const int64_t z0 = s2 ? zs[2] : (s1 ? zs[1] : zs[0]);
     return b + (z - z0) * (ny * nx);
   }
@@ -179,17 +181,18 @@ struct Field3 {
 #if defined(__CUDACC__)
 // Sequential plane cursor over a Field3 (z increasing by one per step): pointer increments, with
 // the segment base re-derived only when a segment boundary is crossed.
+template <typename T>
 struct PlaneCursor {
-  const float* x;
-  const float* y;
+  const T* x;
+  const T* y;
   int64_t z, next_seg;
-  __device__ __forceinline__ void init(const Field3& f, int64_t z0, int64_t off) {
+  __device__ __forceinline__ void init(const Field3<T>& f, int64_t z0, int64_t off) {
     z = z0;
     x = f.xp(z0) + off;
     y = f.yp(z0) + off;
     next_seg = (f.nseg > 1 && z0 < f.zs[1]) ? f.zs[1] : ((f.nseg > 2 && z0 < f.zs[2]) ? f.zs[2] : INT64_MAX);
   }
-  __device__ __forceinline__ void advance(const Field3& f, int64_t off) {
+  __device__ __forceinline__ void advance(const Field3<T>& f, int64_t off) {
     ++z;
     if (z == next_seg) init(f, z, off);
     else { x += f.ny * f.nx; y += f.ny * f.nx; }
@@ -198,27 +201,36 @@ struct PlaneCursor {
 
 // Lighter cursor for hot loops: plane pointers plus the number of planes left in the current
 // segment (32-bit); the caller passes the next plane's index only for the rare re-init.
+template <typename T>
 struct SegCursor {
-  const float* x;
-  const float* y;
+  const T* x;
+  const T* y;
   int left;
-  __device__ __forceinline__ void init(const Field3& f, int64_t z0, int64_t off = 0) {
+  __device__ __forceinline__ void init(const Field3<T>& f, int64_t z0, int64_t off = 0) {
     x = f.xp(z0) + off;
     y = f.yp(z0) + off;
     const int64_t last = f.nseg == 1 ? f.zs[1] : (f.nseg == 2 ? f.zs[2] : f.zs[3]);   // static indices
     const int64_t e = (f.nseg > 1 && z0 < f.zs[1]) ? f.zs[1] : ((f.nseg > 2 && z0 < f.zs[2]) ? f.zs[2] : last);
     left = (int)(e - z0 < INT32_MAX ? e - z0 : INT32_MAX);
   }
-  __device__ __forceinline__ void advance(const Field3& f, int64_t znext, int64_t off = 0) {
+  __device__ __forceinline__ void advance(const Field3<T>& f, int64_t znext, int64_t off = 0) {
     if (--left <= 0) init(f, znext, off);
     else { x += f.ny * f.nx; y += f.ny * f.nx; }
   }
   // same with the plane stride (ny * nx) precomputed by the caller
-  __device__ __forceinline__ void advance_by(const Field3& f, int64_t znext, int64_t off, int64_t plane) {
+  __device__ __forceinline__ void advance_by(const Field3<T>& f, int64_t znext, int64_t off, int64_t plane) {
     if (--left <= 0) init(f, znext, off);
     else { x += plane; y += plane; }
   }
 };
+
+// Element-type helpers: exact min / max in the input type, a (x, y) sample pair.
+__device__ __forceinline__ float tmin(float a, float b) { return fminf(a, b); }
+__device__ __forceinline__ float tmax(float a, float b) { return fmaxf(a, b); }
+__device__ __forceinline__ double tmin(double a, double b) { return fmin(a, b); }
+__device__ __forceinline__ double tmax(double a, double b) { return fmax(a, b); }
+template <typename T>
+struct alignas(2 * sizeof(T)) Pair { T x, y; };
 #endif
 
 struct SsimParams {
@@ -362,6 +374,24 @@ __device__ __forceinline__ float4 ld_stream_f4(const float4* p) {
   float4 r;
   asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
                : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(p));
+  return r;
+}
+
+// One 128-bit vector of the input type: 4 floats or 2 doubles, streamed past L1.
+template <typename T>
+struct Vec16 {
+  static constexpr int N = 16 / (int)sizeof(T);
+  T e[N];
+};
+__device__ __forceinline__ Vec16<float> ld_stream16(const float* p) {
+  const float4 v = ld_stream_f4(reinterpret_cast<const float4*>(p));
+  Vec16<float> r;
+  r.e[0] = v.x; r.e[1] = v.y; r.e[2] = v.z; r.e[3] = v.w;
+  return r;
+}
+__device__ __forceinline__ Vec16<double> ld_stream16(const double* p) {
+  Vec16<double> r;
+  asm volatile("ld.global.nc.L1::no_allocate.v2.f64 {%0,%1}, [%2];" : "=d"(r.e[0]), "=d"(r.e[1]) : "l"(p));
   return r;
 }
 #endif

@@ -14,22 +14,24 @@ namespace czc {
 // Per-thread accumulator: sums about the thread's first element (kx, ky, ke).  The element count
 // is implicit (counted per vector), so no per-element work is spent on it.
 
+template <typename T>
 struct P1Acc {
   double kx, ky, ke;
   double sa, sb, sc, saa, sbb, sab, scc, sae;
   double emin, emax, pmin, pmax, spwr;
   double pthr_hi, pthr_lo;          // candidate thresholds for the exact pwr extrema
   unsigned npwr;                    // count of x != 0 (per thread, < 2^32)
-  float xmin, xmax;
+  T xmin, xmax;                     // exact, in the input type
 };
 
-__device__ __forceinline__ void acc_init(P1Acc& a, float kxf, float kyf) {
+template <typename T>
+__device__ __forceinline__ void acc_init(P1Acc<T>& a, T kxf, T kyf) {
   a.kx = kxf; a.ky = kyf; a.ke = (double)kyf - (double)kxf;
   a.sa = a.sb = a.sc = a.saa = a.sbb = a.sab = a.scc = a.sae = 0;
   a.emin = dinf(); a.emax = -dinf(); a.pmin = dinf(); a.pmax = -dinf(); a.spwr = 0;
   a.pthr_hi = -dinf(); a.pthr_lo = dinf();
   a.npwr = 0;
-  a.xmin = finf(); a.xmax = -finf();
+  a.xmin = (T)dinf(); a.xmax = -(T)dinf();
 }
 
 
@@ -42,8 +44,11 @@ __device__ __forceinline__ void acc_init(P1Acc& a, float kxf, float kyf) {
 // Q (1 - 1e-12) and pmax <= RN(Q) for a larger true quotient Q), and lower the minimum only if
 // q~ < thr_lo = pmin (1 + 1e-10); a zero minimum admits no further candidate (thr_lo = 0), a zero
 // maximum admits only q~ > 0.  Returns whether this element is a candidate; candidates are
-// resolved per vector, warp-uniformly (see acc_vec).
-__device__ __forceinline__ bool acc_elem(P1Acc& a, float xf, float yf, double& ae_out, double& ax_out) {
+// resolved per vector, warp-uniformly (see acc_vec).  float64 inputs: e = y - x is rounded to
+// double exactly as in the oracle (R1), and |x| outside [1e-290, 1e290] (where the approximate
+// reciprocal flushes) takes the IEEE quotient.
+template <typename T>
+__device__ __forceinline__ bool acc_elem(P1Acc<T>& a, T xf, T yf, double& ae_out, double& ax_out) {
   const double x = xf, y = yf;
   const double e = y - x;
   const double da = x - a.kx, db = y - a.ky, dc = e - a.ke;
@@ -56,11 +61,12 @@ __device__ __forceinline__ bool acc_elem(P1Acc& a, float xf, float yf, double& a
   a.sae += ae;
   a.emin = e < a.emin ? e : a.emin;
   a.emax = e > a.emax ? e : a.emax;
-  a.xmin = fminf(a.xmin, xf);
-  a.xmax = fmaxf(a.xmax, xf);
-  const bool nz = xf != 0.0f;
+  a.xmin = tmin(a.xmin, xf);
+  a.xmax = tmax(a.xmax, xf);
+  const bool nz = xf != (T)0;
   const double ax = nz ? fabs(x) : 1.0;
-  const double qa = nz ? ae * rcp_newton1(ax) : 0.0;
+  double qa = nz ? ae * rcp_newton1(ax) : 0.0;
+  if (sizeof(T) == 8 && !(ax >= 1e-290 && ax <= 1e290)) qa = ae / ax;
   a.spwr += qa;
   a.npwr += nz ? 1u : 0u;
   ae_out = ae;
@@ -68,27 +74,31 @@ __device__ __forceinline__ bool acc_elem(P1Acc& a, float xf, float yf, double& a
   return nz && (qa > a.pthr_hi || qa < a.pthr_lo);
 }
 
-__device__ __forceinline__ void acc_resolve(P1Acc& a, double ae, double ax) {
+template <typename T>
+__device__ __forceinline__ void acc_resolve(P1Acc<T>& a, double ae, double ax) {
   const double q = ae / ax;                          // IEEE, correctly rounded
   if (q > a.pmax) { a.pmax = q; a.pthr_hi = q * (1.0 - 1e-10); }
   if (q < a.pmin) { a.pmin = q; a.pthr_lo = q * (1.0 + 1e-10); }   // q = 0 -> thr_lo = 0
 }
 
-__device__ __forceinline__ void acc_vec(P1Acc& a, float4 xv, float4 yv) {
-  double ae0, ax0, ae1, ax1, ae2, ax2, ae3, ax3;
-  const bool c0 = acc_elem(a, xv.x, yv.x, ae0, ax0);
-  const bool c1 = acc_elem(a, xv.y, yv.y, ae1, ax1);
-  const bool c2 = acc_elem(a, xv.z, yv.z, ae2, ax2);
-  const bool c3 = acc_elem(a, xv.w, yv.w, ae3, ax3);
+template <typename T>
+__device__ __forceinline__ void acc_vec(P1Acc<T>& a, const Vec16<T>& xv, const Vec16<T>& yv) {
+  constexpr int N = Vec16<T>::N;
+  double ae[N], ax[N];
+  bool c[N], any = false;
+#pragma unroll
+  for (int j = 0; j < N; j++) {
+    c[j] = acc_elem(a, xv.e[j], yv.e[j], ae[j], ax[j]);
+    any |= c[j];
+  }
   // Warp-uniform resolve; in a full warp the lanes then share their extrema (a lane may report
   // the warp's maximum / minimum: merging takes max / min, so the result is unchanged), which
   // makes later candidates ~32x rarer than with per-lane thresholds.
   const unsigned m = __activemask();
-  if (__any_sync(m, c0 | c1 | c2 | c3)) {
-    if (c0) acc_resolve(a, ae0, ax0);
-    if (c1) acc_resolve(a, ae1, ax1);
-    if (c2) acc_resolve(a, ae2, ax2);
-    if (c3) acc_resolve(a, ae3, ax3);
+  if (__any_sync(m, any)) {
+#pragma unroll
+    for (int j = 0; j < N; j++)
+      if (c[j]) acc_resolve(a, ae[j], ax[j]);
     if (m == 0xffffffffu) {
       double mx = a.pmax, mn = a.pmin;
 #pragma unroll
@@ -103,12 +113,14 @@ __device__ __forceinline__ void acc_vec(P1Acc& a, float4 xv, float4 yv) {
   }
 }
 
-__device__ __forceinline__ void acc_scalar(P1Acc& a, float xf, float yf) {
+template <typename T>
+__device__ __forceinline__ void acc_scalar(P1Acc<T>& a, T xf, T yf) {
   double ae, ax;
   if (acc_elem(a, xf, yf, ae, ax)) acc_resolve(a, ae, ax);
 }
 
-__device__ __forceinline__ P1State acc_to_state(const P1Acc& a, double n) {
+template <typename T>
+__device__ __forceinline__ P1State acc_to_state(const P1Acc<T>& a, double n) {
   P1State s;
   p1_empty(s);
   s.sae = a.sae; s.spwr = a.spwr; s.npwr = (double)a.npwr;
@@ -157,39 +169,41 @@ __device__ __forceinline__ P1State block_merge(P1State s) {
   return s;
 }
 
-// VEC: x and y share the same 16-byte misalignment; elements [head, head + 4*nvec) are read as
-// float4, the <= 6 leftovers (prologue [0, head) and tail) by threads 0..nleft-1.
-template <bool VEC>
+// VEC: x and y share the same 16-byte misalignment; elements [head, head + VN*nvec) are read as
+// 128-bit vectors (VN = 4 floats or 2 doubles), the leftovers (prologue [0, head) and tail) by
+// threads 0..nleft-1.
+template <typename T, bool VEC>
 __global__ void __launch_bounds__(kP1Threads)
-p1_kernel(const float* __restrict__ x, const float* __restrict__ y, int64_t n, int64_t head,
+p1_kernel(const T* __restrict__ x, const T* __restrict__ y, int64_t n, int64_t head,
           P1State* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket) {
+  constexpr int VN = Vec16<T>::N;
   const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
-  const int64_t nvec = VEC ? (n - head) / 4 : 0;
-  const int64_t tail0 = head + 4 * nvec;
+  const int64_t nvec = VEC ? (n - head) / VN : 0;
+  const int64_t tail0 = head + VN * nvec;
   const int64_t nleft = VEC ? head + (n - tail0) : n;   // scalar elements
   auto left_index = [&](int64_t k) -> int64_t { return VEC ? (k < head ? k : tail0 + (k - head)) : k; };
 
-  P1Acc a;
+  P1Acc<T> a;
   int64_t first = -1;   // anchor = the thread's first element
-  if (VEC && gtid < nvec) first = head + 4 * gtid;
+  if (VEC && gtid < nvec) first = head + VN * gtid;
   else if (gtid < nleft) first = left_index(gtid);
-  acc_init(a, first >= 0 ? x[first] : 0.0f, first >= 0 ? y[first] : 0.0f);
+  acc_init(a, first >= 0 ? x[first] : (T)0, first >= 0 ? y[first] : (T)0);
 
   int64_t cnt = 0;                                 // elements processed by this thread
   if (VEC) {
-    const float4* x4 = reinterpret_cast<const float4*>(x + head);
-    const float4* y4 = reinterpret_cast<const float4*>(y + head);
+    const T* x4 = x + head;
+    const T* y4 = y + head;
     int64_t v = gtid;
-    if (gtid < nvec) cnt = 4 * ((nvec - 1 - gtid) / gsz + 1);
+    if (gtid < nvec) cnt = VN * ((nvec - 1 - gtid) / gsz + 1);
     // software pipeline: the next two vectors' loads are in flight while two are processed
     if (v + gsz < nvec) {
-      float4 xa = ld_stream_f4(x4 + v), ya = ld_stream_f4(y4 + v);
-      float4 xb = ld_stream_f4(x4 + v + gsz), yb = ld_stream_f4(y4 + v + gsz);
+      Vec16<T> xa = ld_stream16(x4 + VN * v), ya = ld_stream16(y4 + VN * v);
+      Vec16<T> xb = ld_stream16(x4 + VN * (v + gsz)), yb = ld_stream16(y4 + VN * (v + gsz));
       v += 2 * gsz;
       for (; v + gsz < nvec; v += 2 * gsz) {
-        const float4 xc = ld_stream_f4(x4 + v), yc = ld_stream_f4(y4 + v);
-        const float4 xd = ld_stream_f4(x4 + v + gsz), yd = ld_stream_f4(y4 + v + gsz);
+        const Vec16<T> xc = ld_stream16(x4 + VN * v), yc = ld_stream16(y4 + VN * v);
+        const Vec16<T> xd = ld_stream16(x4 + VN * (v + gsz)), yd = ld_stream16(y4 + VN * (v + gsz));
         acc_vec(a, xa, ya);
         acc_vec(a, xb, yb);
         xa = xc; ya = yc; xb = xd; yb = yd;
@@ -197,7 +211,7 @@ p1_kernel(const float* __restrict__ x, const float* __restrict__ y, int64_t n, i
       acc_vec(a, xa, ya);
       acc_vec(a, xb, yb);
     }
-    for (; v < nvec; v += gsz) acc_vec(a, ld_stream_f4(x4 + v), ld_stream_f4(y4 + v));
+    for (; v < nvec; v += gsz) acc_vec(a, ld_stream16(x4 + VN * v), ld_stream16(y4 + VN * v));
     if (gtid < nleft) {
       const int64_t i = left_index(gtid);
       acc_scalar(a, x[i], y[i]);
@@ -231,24 +245,37 @@ p1_kernel(const float* __restrict__ x, const float* __restrict__ y, int64_t n, i
   }
 }
 
-// Host launcher.  Returns the cuda error of the launch.
-cudaError_t launch_p1(const float* x, const float* y, int64_t n, int grid_cap, P1State* parts,
-                      DevResults* res, unsigned int* ticket, cudaStream_t st) {
+// 128-bit vector path: both arrays element-aligned with the same 16-byte misalignment; head =
+// elements before the first aligned vector.
+template <typename T>
+static bool vec_head(const T* x, const T* y, int64_t n, int64_t* head) {
   const uintptr_t ax = reinterpret_cast<uintptr_t>(x), ay = reinterpret_cast<uintptr_t>(y);
-  const bool vec = (ax % 16) == (ay % 16) && (ax % 4) == 0;
+  const bool vec = (ax % 16) == (ay % 16) && (ax % sizeof(T)) == 0;
+  int64_t h = vec ? (int64_t)(((16 - ax % 16) % 16) / sizeof(T)) : 0;
+  *head = h > n ? n : h;
+  return vec;
+}
+
+// Host launcher.  Returns the cuda error of the launch.
+template <typename T>
+cudaError_t launch_p1(const T* x, const T* y, int64_t n, int grid_cap, P1State* parts,
+                      DevResults* res, unsigned int* ticket, cudaStream_t st) {
   int64_t head = 0;
-  if (vec) head = (int64_t)(((16 - ax % 16) % 16) / 4);
-  if (head > n) head = n;
-  const int64_t work = vec ? ((n - head) / 4 + 8) : n;
+  const bool vec = vec_head(x, y, n, &head);
+  const int64_t work = vec ? ((n - head) / Vec16<T>::N + 8) : n;
   int64_t blocks = (work + kP1Threads - 1) / kP1Threads;
   if (blocks > grid_cap) blocks = grid_cap;
   if (blocks < 1) blocks = 1;
   if (vec)
-    p1_kernel<true><<<(unsigned)blocks, kP1Threads, 0, st>>>(x, y, n, head, parts, res, ticket);
+    p1_kernel<T, true><<<(unsigned)blocks, kP1Threads, 0, st>>>(x, y, n, head, parts, res, ticket);
   else
-    p1_kernel<false><<<(unsigned)blocks, kP1Threads, 0, st>>>(x, y, n, head, parts, res, ticket);
+    p1_kernel<T, false><<<(unsigned)blocks, kP1Threads, 0, st>>>(x, y, n, head, parts, res, ticket);
   return cudaGetLastError();
 }
+template cudaError_t launch_p1<float>(const float*, const float*, int64_t, int, P1State*, DevResults*,
+                                      unsigned int*, cudaStream_t);
+template cudaError_t launch_p1<double>(const double*, const double*, int64_t, int, P1State*, DevResults*,
+                                       unsigned int*, cudaStream_t);
 
 // ------------------------------------------------------------------------------------------------
 // Error PDF / pwr-error PDF (Table I Category I, L107; reading R24).  One pass after P1: the bins
@@ -276,36 +303,37 @@ __device__ __forceinline__ int pdf_bin_err(double e, const PdfRange& r) {
 }
 __device__ __forceinline__ int pdf_bin_pwr(double ae, double ax, const PdfRange& r) {
   if (!(r.rw > 0)) return 0;
-  const double qa = ae * rcp_newton1(ax);
+  double qa = ae * rcp_newton1(ax);
+  if (!(ax >= 1e-290 && ax <= 1e290)) qa = ae / ax;         // float64 inputs only
   const double t = (qa - r.lo) * r.rw;
   if (pdf_near_edge(t, 1e-10 * (fabs(qa) * r.rw + 1.0))) return pdf_clamp((ae / ax - r.lo) / r.w, r.nb);
   return pdf_clamp(t, r.nb);
 }
 
-template <bool VEC>
+template <typename T, bool VEC>
 __global__ void __launch_bounds__(kP1Threads)
-pdf_kernel(const float* __restrict__ x, const float* __restrict__ y, int64_t n, int64_t head, int nb,
+pdf_kernel(const T* __restrict__ x, const T* __restrict__ y, int64_t n, int64_t head, int nb,
            DevResults* __restrict__ res) {
+  constexpr int VN = Vec16<T>::N;
   __shared__ unsigned int h[2][CZC_PDF_MAX_BINS];
   for (int i = threadIdx.x; i < 2 * CZC_PDF_MAX_BINS; i += blockDim.x) (&h[0][0])[i] = 0u;
   __syncthreads();
   const P1State& g = res->p1g;
   const PdfRange re = pdf_range(g.emin, g.emax, nb);
   const PdfRange rp = pdf_range(g.pmin, g.pmax, nb);
-  auto elem = [&](float xf, float yf) {
+  auto elem = [&](T xf, T yf) {
     const double xd = xf, e = (double)yf - xd;
     atomicAdd(&h[0][pdf_bin_err(e, re)], 1u);
-    if (xf != 0.0f) atomicAdd(&h[1][pdf_bin_pwr(fabs(e), fabs(xd), rp)], 1u);
+    if (xf != (T)0) atomicAdd(&h[1][pdf_bin_pwr(fabs(e), fabs(xd), rp)], 1u);
   };
   const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
   if (VEC) {
-    const int64_t nvec = (n - head) / 4, tail0 = head + 4 * nvec;
-    const float4* x4 = reinterpret_cast<const float4*>(x + head);
-    const float4* y4 = reinterpret_cast<const float4*>(y + head);
+    const int64_t nvec = (n - head) / VN, tail0 = head + VN * nvec;
     for (int64_t v = gtid; v < nvec; v += gsz) {
-      const float4 a = ld_stream_f4(x4 + v), b = ld_stream_f4(y4 + v);
-      elem(a.x, b.x); elem(a.y, b.y); elem(a.z, b.z); elem(a.w, b.w);
+      const Vec16<T> a = ld_stream16(x + head + VN * v), b = ld_stream16(y + head + VN * v);
+#pragma unroll
+      for (int j = 0; j < VN; j++) elem(a.e[j], b.e[j]);
     }
     if (gtid < head) elem(x[gtid], y[gtid]);
     if (gtid < n - tail0) elem(x[tail0 + gtid], y[tail0 + gtid]);
@@ -321,23 +349,23 @@ pdf_kernel(const float* __restrict__ x, const float* __restrict__ y, int64_t n, 
 }
 
 // Zeroes the counts, then histograms x[0, n), y[0, n) into res->rec.pdf (needs res->p1g).
-cudaError_t launch_pdf(const float* x, const float* y, int64_t n, int nb, int grid_cap, DevResults* res,
+template <typename T>
+cudaError_t launch_pdf(const T* x, const T* y, int64_t n, int nb, int grid_cap, DevResults* res,
                        cudaStream_t st) {
   cudaError_t e = cudaMemsetAsync(res->rec.pdf, 0, sizeof(res->rec.pdf), st);
   if (e != cudaSuccess) return e;
-  const uintptr_t ax = reinterpret_cast<uintptr_t>(x), ay = reinterpret_cast<uintptr_t>(y);
-  const bool vec = (ax % 16) == (ay % 16) && (ax % 4) == 0;
   int64_t head = 0;
-  if (vec) head = (int64_t)(((16 - ax % 16) % 16) / 4);
-  if (head > n) head = n;
-  const int64_t work = vec ? ((n - head) / 4 + 8) : n;
+  const bool vec = vec_head(x, y, n, &head);
+  const int64_t work = vec ? ((n - head) / Vec16<T>::N + 8) : n;
   int64_t blocks = (work + kP1Threads - 1) / kP1Threads;
   if (blocks > grid_cap) blocks = grid_cap;
   if (blocks < 1) blocks = 1;
-  if (vec) pdf_kernel<true><<<(unsigned)blocks, kP1Threads, 0, st>>>(x, y, n, head, nb, res);
-  else pdf_kernel<false><<<(unsigned)blocks, kP1Threads, 0, st>>>(x, y, n, head, nb, res);
+  if (vec) pdf_kernel<T, true><<<(unsigned)blocks, kP1Threads, 0, st>>>(x, y, n, head, nb, res);
+  else pdf_kernel<T, false><<<(unsigned)blocks, kP1Threads, 0, st>>>(x, y, n, head, nb, res);
   return cudaGetLastError();
 }
+template cudaError_t launch_pdf<float>(const float*, const float*, int64_t, int, int, DevResults*, cudaStream_t);
+template cudaError_t launch_pdf<double>(const double*, const double*, int64_t, int, int, DevResults*, cudaStream_t);
 
 // Slab mode: merge the allgathered per-rank states in rank order (every rank runs the same code
 // on the same bytes, so all ranks hold identical results).
@@ -356,7 +384,7 @@ cudaError_t launch_p1_combine(const P1State* states, int count, DevResults* res,
 
 int p1_max_blocks_per_sm() {
   int nb = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, p1_kernel<true>, kP1Threads, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, p1_kernel<float, true>, kP1Threads, 0);
   return nb > 0 ? nb : 1;
 }
 

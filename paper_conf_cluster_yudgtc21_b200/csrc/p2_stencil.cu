@@ -84,9 +84,9 @@ struct SumOp {
 // grid: (ceil(nx/BX), ceil(ny/BY), zchunks); block (BX, BY), BX * BY = 256.
 //   3-D: <true, true, 32, 8>; 2-D row view (slow axis = rows): <true, false, 256, 1>;
 //   1-D: <false, false, 256, 1>.
-template <bool ZA, bool YA, int BX, int BY>
+template <typename T, bool ZA, bool YA, int BX, int BY>
 __global__ void __launch_bounds__(BX * BY, 2)
-deriv_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+deriv_kernel(Field3<T> s, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
              unsigned int* __restrict__ ticket) {
   constexpr int kTX = BX, kTY = BY;
   // halo cells of one plane tile: the full ring with a y axis, the two x ends without
@@ -121,8 +121,8 @@ deriv_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __res
   const int64_t hcol = hown ? hy * s.nx + hx : 0;
 
   double xm = 0, x0 = 0, ym = 0, y0 = 0;
-  float nxv = 0.f, nyv = 0.f, nhx = 0.f, nhy = 0.f;   // prefetched: own at z+1, halo at z
-  PlaneCursor cown, chalo;                            // own column at z+2, halo cell at z+1
+  T nxv = 0, nyv = 0, nhx = 0, nhy = 0;               // prefetched: own at z+1, halo at z
+  PlaneCursor<T> cown, chalo;                         // own column at z+2, halo cell at z+1
   if (zb < ze) {
     if (own) {
       x0 = s.xp(zb)[col]; y0 = s.yp(zb)[col];
@@ -139,7 +139,7 @@ deriv_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __res
   for (int64_t z = zb; z < ze; z++) {
     const int buf = (int)((z - zb) & 1);
     const double xp = az ? (double)nxv : 0.0, yp = az ? (double)nyv : 0.0;
-    const float hxv = nhx, hyv = nhy;
+    const T hxv = nhx, hyv = nhy;
     // prefetch: own column at z+2, halo at z+1 (cursors advance one plane per step)
     if (own && az && z + 2 <= s.nz - 1 && z + 1 < ze) { nxv = __ldg(cown.x); nyv = __ldg(cown.y); cown.advance(s, col); }
     if (hown && z + 1 < ze) { nhx = __ldg(chalo.x); nhy = __ldg(chalo.y); chalo.advance(s, hcol); }
@@ -175,9 +175,9 @@ deriv_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __res
 // 3-D variant with two points per thread: threads (32, 4) cover a 32 x 8 tile, thread (tx, ty)
 // owns rows ty and ty + 4.  The 25 accumulators are shared by both points (half the registers
 // per point) and the two independent stencils double each warp's instruction-level parallelism.
-template <int PTS>
-__global__ void __launch_bounds__(kTX * kTY / PTS, 4)
-deriv3_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+template <typename T, int PTS>
+__global__ void __launch_bounds__(kTX * kTY / PTS, sizeof(T) == 4 ? 4 : 3)
+deriv3_kernel(Field3<T> s, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
               unsigned int* __restrict__ ticket) {
   constexpr int RY = kTY / PTS;                    // thread rows
   constexpr int kHalo = 2 * (kTX + 2) + 2 * kTY;
@@ -213,12 +213,12 @@ deriv3_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __re
   const int64_t hcol = hown ? hy * s.nx + hx : 0;
 
   double xm[PTS], x0[PTS], ym[PTS], y0[PTS];
-  float nxv[PTS], nyv[PTS];
-  float nhx = 0.f, nhy = 0.f;
-  SegCursor cown, chalo;                          // own column (row 0) at z+2, halo cell at z+1
+  T nxv[PTS], nyv[PTS];
+  T nhx = 0, nhy = 0;
+  SegCursor<T> cown, chalo;                          // own column (row 0) at z+2, halo cell at z+1
   const int64_t plane = s.ny * s.nx;
 #pragma unroll
-  for (int p = 0; p < PTS; p++) { xm[p] = x0[p] = ym[p] = y0[p] = 0; nxv[p] = nyv[p] = 0.f; }
+  for (int p = 0; p < PTS; p++) { xm[p] = x0[p] = ym[p] = y0[p] = 0; nxv[p] = nyv[p] = 0; }
   if (zb < ze) {
 #pragma unroll
     for (int p = 0; p < PTS; p++) {
@@ -249,7 +249,7 @@ deriv3_kernel(Field3 s, int zchunk, double* __restrict__ parts, DevResults* __re
     double xp[PTS], yp[PTS];
 #pragma unroll
     for (int p = 0; p < PTS; p++) { xp[p] = (double)nxv[p]; yp[p] = (double)nyv[p]; }
-    const float hxv = nhx, hyv = nhy;
+    const T hxv = nhx, hyv = nhy;
     if (i + 1 < n) {
 #pragma unroll
       for (int p = 0; p < PTS; p++)
@@ -336,15 +336,15 @@ __device__ __forceinline__ void ac_finish(double (&acc)[TM], double* parts, doub
 // ahead of the walk: QD loads stay in flight in a register queue whose slot u (of the QD-unrolled
 // loop) holds position i0 + u, so both the queue and the ring (QD is a multiple of TM) rotate
 // statically.
-template <int TM, int QD, typename Next>
+template <typename T, int TM, int QD, typename Next>
 __device__ __forceinline__ void walk_line(Next next, int64_t lo, int64_t hi, int64_t end, double mu,
                                           bool own, double (&ring)[TM], double (&acc)[TM]) {
   static_assert(QD % TM == 0, "queue depth must be a multiple of the ring length");
-  float qx[QD], qy[QD];
+  T qx[QD], qy[QD];
 #pragma unroll
   for (int u = 0; u < QD; u++) {
-    qx[u] = 0.f; qy[u] = 0.f;
-    if (own && lo + u < end) { const float2 v = next(); qx[u] = v.x; qy[u] = v.y; }
+    qx[u] = 0; qy[u] = 0;
+    if (own && lo + u < end) { const Pair<T> v = next(); qx[u] = v.x; qy[u] = v.y; }
   }
   for (int64_t i0 = lo; i0 < end; i0 += QD) {
 #pragma unroll
@@ -352,7 +352,7 @@ __device__ __forceinline__ void walk_line(Next next, int64_t lo, int64_t hi, int
       const int64_t i = i0 + u;
       if (i < end) {
         const double eps = ((double)qy[u] - (double)qx[u]) - mu;
-        if (own && i + QD < end) { const float2 v = next(); qx[u] = v.x; qy[u] = v.y; }
+        if (own && i + QD < end) { const Pair<T> v = next(); qx[u] = v.x; qy[u] = v.y; }
         walk_step<TM>(ring, acc, eps, i < hi, u % TM);
       }
     }
@@ -367,19 +367,19 @@ __device__ __forceinline__ void walk_line(Next next, int64_t lo, int64_t hi, int
 // synchronises once and the consumed half of the ring is refilled S positions ahead.  Threads past
 // the row end read stale slot data; their products are discarded by walk_mask (lim = 0).
 constexpr int kWalkThreads = 256;
-template <int TM>
+template <typename T, int TM>
 struct BulkWalkSmem {
   static constexpr int S = 2 * TM;
-  float x[S][kWalkThreads];
-  float y[S][kWalkThreads];
+  T x[S][kWalkThreads];
+  T y[S][kWalkThreads];
   uint64_t bar[S];
 };
 
-// RowPtr(i) -> (const float* xrow, const float* yrow) for position i (already offset to x0).
+// RowPtr(i) -> (const T* xrow, const T* yrow) for position i (already offset to x0).
 // Positions are tracked relative to lo in 32 bits.  Lane v < S of warp 0 issues slot v's copies
 // (after the barrier that frees the slot), so the refill costs one bulk copy pair per lane.
-template <int TM, typename RowPtr>
-__device__ __forceinline__ void bulk_walk(BulkWalkSmem<TM>& sm, RowPtr row_ptr, uint32_t bytes, int64_t lo,
+template <typename T, int TM, typename RowPtr>
+__device__ __forceinline__ void bulk_walk(BulkWalkSmem<T, TM>& sm, RowPtr row_ptr, uint32_t bytes, int64_t lo,
                                           int64_t hi, int64_t end, double mu,
                                           double (&ring)[TM], double (&acc)[TM]) {
   constexpr int S = 2 * TM;
@@ -392,8 +392,8 @@ __device__ __forceinline__ void bulk_walk(BulkWalkSmem<TM>& sm, RowPtr row_ptr, 
   }
   __syncthreads();
   auto issue = [&](int slot, int j) {
-    const float* xr;
-    const float* yr;
+    const T* xr;
+    const T* yr;
     row_ptr(lo + j, xr, yr);
     mbar_expect_tx(&sm.bar[slot], 2 * bytes);
     bulk_g2s(sm.x[slot], xr, bytes, &sm.bar[slot]);
@@ -421,12 +421,12 @@ __device__ __forceinline__ void bulk_walk(BulkWalkSmem<TM>& sm, RowPtr row_ptr, 
 }
 
 // z-walk, TMA: block = 256 consecutive x of row y; grid (x tiles, ny, z chunks).
-template <int TM>
+template <typename E, int TM>
 __global__ void __launch_bounds__(kWalkThreads, 3)
-ac_zwalk_tma(Field3 s, int T, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+ac_zwalk_tma(Field3<E> s, int T, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
              unsigned int* __restrict__ ticket) {
   extern __shared__ __align__(128) unsigned char walk_smem[];
-  BulkWalkSmem<TM>& sm = *reinterpret_cast<BulkWalkSmem<TM>*>(walk_smem);
+  BulkWalkSmem<E, TM>& sm = *reinterpret_cast<BulkWalkSmem<E, TM>*>(walk_smem);
   const int64_t x0 = (int64_t)blockIdx.x * kWalkThreads, gy = blockIdx.y;
   const int64_t gx = x0 + threadIdx.x;
   const double mu = res->p1g.me;
@@ -444,16 +444,16 @@ ac_zwalk_tma(Field3 s, int T, int zchunk, double* __restrict__ parts, DevResults
   double ring[TM], acc[TM];
 #pragma unroll
   for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
-  bulk_walk<TM>(sm, [&](int64_t z, const float*& xr, const float*& yr) { xr = s.xp(z) + off; yr = s.yp(z) + off; },
-                (uint32_t)(ncols * 4), lo, hi, end, mu, ring, acc);
+  bulk_walk<E, TM>(sm, [&](int64_t z, const E*& xr, const E*& yr) { xr = s.xp(z) + off; yr = s.yp(z) + off; },
+                   (uint32_t)(ncols * sizeof(E)), lo, hi, end, mu, ring, acc);
   walk_mask<TM>(acc, own ? (int)m : 0);
   ac_finish<TM>(acc, parts, res->rec.ac[0], ticket);
 }
 
 // z-walk: thread <-> column (y, x); block 32 x 8 columns; grid.z chunks of owned planes.
-template <int TM>
+template <typename E, int TM>
 __global__ void __launch_bounds__(256)
-ac_zwalk(Field3 s, int T, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+ac_zwalk(Field3<E> s, int T, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
          unsigned int* __restrict__ ticket) {
   const int64_t gx = (int64_t)blockIdx.x * kTX + threadIdx.x, gy = (int64_t)blockIdx.y * kTY + threadIdx.y;
   const double mu = res->p1g.me;
@@ -470,10 +470,10 @@ ac_zwalk(Field3 s, int T, int zchunk, double* __restrict__ parts, DevResults* __
   double ring[TM], acc[TM];
 #pragma unroll
   for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
-  PlaneCursor cur;
+  PlaneCursor<E> cur;
   if (own && lo < end) cur.init(s, lo, col);
-  walk_line<TM, 2 * TM>([&]() {         // read the cursor's plane, then step it (never read past end)
-    const float2 v = make_float2(__ldg(cur.x), __ldg(cur.y));
+  walk_line<E, TM, 2 * TM>([&]() {      // read the cursor's plane, then step it (never read past end)
+    const Pair<E> v = {__ldg(cur.x), __ldg(cur.y)};
     cur.advance(s, col);
     return v;
   }, lo, hi, end, mu, own, ring, acc);
@@ -487,7 +487,7 @@ ac_zwalk(Field3 s, int T, int zchunk, double* __restrict__ parts, DevResults* __
 // 32 rows per warp touch 32 lines per load instruction, each line reused over 8 loads (L1).
 template <int TM>
 __global__ void __launch_bounds__(256)
-ac_xwalk_vec(Field3 s, int T, int xchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+ac_xwalk_vec(Field3<float> s, int T, int xchunk, double* __restrict__ parts, DevResults* __restrict__ res,
              unsigned int* __restrict__ ticket) {
   constexpr int LCM = (TM % 4 == 0) ? TM : ((TM % 2 == 0) ? 2 * TM : 4 * TM);   // lcm(4, TM)
   constexpr int NV = LCM / 4;                        // float4 vectors per ring period
@@ -540,9 +540,9 @@ ac_xwalk_vec(Field3 s, int T, int xchunk, double* __restrict__ parts, DevResults
 // coalesced into a warp-private shared-memory tile (transpose), then lane l walks row l.  The
 // staged row's (z, y) advance incrementally (no divisions in the loop).
 constexpr int kXWarps = 4;   // 4 warps x 32 rows per block (tile: 4 x 32 x <=33 doubles <= 34 KB)
-template <int TM>
+template <typename E, int TM>
 __global__ void __launch_bounds__(kXWarps * 32)
-ac_xwalk_smem(Field3 s, int T, int xchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+ac_xwalk_smem(Field3<E> s, int T, int xchunk, double* __restrict__ parts, DevResults* __restrict__ res,
          unsigned int* __restrict__ ticket) {
   constexpr int SEG = (32 / TM) * TM;
   __shared__ double tile[kXWarps][32][SEG + 1];
@@ -569,8 +569,8 @@ ac_xwalk_smem(Field3 s, int T, int xchunk, double* __restrict__ parts, DevResult
   for (int64_t c0 = lo; c0 < end; c0 += SEG) {
     // stage 32 rows x SEG columns of eps, coalesced per row; rows advance (y, z) incrementally
     int64_t zr = zr0, yr = yr0;
-    const float* X = s.xp(zr) + yr * s.nx;
-    const float* Y = s.yp(zr) + yr * s.nx;
+    const E* X = s.xp(zr) + yr * s.nx;
+    const E* Y = s.yp(zr) + yr * s.nx;
     const int64_t c = c0 + lane;
     const bool cin = lane < SEG && c < end;
 #pragma unroll 4
@@ -619,20 +619,30 @@ ac_xwalk_smem(Field3 s, int T, int xchunk, double* __restrict__ parts, DevResult
 // one per block (a persistent grid of the resident block count): no tail wave, and the
 // assignment is static, so the result is deterministic.
 constexpr int kPlTX = 64, kPlTY = 32, kPlThreads = 256, kPlSeg = 8;
-template <int TM>
+template <typename T, int TM>
 struct PlaneTile {
   static_assert(TM % 2 == 0, "even lag templates only");
   static constexpr int HX = kPlTX + TM, HY = kPlTY + TM;
-  static constexpr int NV = (HX + 3) / 4;        // 16-byte groups per staged row
-  static constexpr int PF = 4 * NV;              // staged row pitch (floats), 16-byte multiple
+  static constexpr int EPG = 16 / (int)sizeof(T);        // elements per 16-byte group
+  static constexpr int NV = (HX + EPG - 1) / EPG;        // 16-byte groups per staged row
+  static constexpr int PF = EPG * NV;            // staged row pitch (elements), 16-byte multiple
   static constexpr int PE = (PF + 1) | 1;        // eps row pitch (doubles), odd: conflict-free columns
   double e[HY][PE];
-  float fx[HY][PF];
-  float fy[HY][PF];
+  T fx[HY][PF];
+  T fy[HY][PF];
 };
 
 __device__ __forceinline__ void cp_async4(unsigned dst, const void* src, int src_bytes) {
   asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
+}
+__device__ __forceinline__ void cp_async8(unsigned dst, const void* src, int src_bytes) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
+}
+// one element of the input type, zero-filled when `ok` is false
+template <typename T>
+__device__ __forceinline__ void cp_async_elem(unsigned dst, const T* src, bool ok) {
+  if (sizeof(T) == 4) cp_async4(dst, src, ok ? 4 : 0);
+  else cp_async8(dst, src, ok ? 8 : 0);
 }
 __device__ __forceinline__ void cp_async16(unsigned dst, const void* src, int src_bytes) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
@@ -640,20 +650,24 @@ __device__ __forceinline__ void cp_async16(unsigned dst, const void* src, int sr
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
 
-// Stage the window of one plane.  Warp w copies staged rows w, w + 8, ...; VEC: lane g < NV copies
-// the 16-byte group g of the row (vb = bytes of that group inside the field, fixed per thread);
+// Stage the window of one plane.  Warp w copies staged rows w, w + 8, ...; VEC: lane l copies the
+// 16-byte groups g = l, l + 32, ... of the row (vb = bytes of that group inside the field);
 // scalar: lanes copy single samples.  xt / yt point at the tile origin (y0, x0) of the plane.
-template <int TM, bool VEC>
-__device__ __forceinline__ void plane_stage(unsigned sfx, const float* xt, const float* yt, int64_t nx, int rv,
-                                            int cv, int vb, int warp, int lane) {
-  constexpr int HX = PlaneTile<TM>::HX, HY = PlaneTile<TM>::HY, NV = PlaneTile<TM>::NV, PF = PlaneTile<TM>::PF;
+template <typename T, int TM, bool VEC>
+__device__ __forceinline__ void plane_stage(unsigned sfx, const T* xt, const T* yt, int64_t nx, int rv,
+                                            int cv, int warp, int lane) {
+  using PT = PlaneTile<T, TM>;
+  constexpr int HX = PT::HX, HY = PT::HY, NV = PT::NV, PF = PT::PF, EPG = PT::EPG;
   constexpr int RS = kPlThreads / 32;                             // row stride
-  constexpr unsigned dy = (unsigned)(sizeof(float) * HY * PF);   // fx -> fy
+  constexpr unsigned dy = (unsigned)(sizeof(T) * HY * PF);       // fx -> fy
   if (VEC) {
-    if (lane < NV) {
-      const float* px = xt + warp * nx + 4 * lane;
-      const float* py = yt + warp * nx + 4 * lane;
-      unsigned d = sfx + (unsigned)(sizeof(float) * (warp * PF + 4 * lane));
+#pragma unroll
+    for (int g = lane; g < NV; g += 32) {
+      int vb = cv - EPG * g;
+      vb = vb <= 0 ? 0 : (vb >= EPG ? 16 : (int)sizeof(T) * vb);
+      const T* px = xt + warp * nx + EPG * g;
+      const T* py = yt + warp * nx + EPG * g;
+      unsigned d = sfx + (unsigned)(sizeof(T) * (warp * PF + EPG * g));
       for (int r = warp; r < HY; r += RS) {
         if (r < rv) {
           cp_async16(d, px, vb);
@@ -662,7 +676,7 @@ __device__ __forceinline__ void plane_stage(unsigned sfx, const float* xt, const
           cp_async16(d, xt, 0);
           cp_async16(d + dy, yt, 0);
         }
-        px += RS * nx; py += RS * nx; d += sizeof(float) * RS * PF;
+        px += RS * nx; py += RS * nx; d += sizeof(T) * RS * PF;
       }
     }
   } else {
@@ -673,9 +687,9 @@ __device__ __forceinline__ void plane_stage(unsigned sfx, const float* xt, const
         if (c < HX) {
           const bool ok = r < rv && c < cv;
           const int64_t o = ok ? r * nx + c : 0;
-          const unsigned d = sfx + (unsigned)(sizeof(float) * (r * PF + c));
-          cp_async4(d, xt + o, ok ? 4 : 0);
-          cp_async4(d + dy, yt + o, ok ? 4 : 0);
+          const unsigned d = sfx + (unsigned)(sizeof(T) * (r * PF + c));
+          cp_async_elem(d, xt + o, ok);
+          cp_async_elem(d + dy, yt + o, ok);
         }
       }
     }
@@ -703,8 +717,8 @@ __device__ __forceinline__ void seg_products(const double (&v)[kPlSeg + TM], int
 
 // limx: R_t bound of the y-role's column (from x), limy: of the x-role's row (from y), both
 // already capped by the plane's z bound.
-template <int TM, bool LIM>
-__device__ __forceinline__ void plane_walks(const PlaneTile<TM>& sm, int tid, int limx, int limy, double (&acc)[TM]) {
+template <typename T, int TM, bool LIM>
+__device__ __forceinline__ void plane_walks(const PlaneTile<T, TM>& sm, int tid, int limx, int limy, double (&acc)[TM]) {
   double v[kPlSeg + TM];
   {  // y-role
     const int c = tid & (kPlTX - 1), ys = (tid / kPlTX) * kPlSeg;
@@ -722,12 +736,13 @@ __device__ __forceinline__ void plane_walks(const PlaneTile<TM>& sm, int tid, in
 
 // grid: persistent (gridDim.x blocks); block 256; requires ny > 1.
 // VEC: rows 16-byte aligned (nx % 4 == 0, aligned plane segments) and (32 + TM) * nx < 2^31.
-template <int TM, bool VEC>
+template <typename T, int TM, bool VEC>
 __global__ void __launch_bounds__(kPlThreads, TM <= 10 ? 3 : 2)
-ac_plane(Field3 s, double* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket) {
+ac_plane(Field3<T> s, double* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket) {
   extern __shared__ __align__(128) unsigned char plane_smem[];
-  PlaneTile<TM>& sm = *reinterpret_cast<PlaneTile<TM>*>(plane_smem);
-  constexpr int HY = PlaneTile<TM>::HY, NV = PlaneTile<TM>::NV;
+  using PT = PlaneTile<T, TM>;
+  PT& sm = *reinterpret_cast<PT*>(plane_smem);
+  constexpr int HY = PT::HY, NV = PT::NV, EPG = PT::EPG;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const unsigned sfx = (unsigned)__cvta_generic_to_shared(&sm.fx[0][0]);
   const int r0 = tid / NV, g0 = tid % NV;          // this thread's first conversion group
@@ -748,17 +763,15 @@ ac_plane(Field3 s, double* __restrict__ parts, DevResults* __restrict__ res, uns
     const bool xy_inner = x0 + kPlTX + TM <= s.nx && y0 + kPlTY + TM <= s.ny;
     // staged cells outside the field hold eps = 0
     const int rv = (int)(s.ny - y0 < HY ? s.ny - y0 : HY);
-    const int cv = (int)(s.nx - x0 < PlaneTile<TM>::PF ? s.nx - x0 : PlaneTile<TM>::PF);
-    int vb = cv - 4 * lane;
-    vb = vb <= 0 ? 0 : (vb >= 4 ? 16 : 4 * vb);
+    const int cv = (int)(s.nx - x0 < PT::PF ? s.nx - x0 : PT::PF);
     const int64_t torg = y0 * s.nx + x0;
     // per-segment R_t bounds from x (y-role column) and y (x-role row)
     const int64_t mx = s.nx - 1 - (x0 + (tid & (kPlTX - 1))), my = s.ny - 1 - (y0 + (tid & 31));
     const int limx0 = mx < TM ? (int)(mx < -1 ? -1 : mx) : TM, limy0 = my < TM ? (int)(my < -1 ? -1 : my) : TM;
     __syncthreads();                       // previous run's walks are done with the tile
-    PlaneCursor cur;
+    PlaneCursor<T> cur;
     cur.init(s, zb, torg);
-    plane_stage<TM, VEC>(sfx, cur.x, cur.y, s.nx, rv, cv, vb, warp, lane);
+    plane_stage<T, TM, VEC>(sfx, cur.x, cur.y, s.nx, rv, cv, warp, lane);
     for (int64_t z = zb; z < ze; z++) {
       cp_async_wait_all();
       __syncthreads();                     // plane z staged; previous walks done with sm.e
@@ -766,20 +779,14 @@ ac_plane(Field3 s, double* __restrict__ parts, DevResults* __restrict__ res, uns
         // all 16-byte groups of the staged window, 256 at a time (row r, group g of the row)
         int r = r0, g = g0;
         for (int i = tid; i < HY * NV; i += kPlThreads) {
-          const float4 a = *reinterpret_cast<const float4*>(&sm.fx[r][4 * g]);
-          const float4 b = *reinterpret_cast<const float4*>(&sm.fy[r][4 * g]);
-          double e0 = ((double)b.x - (double)a.x) - mu, e1 = ((double)b.y - (double)a.y) - mu;
-          double e2 = ((double)b.z - (double)a.z) - mu, e3 = ((double)b.w - (double)a.w) - mu;
-          if (!xy_inner) {
-            const int c = 4 * g;
-            const bool rin = r < rv;
-            e0 = rin && c < cv ? e0 : 0.0;
-            e1 = rin && c + 1 < cv ? e1 : 0.0;
-            e2 = rin && c + 2 < cv ? e2 : 0.0;
-            e3 = rin && c + 3 < cv ? e3 : 0.0;
+          const Vec16<T> a = *reinterpret_cast<const Vec16<T>*>(&sm.fx[r][EPG * g]);
+          const Vec16<T> b = *reinterpret_cast<const Vec16<T>*>(&sm.fy[r][EPG * g]);
+          double* er = &sm.e[r][EPG * g];
+#pragma unroll
+          for (int j = 0; j < EPG; j++) {
+            const double ej = ((double)b.e[j] - (double)a.e[j]) - mu;
+            er[j] = (xy_inner || (r < rv && EPG * g + j < cv)) ? ej : 0.0;
           }
-          double* er = &sm.e[r][4 * g];
-          er[0] = e0; er[1] = e1; er[2] = e2; er[3] = e3;
           r += kPlThreads / NV;
           g += kPlThreads % NV;
           if (g >= NV) { g -= NV; r++; }
@@ -788,13 +795,13 @@ ac_plane(Field3 s, double* __restrict__ parts, DevResults* __restrict__ res, uns
       __syncthreads();                     // eps ready, staging buffer free
       if (z + 1 < ze) {
         cur.advance(s, torg);
-        plane_stage<TM, VEC>(sfx, cur.x, cur.y, s.nx, rv, cv, vb, warp, lane);
+        plane_stage<T, TM, VEC>(sfx, cur.x, cur.y, s.nx, rv, cv, warp, lane);
       }
       // R_t bound from the z axis (active only for 3-D fields)
       const int64_t mz64 = s.nz > 1 ? s.nz - 1 - z : TM;
       const int mz = mz64 > TM ? TM : (int)mz64;
-      if (xy_inner && mz >= TM) plane_walks<TM, false>(sm, tid, TM, TM, acc);
-      else plane_walks<TM, true>(sm, tid, limx0 < mz ? limx0 : mz, limy0 < mz ? limy0 : mz, acc);
+      if (xy_inner && mz >= TM) plane_walks<T, TM, false>(sm, tid, TM, TM, acc);
+      else plane_walks<T, TM, true>(sm, tid, limx0 < mz ? limx0 : mz, limy0 < mz ? limy0 : mz, acc);
     }
   }
   ac_finish<TM>(acc, parts, res->rec.ac[1], ticket);
@@ -808,16 +815,18 @@ static int sm_count() {
   return n > 0 ? n : 1;
 }
 
-static int64_t deriv_zplanes(const Field3& s) {
+template <typename T>
+static int64_t deriv_zplanes(const Field3<T>& s) {
   int64_t zlo = s.nz > 1 ? 1 : 0, zhi = s.nz > 1 ? s.nz - 1 : 1;
   if (zlo < s.zown0) zlo = s.zown0;
   if (zhi > s.zown1) zhi = s.zown1;
   return zhi > zlo ? zhi - zlo : 1;
 }
 // 2-D fields (one plane, never slab-sharded) are streamed along their rows: view (ny, 1, nx).
-static Field3 deriv_view(const Field3& s) {
+template <typename T>
+static Field3<T> deriv_view(const Field3<T>& s) {
   if (!(s.nz == 1 && s.ny > 1)) return s;
-  Field3 v = s;
+  Field3<T> v = s;
   v.nz = s.ny; v.ny = 1;
   v.zown0 = 0; v.zown1 = s.ny;
   v.zs[0] = 0; v.zs[1] = s.ny;
@@ -825,7 +834,8 @@ static Field3 deriv_view(const Field3& s) {
 }
 // Launch shape: (BX, BY) tiles x chunks of the streamed axis; the chunk length is the requested
 // one unless that leaves fewer than ~8 blocks per SM (short or 2-D fields), never below 8 planes.
-static dim3 deriv_grid(const Field3& s, int zchunk, int* zc) {
+template <typename T>
+static dim3 deriv_grid(const Field3<T>& s, int zchunk, int* zc) {
   const int bx = s.ny > 1 ? kTX : 256, by = s.ny > 1 ? kTY : 1;
   const int64_t tiles = cdiv(s.nx, bx) * cdiv(s.ny, by), planes = deriv_zplanes(s);
   int64_t c = zchunk;
@@ -835,21 +845,23 @@ static dim3 deriv_grid(const Field3& s, int zchunk, int* zc) {
   *zc = (int)c;
   return dim3((unsigned)cdiv(s.nx, bx), (unsigned)cdiv(s.ny, by), (unsigned)cdiv(planes, c));
 }
-int64_t deriv_blocks(const Field3& s0, int zchunk) {
+template <typename T>
+int64_t deriv_blocks(const Field3<T>& s0, int zchunk) {
   int zc;
   const dim3 g = deriv_grid(deriv_view(s0), zchunk, &zc);
   return (int64_t)g.x * g.y * g.z;
 }
 
-cudaError_t launch_deriv(const Field3& s0, int zchunk, double* parts, DevResults* res,
+template <typename T>
+cudaError_t launch_deriv(const Field3<T>& s0, int zchunk, double* parts, DevResults* res,
                          unsigned int* ticket, cudaStream_t st) {
-  const Field3 s = deriv_view(s0);
+  const Field3<T> s = deriv_view(s0);
   int zc;
   const dim3 grid = deriv_grid(s, zchunk, &zc);
-  if (s.ny > 1 && s.nz > 2) deriv3_kernel<2><<<grid, dim3(kTX, kTY / 2), 0, st>>>(s, zc, parts, res, ticket);
-  else if (s.ny > 1) deriv_kernel<true, true, kTX, kTY><<<grid, dim3(kTX, kTY), 0, st>>>(s, zc, parts, res, ticket);
-  else if (s.nz > 1) deriv_kernel<true, false, 256, 1><<<grid, dim3(256, 1), 0, st>>>(s, zc, parts, res, ticket);
-  else deriv_kernel<false, false, 256, 1><<<grid, dim3(256, 1), 0, st>>>(s, zc, parts, res, ticket);
+  if (s.ny > 1 && s.nz > 2) deriv3_kernel<T, 2><<<grid, dim3(kTX, kTY / 2), 0, st>>>(s, zc, parts, res, ticket);
+  else if (s.ny > 1) deriv_kernel<T, true, true, kTX, kTY><<<grid, dim3(kTX, kTY), 0, st>>>(s, zc, parts, res, ticket);
+  else if (s.nz > 1) deriv_kernel<T, true, false, 256, 1><<<grid, dim3(256, 1), 0, st>>>(s, zc, parts, res, ticket);
+  else deriv_kernel<T, false, false, 256, 1><<<grid, dim3(256, 1), 0, st>>>(s, zc, parts, res, ticket);
   return cudaGetLastError();
 }
 
@@ -861,7 +873,8 @@ struct AcGrids {
   bool rz, ry, rx;
   int zc, pzc, xc;
 };
-static AcGrids ac_grids(const Field3& s, int T) {
+template <typename E>
+static AcGrids ac_grids(const Field3<E>& s, int T) {
   AcGrids g{};
   const int64_t nzo = s.zown1 - s.zown0;
   g.zc = 50; g.xc = 128;    // xc % 4 == 0 for the vector x-walk
@@ -877,20 +890,22 @@ static AcGrids ac_grids(const Field3& s, int T) {
   g.xvec = dim3((unsigned)cdiv(nzo * s.ny, 256), (unsigned)cdiv(s.nx, g.xc), 1);
   return g;
 }
-int64_t ac_blocks(const Field3& s, int T) {
+template <typename E>
+int64_t ac_blocks(const Field3<E>& s, int T) {
   const AcGrids g = ac_grids(s, T);
   auto n = [](dim3 d) { return (int64_t)d.x * d.y * d.z; };
   auto mx = [](int64_t a, int64_t b) { return a > b ? a : b; };
   return mx(n(g.z), n(g.zt)) + n(g.pl) + mx(n(g.x), n(g.xvec));
 }
 
-template <int TM>
-static cudaError_t launch_ac_t(const Field3& s, int T, double* parts, DevResults* res,
+template <typename E, int TM>
+static cudaError_t launch_ac_t(const Field3<E>& s, int T, double* parts, DevResults* res,
                                unsigned int* tickets, cudaStream_t st) {
   const AcGrids g = ac_grids(s, T);
   auto n = [](dim3 d) { return (size_t)d.x * d.y * d.z; };
-  // rows 16-byte aligned (nx % 4 == 0, aligned segments): TMA bulk-copy z-walk and vector x-walk
-  bool vec = (s.nx % 4) == 0;
+  // rows 16-byte aligned (nx * sizeof(E) % 16 == 0, aligned segments): TMA bulk-copy z-walk and
+  // 16-byte plane staging; the vector x-walk (1-D fields) is float32 only
+  bool vec = (s.nx * (int64_t)sizeof(E)) % 16 == 0;
   for (int k = 0; k < s.nseg; k++)
     vec = vec && (reinterpret_cast<uintptr_t>(s.xs[k]) % 16) == 0 && (reinterpret_cast<uintptr_t>(s.ys[k]) % 16) == 0;
   double* pz = parts;
@@ -899,37 +914,55 @@ static cudaError_t launch_ac_t(const Field3& s, int T, double* parts, DevResults
   cudaError_t e = cudaMemsetAsync(res->rec.ac, 0, sizeof(res->rec.ac), st);
   if (e != cudaSuccess) return e;
   if (g.rz && vec) {
-    constexpr int wsm = (int)sizeof(BulkWalkSmem<TM>);
-    if ((e = set_smem_once<ac_zwalk_tma<TM>>(wsm)) != cudaSuccess) return e;
-    ac_zwalk_tma<TM><<<g.zt, kWalkThreads, wsm, st>>>(s, T, g.zc, pz, res, tickets + 0);
+    constexpr int wsm = (int)sizeof(BulkWalkSmem<E, TM>);
+    if ((e = set_smem_once<ac_zwalk_tma<E, TM>>(wsm)) != cudaSuccess) return e;
+    ac_zwalk_tma<E, TM><<<g.zt, kWalkThreads, wsm, st>>>(s, T, g.zc, pz, res, tickets + 0);
   } else if (g.rz) {
-    ac_zwalk<TM><<<g.z, dim3(kTX, kTY), 0, st>>>(s, T, g.zc, pz, res, tickets + 0);
+    ac_zwalk<E, TM><<<g.z, dim3(kTX, kTY), 0, st>>>(s, T, g.zc, pz, res, tickets + 0);
   }
   if (g.ry) {
-    constexpr int psm = (int)sizeof(PlaneTile<TM>);
+    constexpr int psm = (int)sizeof(PlaneTile<E, TM>);
     // 16-byte staging needs aligned rows; tile-relative offsets are 32-bit
     const bool pvec = vec && (int64_t)(kPlTY + TM) * s.nx < ((int64_t)1 << 31);
-    auto kern = pvec ? ac_plane<TM, true> : ac_plane<TM, false>;
-    if ((e = pvec ? set_smem_once<ac_plane<TM, true>>(psm) : set_smem_once<ac_plane<TM, false>>(psm)) != cudaSuccess) return e;
+    auto kern = pvec ? ac_plane<E, TM, true> : ac_plane<E, TM, false>;
+    if ((e = pvec ? set_smem_once<ac_plane<E, TM, true>>(psm) : set_smem_once<ac_plane<E, TM, false>>(psm)) != cudaSuccess)
+      return e;
     kern<<<g.pl, kPlThreads, psm, st>>>(s, pp, res, tickets + 1);
-  } else if (g.rx && vec) {
-    ac_xwalk_vec<TM><<<g.xvec, 256, 0, st>>>(s, T, g.xc, px, res, tickets + 2);
   } else if (g.rx) {
-    ac_xwalk_smem<TM><<<g.x, kXWarps * 32, 0, st>>>(s, T, g.xc, px, res, tickets + 2);
+    bool done = false;
+    if constexpr (sizeof(E) == 4) {
+      if (vec) {
+        ac_xwalk_vec<TM><<<g.xvec, 256, 0, st>>>(s, T, g.xc, px, res, tickets + 2);
+        done = true;
+      }
+    }
+    if (!done) ac_xwalk_smem<E, TM><<<g.x, kXWarps * 32, 0, st>>>(s, T, g.xc, px, res, tickets + 2);
   }
   return cudaGetLastError();
 }
 
 // tickets: three consecutive counters (z, y, x walks)
-cudaError_t launch_ac(const Field3& s, int T, int, double* parts, DevResults* res,
+template <typename E>
+cudaError_t launch_ac(const Field3<E>& s, int T, int, double* parts, DevResults* res,
                       unsigned int* tickets, cudaStream_t st) {
-  if (T <= 2) return launch_ac_t<2>(s, T, parts, res, tickets, st);
-  if (T <= 4) return launch_ac_t<4>(s, T, parts, res, tickets, st);
-  if (T <= 6) return launch_ac_t<6>(s, T, parts, res, tickets, st);
-  if (T <= 8) return launch_ac_t<8>(s, T, parts, res, tickets, st);
-  if (T <= 10) return launch_ac_t<10>(s, T, parts, res, tickets, st);
-  if (T <= 12) return launch_ac_t<12>(s, T, parts, res, tickets, st);
-  return launch_ac_t<16>(s, T, parts, res, tickets, st);
+  if (T <= 2) return launch_ac_t<E, 2>(s, T, parts, res, tickets, st);
+  if (T <= 4) return launch_ac_t<E, 4>(s, T, parts, res, tickets, st);
+  if (T <= 6) return launch_ac_t<E, 6>(s, T, parts, res, tickets, st);
+  if (T <= 8) return launch_ac_t<E, 8>(s, T, parts, res, tickets, st);
+  if (T <= 10) return launch_ac_t<E, 10>(s, T, parts, res, tickets, st);
+  if (T <= 12) return launch_ac_t<E, 12>(s, T, parts, res, tickets, st);
+  return launch_ac_t<E, 16>(s, T, parts, res, tickets, st);
 }
+
+#define CZC_P2_INST(E)                                                                              \
+  template int64_t deriv_blocks<E>(const Field3<E>&, int);                                          \
+  template int64_t ac_blocks<E>(const Field3<E>&, int);                                             \
+  template cudaError_t launch_deriv<E>(const Field3<E>&, int, double*, DevResults*, unsigned int*,  \
+                                       cudaStream_t);                                               \
+  template cudaError_t launch_ac<E>(const Field3<E>&, int, int, double*, DevResults*, unsigned int*, \
+                                    cudaStream_t);
+CZC_P2_INST(float)
+CZC_P2_INST(double)
+#undef CZC_P2_INST
 
 }  // namespace czc

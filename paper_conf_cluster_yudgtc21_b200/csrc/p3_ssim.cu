@@ -32,15 +32,15 @@ namespace czc {
 constexpr int kP3Warps = 8;
 constexpr int kP3Threads = 32 * kP3Warps;
 
-template <int WX, int WY, int WZ, int G>
+template <typename T, int WX, int WY, int WZ, int G>
 struct SsimGeom {
   static constexpr int TX = 32 - WX + 1;                 // origins per tile along x
   static constexpr int TY = kP3Warps * G;                // origins per tile along y
   static constexpr int FY = TY + WY - 1;                 // footprint rows
   static constexpr int KC = (FY + kP3Warps - 1) / kP3Warps;   // z-walk rows per thread
   static constexpr int ZSTRIDE = FY * 32;                // one component plane of the exchange
-  // exchange buffer: { 4 double comps, 2 float comps } x FY x 32, double-buffered
-  static constexpr size_t buf_bytes = (size_t)ZSTRIDE * (4 * sizeof(double) + 2 * sizeof(float));
+  // exchange buffer: { 4 double comps, 2 min/max comps of the input type } x FY x 32, double-buffered
+  static constexpr size_t buf_bytes = (size_t)ZSTRIDE * (4 * sizeof(double) + 2 * sizeof(T));
   static constexpr size_t smem = 2 * buf_bytes;
 };
 
@@ -70,29 +70,31 @@ __device__ __forceinline__ double lane_window_sum(double v) {
 
 // min / max over lanes [l, l+W): doubling to the largest power of two <= W, then one
 // overlapping combine (max and min are idempotent).
-template <int W, bool IS_MAX>
-__device__ __forceinline__ float lane_window_ext(float v) {
-  float q = v;
+template <int W, bool IS_MAX, typename T>
+__device__ __forceinline__ T lane_window_ext(T v) {
+  T q = v;
   int k = 0;
 #pragma unroll
   for (int j = 1; j < 5; j++)
     if ((1 << j) <= W) {
-      const float o = shf(q, 1 << (j - 1));
-      q = IS_MAX ? fmaxf(q, o) : fminf(q, o);
+      const T o = __shfl_down_sync(0xffffffffu, q, 1 << (j - 1));
+      q = IS_MAX ? tmax(q, o) : tmin(q, o);
       k = j;
     }
   if ((1 << k) != W) {
-    const float o = shf(q, W - (1 << k));
-    q = IS_MAX ? fmaxf(q, o) : fminf(q, o);
+    const T o = __shfl_down_sync(0xffffffffu, q, W - (1 << k));
+    q = IS_MAX ? tmax(q, o) : tmin(q, o);
   }
   return q;
 }
 
-template <int WX, int WY, int WZ, int G>
-__global__ void __launch_bounds__(kP3Threads, (SsimGeom<WX, WY, WZ, G>::KC * WZ <= 24) ? 2 : 1)
-p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __restrict__ res,
+// T = float: the x ring and the exchanged extrema are floats (exact); T = double: doubles, one
+// block per SM for the larger register ring.
+template <typename T, int WX, int WY, int WZ, int G>
+__global__ void __launch_bounds__(kP3Threads, (SsimGeom<T, WX, WY, WZ, G>::KC * WZ * sizeof(T) <= 96) ? 2 : 1)
+p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __restrict__ res,
           unsigned int* __restrict__ ticket, double* __restrict__ dbg) {
-  using Gm = SsimGeom<WX, WY, WZ, G>;
+  using Gm = SsimGeom<T, WX, WY, WZ, G>;
   constexpr int TX = Gm::TX, FY = Gm::FY, KC = Gm::KC, ZS = Gm::ZSTRIDE;
   constexpr double invM = 1.0 / (double)(WX * WY * WZ);
   extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -127,16 +129,17 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
   // (zb + n - WZ), which is re-read from L2 instead of being kept in the register ring.  Both
   // streams advance through plane cursors (pointer increments, no per-plane address math).
   const int nsteps = (int)(zend - zb);
-  SegCursor cin, cold;
+  SegCursor<T> cin, cold;
   if (nsteps > 0) { cin.init(f, zb); cold.init(f, zb); }
-  auto load = [&](int n, float2 (&dst)[KC], float (&yold)[KC]) {
+  auto load = [&](int n, Pair<T> (&dst)[KC], T (&yold)[KC]) {
     if (n < nsteps) {
       const bool has_old = n >= WZ;
 #pragma unroll
       for (int k = 0; k < KC; k++) {
         const bool v = (vbits >> k) & 1u;
-        dst[k] = v ? make_float2(__ldg(cin.x + off[k]), __ldg(cin.y + off[k])) : make_float2(0.f, 0.f);
-        yold[k] = (v && has_old) ? __ldg(cold.y + off[k]) : 0.f;
+        dst[k].x = v ? __ldg(cin.x + off[k]) : (T)0;
+        dst[k].y = v ? __ldg(cin.y + off[k]) : (T)0;
+        yold[k] = (v && has_old) ? __ldg(cold.y + off[k]) : (T)0;
       }
       cin.advance(f, zb + n + 1);
       if (has_old) cold.advance(f, zb + n + 1 - WZ);
@@ -144,16 +147,16 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
   };
 
   double sm[KC][4];
-  float ring[KC][WZ];                                    // x of the last WZ planes
+  T ring[KC][WZ];                                        // x of the last WZ planes
 #pragma unroll
   for (int k = 0; k < KC; k++) {
 #pragma unroll
     for (int m = 0; m < 4; m++) sm[k][m] = 0;
 #pragma unroll
-    for (int s = 0; s < WZ; s++) ring[k][s] = 0.f;
+    for (int s = 0; s < WZ; s++) ring[k][s] = 0;
   }
-  float2 nxt[KC];                                        // prefetched next plane
-  float nyo[KC];                                         // ... and its leaving y sample
+  Pair<T> nxt[KC];                                       // prefetched next plane
+  T nyo[KC];                                             // ... and its leaving y sample
   load(0, nxt, nyo);
 
   double ssum = 0, scnt = 0;
@@ -175,11 +178,11 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
       if (step >= nsteps) break;                         // block-uniform
       // the prefetched plane is consumed by the z-walk below, then the next one is requested
       // into the same registers (no copies; its latency hides behind the y / x passes)
-      const float2 (&v)[KC] = nxt;
-      const float (&yo)[KC] = nyo;
+      const Pair<T> (&v)[KC] = nxt;
+      const T (&yo)[KC] = nyo;
       const int buf = step & 1;
       double* Zd = reinterpret_cast<double*>(smem_raw + buf * Gm::buf_bytes);
-      float* Zm = reinterpret_cast<float*>(Zd + 4 * ZS);
+      T* Zm = reinterpret_cast<T*>(Zd + 4 * ZS);
       // ---- (a) z-walk --------------------------------------------------------------------
 #pragma unroll
       for (int k = 0; k < KC; k++) {
@@ -196,9 +199,9 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
         ring[k][s] = v[k].x;
         const int r = warp + kP3Warps * k;
         if (step >= WZ - 1 && r < FY) {
-          float mn = ring[k][0], mx = ring[k][0];
+          T mn = ring[k][0], mx = ring[k][0];
 #pragma unroll
-          for (int t = 1; t < WZ; t++) { mn = fminf(mn, ring[k][t]); mx = fmaxf(mx, ring[k][t]); }
+          for (int t = 1; t < WZ; t++) { mn = tmin(mn, ring[k][t]); mx = tmax(mx, ring[k][t]); }
           const int c = r * 32 + lane;
 #pragma unroll
           for (int m = 0; m < 4; m++) Zd[m * ZS + c] = sm[k][m];
@@ -214,14 +217,14 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
       // ---- (b) y-pass over WY rows, (c) x-pass with shuffles, mix ------------------------
       // ---- (b) y-pass: the G origin rows of this warp (running sums over WY rows) ------------
       double h[G][4];
-      float hmn[G], hmx[G];
+      T hmn[G], hmx[G];
       {
         // y-window min/max: the WY - G + 1 rows shared by all G windows are reduced once
-        float cmn = Zm[(warp * G + G - 1) * 32 + lane], cmx = Zm[ZS + (warp * G + G - 1) * 32 + lane];
+        T cmn = Zm[(warp * G + G - 1) * 32 + lane], cmx = Zm[ZS + (warp * G + G - 1) * 32 + lane];
 #pragma unroll
         for (int i = G; i < WY; i++) {
-          cmn = fminf(cmn, Zm[(warp * G + i) * 32 + lane]);
-          cmx = fmaxf(cmx, Zm[ZS + (warp * G + i) * 32 + lane]);
+          cmn = tmin(cmn, Zm[(warp * G + i) * 32 + lane]);
+          cmx = tmax(cmx, Zm[ZS + (warp * G + i) * 32 + lane]);
         }
 #pragma unroll
         for (int g = 0; g < G; g++) {
@@ -237,16 +240,16 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
               h[g][m] = h[g - 1][m] + (Zd[m * ZS + (oy + WY - 1) * 32 + lane] - Zd[m * ZS + (oy - 1) * 32 + lane]);
             }
           }
-          float mn = cmn, mx = cmx;                      // rows [G-1, WY) relative to warp*G
+          T mn = cmn, mx = cmx;                          // rows [G-1, WY) relative to warp*G
 #pragma unroll
           for (int i = g; i < G - 1; i++) {              // rows oy .. warp*G + G - 2
-            mn = fminf(mn, Zm[(warp * G + i) * 32 + lane]);
-            mx = fmaxf(mx, Zm[ZS + (warp * G + i) * 32 + lane]);
+            mn = tmin(mn, Zm[(warp * G + i) * 32 + lane]);
+            mx = tmax(mx, Zm[ZS + (warp * G + i) * 32 + lane]);
           }
 #pragma unroll
           for (int i = WY; i < WY + g; i++) {            // rows warp*G + WY .. oy + WY - 1
-            mn = fminf(mn, Zm[(warp * G + i) * 32 + lane]);
-            mx = fmaxf(mx, Zm[ZS + (warp * G + i) * 32 + lane]);
+            mn = tmin(mn, Zm[(warp * G + i) * 32 + lane]);
+            mx = tmax(mx, Zm[ZS + (warp * G + i) * 32 + lane]);
           }
           hmn[g] = mn;
           hmx[g] = mx;
@@ -254,7 +257,7 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
       }
       // ---- (c) x-pass for all G rows together (independent shuffle chains -> ILP), then mix --
       double S[G][4];
-      float wmn[G], wmx[G];
+      T wmn[G], wmx[G];
 #pragma unroll
       for (int g = 0; g < G; g++) {
 #pragma unroll
@@ -298,45 +301,50 @@ p3_kernel(Field3 f, SsimParams p, double* __restrict__ parts, DevResults* __rest
 
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
-template <int WX, int WY, int WZ, int G>
-static cudaError_t launch_t(const Field3& f, const SsimParams& p, double* parts,
+template <typename T, int WX, int WY, int WZ, int G>
+static cudaError_t launch_t(const Field3<T>& f, const SsimParams& p, double* parts,
                             DevResults* res, unsigned int* ticket, double* dbg, cudaStream_t st,
                             int64_t* nblocks_out) {
-  using Gm = SsimGeom<WX, WY, WZ, G>;
+  using Gm = SsimGeom<T, WX, WY, WZ, G>;
   int64_t zhi = f.zown1 < f.nz - WZ + 1 ? f.zown1 : f.nz - WZ + 1;
   const int64_t noz = zhi > f.zown0 ? zhi - f.zown0 : 1;
   dim3 grid((unsigned)cdiv(f.nx - WX + 1, Gm::TX), (unsigned)cdiv(f.ny - WY + 1, Gm::TY),
             (unsigned)cdiv(noz, p.zchunk));
   if (nblocks_out) { *nblocks_out = (int64_t)grid.x * grid.y * grid.z; return cudaSuccess; }
   if (f.ny * f.nx >= (int64_t)1 << 31) return cudaErrorInvalidValue;   // 32-bit in-plane offsets
-  cudaError_t e = set_smem_once<p3_kernel<WX, WY, WZ, G>>((int)Gm::smem);
+  cudaError_t e = set_smem_once<p3_kernel<T, WX, WY, WZ, G>>((int)Gm::smem);
   if (e != cudaSuccess) return e;
-  p3_kernel<WX, WY, WZ, G><<<grid, kP3Threads, Gm::smem, st>>>(f, p, parts, res, ticket, dbg);
+  p3_kernel<T, WX, WY, WZ, G><<<grid, kP3Threads, Gm::smem, st>>>(f, p, parts, res, ticket, dbg);
   return cudaGetLastError();
 }
 
 // kind 3: cubic window (3-D); 2: square window, z inactive (2-D); 1: x only (1-D).
-template <int W>
-static cudaError_t dispatch_w(int kind, const Field3& f, const SsimParams& p, double* parts,
+template <typename T, int W>
+static cudaError_t dispatch_w(int kind, const Field3<T>& f, const SsimParams& p, double* parts,
                               DevResults* res, unsigned int* ticket, double* dbg, cudaStream_t st, int64_t* nb) {
   constexpr int G = W <= 8 ? 2 : 1;                     // keep the z-walk state in registers
-  if (kind == 3) return launch_t<W, W, W, G>(f, p, parts, res, ticket, dbg, st, nb);
-  if (kind == 2) return launch_t<W, W, 1, 2>(f, p, parts, res, ticket, dbg, st, nb);
-  return launch_t<W, 1, 1, 1>(f, p, parts, res, ticket, dbg, st, nb);
+  if (kind == 3) return launch_t<T, W, W, W, G>(f, p, parts, res, ticket, dbg, st, nb);
+  if (kind == 2) return launch_t<T, W, W, 1, 2>(f, p, parts, res, ticket, dbg, st, nb);
+  return launch_t<T, W, 1, 1, 1>(f, p, parts, res, ticket, dbg, st, nb);
 }
 
 // Returns cudaErrorInvalidValue for unsupported W.  If nblocks_out != NULL only the grid size
 // is computed (no launch).
-cudaError_t launch_ssim(int kind, int W, const Field3& f, const SsimParams& p,
+template <typename T>
+cudaError_t launch_ssim(int kind, int W, const Field3<T>& f, const SsimParams& p,
                         double* parts, DevResults* res, unsigned int* ticket, double* dbg,
                         cudaStream_t st, int64_t* nblocks_out) {
   switch (W) {
-#define CZC_W(w) case w: return dispatch_w<w>(kind, f, p, parts, res, ticket, dbg, st, nblocks_out);
+#define CZC_W(w) case w: return dispatch_w<T, w>(kind, f, p, parts, res, ticket, dbg, st, nblocks_out);
     CZC_W(2) CZC_W(3) CZC_W(4) CZC_W(5) CZC_W(6) CZC_W(7) CZC_W(8) CZC_W(9) CZC_W(10)
     CZC_W(11) CZC_W(12) CZC_W(13) CZC_W(14) CZC_W(15) CZC_W(16)
 #undef CZC_W
     default: return cudaErrorInvalidValue;
   }
 }
+template cudaError_t launch_ssim<float>(int, int, const Field3<float>&, const SsimParams&, double*, DevResults*,
+                                        unsigned int*, double*, cudaStream_t, int64_t*);
+template cudaError_t launch_ssim<double>(int, int, const Field3<double>&, const SsimParams&, double*, DevResults*,
+                                         unsigned int*, double*, cudaStream_t, int64_t*);
 
 }  // namespace czc

@@ -26,7 +26,7 @@ def _czc():
 
 
 # Record layout (mirrors czc_internal.cuh `Record`): P1State {n, mx, my, me, m2x, m2y, cxy, m2e, sae,
-# emin, emax, pmin, pmax, spwr, npwr : double; xmin, xmax : float}, deriv[25], ac[3][16], ssim[3],
+# emin, emax, pmin, pmax, spwr, npwr, xmin, xmax : double}, deriv[25], ac[3][16], ssim[3],
 # pdf[2][256] (uint64 counts of the error / pwr-error PDFs, binned over the GLOBAL ranges).
 PDF_MAX = 256
 
@@ -57,7 +57,7 @@ def p1_state(x, y):
             ((yd - yd.mean()) ** 2).sum(), ((xd - xd.mean()) * (yd - yd.mean())).sum(),
             ((e - e.mean()) ** 2).sum(), np.abs(e).sum(), e.min(), e.max(),
             q.min() if q.size else math.inf, q.max() if q.size else -math.inf, q.sum(), float(q.size)]
-    return struct.pack("<15d2f", *vals, float(x.min()), float(x.max()))
+    return struct.pack("<17d", *vals, float(x.min()), float(x.max()))
 
 
 def deriv_fields(f):

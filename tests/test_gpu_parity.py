@@ -314,7 +314,7 @@ def test_status_codes(czc):
     with czc.Assessor() as a:
         r = czc.Result()
         shape = czc.make_shape([6, 7, 8])
-        assert lib.czc_assess(a.ctx, x.data_ptr(), x.data_ptr(), ctypes.byref(shape), 1, czc.M_P1, ctypes.byref(r)) == 3
+        assert lib.czc_assess(a.ctx, x.data_ptr(), x.data_ptr(), ctypes.byref(shape), 2, czc.M_P1, ctypes.byref(r)) == 3
         bad = czc.make_shape([6, 0, 8])
         assert lib.czc_assess(a.ctx, x.data_ptr(), x.data_ptr(), ctypes.byref(bad), 0, czc.M_P1, ctypes.byref(r)) == 2
         slab = czc.make_shape([6, 7, 8], z0=2, nz_local=3)            # slab shape without ranks
@@ -506,6 +506,20 @@ def test_full_size_nyx(czc, orc):
     assert _sampled_ssim(orc, xn, yn, d, [8, 8, 8], 300, 31) < 1e-6
 
 
+def test_ordered_after_default_stream_work(czc):
+    """A context made on torch's default stream (handle 0 -> the library's own stream) must see
+    the fields that default-stream kernels are still writing: the library stream is blocking, so
+    it waits for them (regression: a non-blocking stream read half-written inputs and raced the
+    ticket reset)."""
+    n = 640
+    for _ in range(2):
+        x = torch.full((n, n, n), 3.0, dtype=torch.float32, device="cuda")
+        y = torch.full((n, n, n), 3.5, dtype=torch.float32, device="cuda")
+        with czc.Assessor() as a:
+            g = a.assess(x, y, czc.M_P1)
+        assert g["n"] == n ** 3 and g["x_min"] == 3.0 and g["err_min"] == 0.5 and g["mse"] == 0.25
+
+
 def test_maximum_size_closed_forms(czc):
     """BASELINE configs[4] size on ONE GPU: a 2048^3 pair (68.7 GB, 8.6e9 elements) with
     x = v constant and y = v + c (c = 2^-10 exact): every metric has a closed form — e = c,
@@ -539,3 +553,83 @@ def test_maximum_size_closed_forms(czc):
     assert g["n_windows"] == (n - 7) ** 3
     assert abs(g["ssim"] - A / (A + c * c)) < 1e-12
     assert g["err_pdf"][0] == N and g["err_pdf_width"] == 0.0 and g["pwr_pdf"][0] == N
+
+
+# ---------------------------------------------------------------- float64 inputs (NEXT row f3)
+def f64_pair(cfg, dims, seed=7):
+    """A float64 pair with full 53-bit mantissas: the float32 recipe of `cfg`, the original
+    perturbed by 1e-9 relative and the reconstruction error by 1e-6 relative (values no float32
+    can hold, so every kernel really reads doubles)."""
+    x, y = synth.make_pair(synth.config(cfg, dims=dims))
+    r = np.random.default_rng(seed)
+    xd = x.numpy().astype(np.float64)
+    e = y.numpy().astype(np.float64) - xd
+    xd = xd * (1.0 + 1e-9 * r.standard_normal(xd.shape))
+    yd = xd + e * (1.0 + 1e-6 * r.standard_normal(xd.shape))
+    assert np.any(xd.astype(np.float32).astype(np.float64) != xd)
+    return xd, yd
+
+
+@pytest.mark.parametrize("cfg,dims,w", [("C1", (64, 64, 64), 7), ("C2", (40, 70, 90), 8),
+                                        ("C2q", (21, 66, 75), 8), ("C3", (33, 45, 61), 6),
+                                        ("C4", (180, 360), 8), ("C4", (3, 2001), 5)])
+def test_f64_parity_configs(czc, orc, cfg, dims, w):
+    xd, yd = f64_pair(cfg, dims)
+    if dims[0] == 3:
+        xd, yd = xd[1].copy(), yd[1].copy()                      # 1-D
+    g, o = run_both(czc, orc, xd, yd, window=w)
+    assert g["computed_mask"] == czc.M_ALL
+    full_check(g, o)
+
+
+def test_f64_float_representable_matches_f32_path(czc, orc):
+    """Float data widened to double: the float64 kernels must give the float32 kernels' exact
+    fields bit for bit and agree with them (and the oracle) within the tolerances elsewhere."""
+    x, y = synth.make_pair(synth.config("C2", dims=(30, 50, 70)))
+    with czc.Assessor(ssim_window=8) as a:
+        g32 = a.assess(x.cuda(), y.cuda(), czc.M_FULL)
+        g64 = a.assess(x.double().cuda(), y.double().cuda(), czc.M_FULL)
+    for k in ("x_min", "x_max", "err_min", "err_max", "err_maxabs", "pwr_min", "pwr_max", "n_pwr",
+              "n_windows", "n_interior", "der1_maxabs", "lap_f_min", "grad_f_max"):
+        assert g32[k] == g64[k], k
+    assert np.array_equal(g32["err_pdf"], g64["err_pdf"]) and np.array_equal(g32["pwr_pdf"], g64["pwr_pdf"])
+    for k in ("mse", "psnr", "pearson", "ssim", "der2_mae", "div_mse"):
+        assert abs(g32[k] - g64[k]) <= 1e-12 * max(1.0, abs(g32[k])), k
+
+
+def test_f64_slab_host_pdf_and_misaligned(czc, orc):
+    """float64 through the loopback slab path, the pipelined host path, the PDF pass, and views
+    that are 8- but not 16-byte aligned (scalar prologue of the vector path)."""
+    xd, yd = f64_pair("C2", (36, 48, 58))
+    o = {}
+    o.update(orc.p1(xd, yd))
+    o.update(orc.deriv(xd, yd))
+    o["ac"], o["ac_count"] = orc.autocorr(xd, yd, 10)
+    o["ssim"], o["n_windows"] = orc.ssim(xd, yd, [8] * 3)
+    tx, ty = torch.from_numpy(xd), torch.from_numpy(yd)
+    with czc.Assessor(ssim_window=8, loopback_slabs=3) as a:
+        full_check(a.assess(tx.cuda(), ty.cuda()), o)
+    with czc.Assessor(ssim_window=8) as a:
+        full_check(a.assess_host(tx.pin_memory().numpy(), ty.pin_memory().numpy()), o)
+    with czc.Assessor(ndim=1, pdf_bins=64) as a:
+        g = a.assess(tx.cuda().reshape(-1), ty.cuda().reshape(-1), czc.M_PDF | czc.M_P1)
+        pdf_check(g, orc.pdf(xd.ravel(), yd.ravel(), 64), 64)
+        xf, yf = tx.cuda().reshape(-1), ty.cuda().reshape(-1)
+        for ox, oy in ((1, 1), (1, 2)):
+            n = xf.numel() - 2
+            g = a.assess(xf[ox:ox + n], yf[oy:oy + n], czc.M_P1 | czc.M_PDF)
+            errors = []
+            check_p1(g, orc.p1(xd.ravel()[ox:ox + n], yd.ravel()[oy:oy + n]), errors)
+            report(errors)
+            pdf_check(g, orc.pdf(xd.ravel()[ox:ox + n], yd.ravel()[oy:oy + n], 64), 64)
+
+
+def test_f64_dtype_errors(czc):
+    x = torch.zeros(4, 5, 6, device="cuda", dtype=torch.float64)
+    with czc.Assessor() as a:
+        with pytest.raises(TypeError):
+            a.assess(x, x.float())
+        import ctypes
+        r = czc.Result()
+        assert czc.lib.czc_assess(a.ctx, x.data_ptr(), x.data_ptr(), ctypes.byref(czc.make_shape([4, 5, 6])),
+                                  2, czc.M_P1, ctypes.byref(r)) == 3
