@@ -195,9 +195,12 @@ def run_ours(args, rank, world, local):
         dist.broadcast_object_list(obj, src=0)
         uid = obj[0]
     stream = torch.cuda.current_stream(dev)
-    cfg = dict(ssim_window=8, ssim_step=1, ac_max_lag=10, timing=True)
+    cfg = dict(ssim_window=8, ssim_step=1, ac_max_lag=10)
     if world > 1:
         cfg.update(rank=rank, nranks=world, nccl_uid=uid)
+    # the timed steps run as users run them (single GPU: the launch sequence replays as one CUDA
+    # graph); per-kernel times come from a second context with per-kernel events (timing=True,
+    # direct launches) over as many untimed-for-value steps afterwards
     a = czc.Assessor(ndim=3, device=local, stream=stream, **cfg)
     kw = dict(dims=gdims, z0=z0) if world > 1 else {}
 
@@ -223,12 +226,18 @@ def run_ours(args, rank, world, local):
                                                         # the dirty lines are written back before the
                                                         # step starts and L2 holds only clean lines
         ev[i][0].record(stream)
-        r = a.assess(xd, yd, czc.M_ALL, **kw)
+        a.assess(xd, yd, czc.M_ALL, **kw)
         ev[i][1].record(stream)
-        kms.append(r["kernel_ms"])
     barrier()
     t_wall = time.perf_counter() - t_wall
     clocks = sampler.stop()
+    with czc.Assessor(ndim=3, device=local, stream=stream, timing=True, **cfg) as at:
+        for i in range(args.warmup + args.steps):
+            flush.zero_()
+            clean.sum()
+            r = at.assess(xd, yd, czc.M_ALL, **kw)
+            if i >= args.warmup:
+                kms.append(r["kernel_ms"])
     step_ms = [s.elapsed_time(e) for s, e in ev]
     tot_ms = sum(step_ms)
     if world > 1:
