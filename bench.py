@@ -40,6 +40,7 @@ def parse():
     p.add_argument("--config", default="C2")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-f64", action="store_true", help="skip the float64-input measurement")
     return p.parse_args()
 
 
@@ -291,6 +292,37 @@ def run_ours(args, rank, world, local):
                "h2d_bytes_per_step": nbytes_rank, "d2h_bytes_per_step": d2h_host,
                "ms_per_step": round(e_tot / nsteps_e2e, 4)}
 
+    # float64 inputs (NEXT row f3): the same field widened to double, 16 B per element pair
+    f64 = None
+    if world == 1 and not args.no_f64:
+        xd64, yd64 = xd.double(), yd.double()
+        n64 = 2 * xd64.numel() * 8
+        with czc.Assessor(ndim=3, device=local, stream=stream, **cfg) as a64, \
+                czc.Assessor(ndim=3, device=local, stream=stream, timing=True, **cfg) as t64:
+            for _ in range(args.warmup):
+                a64.assess(xd64, yd64, czc.M_ALL)
+            tot64, k64 = 0.0, []
+            for i in range(args.steps):
+                flush.zero_()
+                clean.sum()
+                s_ev, e_ev = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                s_ev.record(stream)
+                a64.assess(xd64, yd64, czc.M_ALL)
+                e_ev.record(stream)
+                e_ev.synchronize()
+                tot64 += s_ev.elapsed_time(e_ev)
+                flush.zero_()
+                clean.sum()
+                k64.append(t64.assess(xd64, yd64, czc.M_ALL)["kernel_ms"])
+        sh64 = {name: statistics.mean(k[i] for k in k64)
+                for i, name in enumerate(("P1", "P2_deriv", "P2_autocorr", "P3_ssim"))}
+        f64 = {"value": round(n64 * args.steps / (tot64 * 1e-3) / 1e9, 3), "unit": UNIT,
+               "ms_per_step": round(tot64 / args.steps, 4), "dtype": "f64",
+               "workload": f"the same field widened to float64 ({n64 / 1e6:.0f} MB pair)",
+               "per_pattern_ms": {k: round(v, 4) for k, v in sh64.items()},
+               "per_pattern_gbs": {k: round(n64 / (v * 1e-3) / 1e9, 2) for k, v in sh64.items() if v > 0}}
+        del xd64, yd64
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         v, dt, cores, desc = oracle_sample(spec, planes=spec.dims[0])
@@ -315,7 +347,8 @@ def run_ours(args, rank, world, local):
                          "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
                          "peak_source": peak_src, "traffic_source": traffic_src,
                          "algorithmic_bytes_per_launch": alg_bytes},
-            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches_per_step * args.steps,
+            "cpu_baseline": cpu, "e2e": e2e, "float64_inputs": f64,
+            "gpu_launches": launches_per_step * args.steps,
             "clocks": clocks, "wall_s_timed_region": round(t_wall, 4),
         }
         print(json.dumps(line), flush=True)

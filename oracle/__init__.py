@@ -52,7 +52,8 @@ class _Deriv(ctypes.Structure):
 
 def build(force: bool = False) -> str:
     """Compile liboracle.so with gcc (-O2 -fopenmp -ffp-contract=off)."""
-    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
+    srcs = (_SRC, os.path.join(_HERE, "czc_oracle_t.inc"), os.path.join(_HERE, "czc_oracle.h"))
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < max(os.path.getmtime(f) for f in srcs):
         cmd = ["gcc", "-O2", "-fopenmp", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared",
                "-std=c11", "-Wall", "-o", _SO, _SRC, "-lm"]
         subprocess.check_call(cmd)

@@ -10,7 +10,7 @@ python -m paper_conf_cluster_yudgtc21_b200.build > gpurun_out/build.log 2>&1 || 
 timeout 600 python bench.py > gpurun_out/bench_${TAG}.json 2> gpurun_out/bench_${TAG}.err
 timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/bench_ref_${TAG}.json 2> gpurun_out/bench_ref_${TAG}.err
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
-    --log-file gpurun_out/launches_${TAG}.csv python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline > gpurun_out/ncu_bench_${TAG}.log 2>&1
+    --log-file gpurun_out/launches_${TAG}.csv python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline --no-f64 > gpurun_out/ncu_bench_${TAG}.log 2>&1
 timeout 1200 ncu --set full --clock-control none --import-source on -f -o gpurun_out/prof_${TAG} \
     python tools/ncu_target.py C2 1 > gpurun_out/ncu_full_${TAG}.log 2>&1
 cat gpurun_out/bench_${TAG}.json gpurun_out/bench_ref_${TAG}.json
