@@ -113,17 +113,16 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
   const double K = (zb < zend) ? (double)f.xp(zb)[ky * f.nx + kx] : 0.0;
   const double Lglob = (double)res->p1g.xmax - (double)res->p1g.xmin;
 
-  // in-plane offsets (a plane has < 2^31 elements; the launcher checks) and validity bits
-  const int64_t gx = x0 + lane;
+  // In-plane offsets (a plane has < 2^31 elements; the launcher checks).  Footprint rows and
+  // columns past the field edge read the clamped edge sample instead of being predicated: they
+  // feed only windows whose origin is outside the window grid, which the `ok` mask drops, and
+  // every row adds and later subtracts the same samples.
+  const int64_t gxc = x0 + lane < f.nx ? x0 + lane : f.nx - 1;
   int off[KC];
-  unsigned vbits = 0;
 #pragma unroll
   for (int k = 0; k < KC; k++) {
-    const int r = warp + kP3Warps * k;
-    const int64_t gy = y0 + r;
-    const bool v = r < FY && gy < f.ny && gx < f.nx;
-    vbits |= (v ? 1u : 0u) << k;
-    off[k] = v ? (int)(gy * f.nx + gx) : 0;
+    const int64_t gy = y0 + warp + kP3Warps * k;
+    off[k] = (int)((gy < f.ny ? gy : f.ny - 1) * f.nx + gxc);
   }
   // Prefetch of plane zb + n (x, y) and of the y sample of the plane leaving the z-window
   // (zb + n - WZ), which is re-read from L2 instead of being kept in the register ring.  Both
@@ -131,15 +130,15 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
   const int nsteps = (int)(zend - zb);
   SegCursor<T> cin, cold;
   if (nsteps > 0) { cin.init(f, zb); cold.init(f, zb); }
-  auto load = [&](int n, Pair<T> (&dst)[KC], T (&yold)[KC]) {
-    if (n < nsteps) {
-      const bool has_old = n >= WZ;
+  Pair<T> nxt[KC];                                       // prefetched next plane
+  T nyo[KC];                                             // ... and its leaving y sample
+  auto load = [&](int n, bool has_old) {                 // has_old: n >= WZ (constant per call site)
+    if (n < nsteps) {                                    // block-uniform
 #pragma unroll
       for (int k = 0; k < KC; k++) {
-        const bool v = (vbits >> k) & 1u;
-        dst[k].x = v ? __ldg(cin.x + off[k]) : (T)0;
-        dst[k].y = v ? __ldg(cin.y + off[k]) : (T)0;
-        yold[k] = (v && has_old) ? __ldg(cold.y + off[k]) : (T)0;
+        nxt[k].x = __ldg(cin.x + off[k]);
+        nxt[k].y = __ldg(cin.y + off[k]);
+        nyo[k] = has_old ? __ldg(cold.y + off[k]) : (T)0;
       }
       cin.advance(f, zb + n + 1);
       if (has_old) cold.advance(f, zb + n + 1 - WZ);
@@ -155,11 +154,10 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
 #pragma unroll
     for (int s = 0; s < WZ; s++) ring[k][s] = 0;
   }
-  Pair<T> nxt[KC];                                       // prefetched next plane
-  T nyo[KC];                                             // ... and its leaving y sample
-  load(0, nxt, nyo);
+  load(0, false);
 
-  double ssum = 0, scnt = 0;
+  double ssum = 0;
+  unsigned scnt = 0;
   const bool range_global = p.range_mode != 0;
   // origin-grid membership: x and y are fixed per thread, z advances one plane per step
   const int64_t gxl = x0 + lane;
@@ -171,125 +169,137 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
     gok[g] = xok && gy <= f.ny - WY && (gy % p.sy) == 0;
   }
   int zph = (int)(zb % p.sz);                            // phase of origin plane zb
-  for (int s0 = 0; s0 < nsteps; s0 += WZ) {
+
+  // One plane step; s = step mod WZ (the ring slot) and warm = (step >= WZ: a plane leaves the
+  // z-window) are compile-time constants at every call site, so the ring rotates statically and
+  // the warm-up planes carry no per-step tests.
+  auto step_body = [&](const int step, const int s, const bool warm) {
+    // the prefetched plane is consumed by the z-walk below, then the next one is requested
+    // into the same registers (no copies; its latency hides behind the y / x passes)
+    const int buf = step & 1;
+    double* Zd = reinterpret_cast<double*>(smem_raw + buf * Gm::buf_bytes);
+    T* Zm = reinterpret_cast<T*>(Zd + 4 * ZS);
+    const bool full = warm || s == WZ - 1;               // a complete z-window ends here
+    // ---- (a) z-walk --------------------------------------------------------------------
+#pragma unroll
+    for (int k = 0; k < KC; k++) {
+      {
+        const double xd = nxt[k].x, yd = nxt[k].y;
+        const double a = xd - K, b = yd - K, e = yd - xd;
+        sm[k][0] += a; sm[k][1] += e; sm[k][2] = fma(a, b, sm[k][2]); sm[k][3] = fma(e, e, sm[k][3]);
+      }
+      if (warm) {
+        const double xd = ring[k][s], yd = nyo[k];
+        const double a = xd - K, b = yd - K, e = yd - xd;
+        sm[k][0] -= a; sm[k][1] -= e; sm[k][2] = fma(-a, b, sm[k][2]); sm[k][3] = fma(-e, e, sm[k][3]);
+      }
+      ring[k][s] = nxt[k].x;
+      const int r = warp + kP3Warps * k;
+      if (full && (kP3Warps * (k + 1) <= FY || r < FY)) {
+        T mn = ring[k][0], mx = ring[k][0];
+#pragma unroll
+        for (int t = 1; t < WZ; t++) { mn = tmin(mn, ring[k][t]); mx = tmax(mx, ring[k][t]); }
+        const int c = r * 32 + lane;
+#pragma unroll
+        for (int m = 0; m < 4; m++) Zd[m * ZS + c] = sm[k][m];
+        Zm[c] = mn;
+        Zm[ZS + c] = mx;
+      }
+    }
+    load(step + 1, warm || s == WZ - 1);
+    if (!full) return;                                   // no complete z-window yet
+    __syncthreads();
+    const bool zok = zph == 0;                           // origin plane zb + step - WZ + 1
+    zph = zph + 1 == p.sz ? 0 : zph + 1;
+    // ---- (b) y-pass: the G origin rows of this warp (running sums over WY rows) ------------
+    double h[G][4];
+    T hmn[G], hmx[G];
+    {
+      // y-window min/max: the WY - G + 1 rows shared by all G windows are reduced once
+      T cmn = Zm[(warp * G + G - 1) * 32 + lane], cmx = Zm[ZS + (warp * G + G - 1) * 32 + lane];
+#pragma unroll
+      for (int i = G; i < WY; i++) {
+        cmn = tmin(cmn, Zm[(warp * G + i) * 32 + lane]);
+        cmx = tmax(cmx, Zm[ZS + (warp * G + i) * 32 + lane]);
+      }
+#pragma unroll
+      for (int g = 0; g < G; g++) {
+        const int oy = warp * G + g;
+#pragma unroll
+        for (int m = 0; m < 4; m++) {
+          if (g == 0) {
+            double acc = 0;
+#pragma unroll
+            for (int i = 0; i < WY; i++) acc += Zd[m * ZS + (oy + i) * 32 + lane];
+            h[g][m] = acc;
+          } else {
+            h[g][m] = h[g - 1][m] + (Zd[m * ZS + (oy + WY - 1) * 32 + lane] - Zd[m * ZS + (oy - 1) * 32 + lane]);
+          }
+        }
+        T mn = cmn, mx = cmx;                            // rows [G-1, WY) relative to warp*G
+#pragma unroll
+        for (int i = g; i < G - 1; i++) {                // rows oy .. warp*G + G - 2
+          mn = tmin(mn, Zm[(warp * G + i) * 32 + lane]);
+          mx = tmax(mx, Zm[ZS + (warp * G + i) * 32 + lane]);
+        }
+#pragma unroll
+        for (int i = WY; i < WY + g; i++) {              // rows warp*G + WY .. oy + WY - 1
+          mn = tmin(mn, Zm[(warp * G + i) * 32 + lane]);
+          mx = tmax(mx, Zm[ZS + (warp * G + i) * 32 + lane]);
+        }
+        hmn[g] = mn;
+        hmx[g] = mx;
+      }
+    }
+    // ---- (c) x-pass for all G rows together (independent shuffle chains -> ILP), then mix --
+    double S[G][4];
+    T wmn[G], wmx[G];
+#pragma unroll
+    for (int g = 0; g < G; g++) {
+#pragma unroll
+      for (int m = 0; m < 4; m++) S[g][m] = lane_window_sum<WX>(h[g][m]);
+      wmn[g] = lane_window_ext<WX, false>(hmn[g]);
+      wmx[g] = lane_window_ext<WX, true>(hmx[g]);
+    }
+#pragma unroll
+    for (int g = 0; g < G; g++) {
+      const bool ok = zok && gok[g];
+      // computed by every lane (no divergence); invalid lanes are masked out of the sums
+      const double mua = S[g][0] * invM, mue = S[g][1] * invM;
+      const double mux = K + mua, muy = mux + mue;
+      const double sxy = S[g][2] * invM - mua * (mua + mue);
+      const double see = S[g][3] * invM - mue * mue;
+      double L = range_global ? Lglob : (double)wmx[g] - (double)wmn[g];
+      L = (L == 0.0) ? 1.0 : L;
+      const double C1 = (0.01 * L) * (0.01 * L), C2 = (0.03 * L) * (0.03 * L);
+      const double A = 2.0 * mux * muy + C1, B = 2.0 * sxy + C2;
+      // A, B, A + mu_e^2, B + s_e^2 > 0 (C1, C2 > 0); |rel err of the reciprocal| <= 2u
+      const double ssim = (A * B) * fast_rcp((A + mue * mue) * (B + see));
+      ssum += ok ? ssim : 0.0;
+      scnt += ok ? 1u : 0u;
+      if (dbg && ok) {
+        const int64_t oz = zb + step - WZ + 1, gy = y0 + warp * G + g;
+        dbg[((oz / p.sz) * p.nwy + gy / p.sy) * p.nwx + (x0 + lane) / p.sx] = ssim;
+      }
+    }
+  };
+
+  // warm-up: planes 0 .. WZ-1 (the last one completes the first z-window)
+#pragma unroll
+  for (int s = 0; s < WZ; s++) {
+    if (s >= nsteps) break;                              // block-uniform
+    step_body(s, s, false);
+  }
+  for (int s0 = WZ; s0 < nsteps; s0 += WZ) {
 #pragma unroll
     for (int s = 0; s < WZ; s++) {
       const int step = s0 + s;                           // == s (mod WZ)
       if (step >= nsteps) break;                         // block-uniform
-      // the prefetched plane is consumed by the z-walk below, then the next one is requested
-      // into the same registers (no copies; its latency hides behind the y / x passes)
-      const Pair<T> (&v)[KC] = nxt;
-      const T (&yo)[KC] = nyo;
-      const int buf = step & 1;
-      double* Zd = reinterpret_cast<double*>(smem_raw + buf * Gm::buf_bytes);
-      T* Zm = reinterpret_cast<T*>(Zd + 4 * ZS);
-      // ---- (a) z-walk --------------------------------------------------------------------
-#pragma unroll
-      for (int k = 0; k < KC; k++) {
-        {
-          const double xd = v[k].x, yd = v[k].y;
-          const double a = xd - K, b = yd - K, e = yd - xd;
-          sm[k][0] += a; sm[k][1] += e; sm[k][2] = fma(a, b, sm[k][2]); sm[k][3] = fma(e, e, sm[k][3]);
-        }
-        if (step >= WZ) {
-          const double xd = ring[k][s], yd = yo[k];
-          const double a = xd - K, b = yd - K, e = yd - xd;
-          sm[k][0] -= a; sm[k][1] -= e; sm[k][2] = fma(-a, b, sm[k][2]); sm[k][3] = fma(-e, e, sm[k][3]);
-        }
-        ring[k][s] = v[k].x;
-        const int r = warp + kP3Warps * k;
-        if (step >= WZ - 1 && r < FY) {
-          T mn = ring[k][0], mx = ring[k][0];
-#pragma unroll
-          for (int t = 1; t < WZ; t++) { mn = tmin(mn, ring[k][t]); mx = tmax(mx, ring[k][t]); }
-          const int c = r * 32 + lane;
-#pragma unroll
-          for (int m = 0; m < 4; m++) Zd[m * ZS + c] = sm[k][m];
-          Zm[c] = mn;
-          Zm[ZS + c] = mx;
-        }
-      }
-      load(step + 1, nxt, nyo);
-      if (step < WZ - 1) continue;                       // no complete z-window yet
-      __syncthreads();
-      const bool zok = zph == 0;                         // origin plane zb + step - WZ + 1
-      zph = zph + 1 == p.sz ? 0 : zph + 1;
-      // ---- (b) y-pass over WY rows, (c) x-pass with shuffles, mix ------------------------
-      // ---- (b) y-pass: the G origin rows of this warp (running sums over WY rows) ------------
-      double h[G][4];
-      T hmn[G], hmx[G];
-      {
-        // y-window min/max: the WY - G + 1 rows shared by all G windows are reduced once
-        T cmn = Zm[(warp * G + G - 1) * 32 + lane], cmx = Zm[ZS + (warp * G + G - 1) * 32 + lane];
-#pragma unroll
-        for (int i = G; i < WY; i++) {
-          cmn = tmin(cmn, Zm[(warp * G + i) * 32 + lane]);
-          cmx = tmax(cmx, Zm[ZS + (warp * G + i) * 32 + lane]);
-        }
-#pragma unroll
-        for (int g = 0; g < G; g++) {
-          const int oy = warp * G + g;
-#pragma unroll
-          for (int m = 0; m < 4; m++) {
-            if (g == 0) {
-              double acc = 0;
-#pragma unroll
-              for (int i = 0; i < WY; i++) acc += Zd[m * ZS + (oy + i) * 32 + lane];
-              h[g][m] = acc;
-            } else {
-              h[g][m] = h[g - 1][m] + (Zd[m * ZS + (oy + WY - 1) * 32 + lane] - Zd[m * ZS + (oy - 1) * 32 + lane]);
-            }
-          }
-          T mn = cmn, mx = cmx;                          // rows [G-1, WY) relative to warp*G
-#pragma unroll
-          for (int i = g; i < G - 1; i++) {              // rows oy .. warp*G + G - 2
-            mn = tmin(mn, Zm[(warp * G + i) * 32 + lane]);
-            mx = tmax(mx, Zm[ZS + (warp * G + i) * 32 + lane]);
-          }
-#pragma unroll
-          for (int i = WY; i < WY + g; i++) {            // rows warp*G + WY .. oy + WY - 1
-            mn = tmin(mn, Zm[(warp * G + i) * 32 + lane]);
-            mx = tmax(mx, Zm[ZS + (warp * G + i) * 32 + lane]);
-          }
-          hmn[g] = mn;
-          hmx[g] = mx;
-        }
-      }
-      // ---- (c) x-pass for all G rows together (independent shuffle chains -> ILP), then mix --
-      double S[G][4];
-      T wmn[G], wmx[G];
-#pragma unroll
-      for (int g = 0; g < G; g++) {
-#pragma unroll
-        for (int m = 0; m < 4; m++) S[g][m] = lane_window_sum<WX>(h[g][m]);
-        wmn[g] = lane_window_ext<WX, false>(hmn[g]);
-        wmx[g] = lane_window_ext<WX, true>(hmx[g]);
-      }
-#pragma unroll
-      for (int g = 0; g < G; g++) {
-        const bool ok = zok && gok[g];
-        // computed by every lane (no divergence); invalid lanes are masked out of the sums
-        const double mua = S[g][0] * invM, mue = S[g][1] * invM;
-        const double mux = K + mua, muy = mux + mue;
-        const double sxy = S[g][2] * invM - mua * (mua + mue);
-        const double see = S[g][3] * invM - mue * mue;
-        double L = range_global ? Lglob : (double)wmx[g] - (double)wmn[g];
-        L = (L == 0.0) ? 1.0 : L;
-        const double C1 = (0.01 * L) * (0.01 * L), C2 = (0.03 * L) * (0.03 * L);
-        const double A = 2.0 * mux * muy + C1, B = 2.0 * sxy + C2;
-        // A, B, A + mu_e^2, B + s_e^2 > 0 (C1, C2 > 0); |rel err of the reciprocal| <= 2u
-        const double ssim = (A * B) * fast_rcp((A + mue * mue) * (B + see));
-        ssum += ok ? ssim : 0.0;
-        scnt += ok ? 1.0 : 0.0;
-        if (dbg && ok) {
-          const int64_t oz = zb + step - WZ + 1, gy = y0 + warp * G + g;
-          dbg[((oz / p.sz) * p.nwy + gy / p.sy) * p.nwx + (x0 + lane) / p.sx] = ssim;
-        }
-      }
+      step_body(step, s, true);
     }
   }
 
-  double rec[kSsimSlots] = {ssum, scnt, 0.0};
+  double rec[kSsimSlots] = {ssum, (double)scnt, 0.0};
   const unsigned bid = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
   struct Sum { __device__ int operator()(int) const { return OP_SUM; } };
   __syncthreads();
