@@ -26,21 +26,26 @@ int czco_threads(void) {
 #endif
 }
 
-/* Right-align a shape into (nz, ny, nx); returns 0 if invalid. */
-static int shape3(int ndim, const int64_t* dims, int64_t n3[3]) {
-  if (ndim < 1 || ndim > 3 || !dims) return 0;
-  n3[0] = n3[1] = n3[2] = 1;
+/* Shapes: ndim 1..4 (4-D is NEXT row f3), right-aligned into NA = 4 axes with leading 1s (an
+ * axis of extent 1 is inactive).  Returns 0 if invalid. */
+#define NA 4
+static int shape4(int ndim, const int64_t* dims, int64_t n[NA]) {
+  if (ndim < 1 || ndim > NA || !dims) return 0;
+  for (int a = 0; a < NA; a++) n[a] = 1;
   for (int i = 0; i < ndim; i++) {
     if (dims[i] < 1) return 0;
-    n3[3 - ndim + i] = dims[i];
+    n[NA - ndim + i] = dims[i];
   }
   return 1;
 }
-
-/* Type-independent helpers of the pattern sections below. */
-static int window3(int ndim, const int64_t* v, int64_t out[3], int64_t fill) {
-  out[0] = out[1] = out[2] = fill;
-  for (int i = 0; i < ndim; i++) out[3 - ndim + i] = v[i];
+static void strides4(const int64_t n[NA], int64_t st[NA]) {
+  st[NA - 1] = 1;
+  for (int a = NA - 2; a >= 0; a--) st[a] = st[a + 1] * n[a + 1];
+}
+/* Per-axis window extents / steps / origins right-aligned like the shape (leading `fill`). */
+static int window4(int ndim, const int64_t* v, int64_t out[NA], int64_t fill) {
+  for (int a = 0; a < NA; a++) out[a] = fill;
+  for (int i = 0; i < ndim; i++) out[NA - ndim + i] = v[i];
   return 1;
 }
 

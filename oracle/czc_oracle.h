@@ -11,9 +11,10 @@
  * silent or garbled the reading taken is SURVEY.md §8(c)'s register (R1..R23), listed again in
  * DESIGN.md §2.  Citations "Lnnn" are lines of PAPER.md.
  *
- * Shapes: ndim in 1..3, dims slowest-first, C order (x = last axis contiguous).  Internally a shape
- * is right-aligned into (nz, ny, nx) with leading 1s; an axis with n == 1 is "inactive" (it
- * carries no stencil neighbour, no lag and a window extent of 1).  D = number of active axes.
+ * Shapes: ndim in 1..4 (4-D: NEXT row f3, L92), dims slowest-first, C order (x = last axis
+ * contiguous).  Internally a shape is right-aligned into four axes with leading 1s; an axis with
+ * n == 1 is "inactive" (it carries no stencil neighbour, no lag and a window extent of 1).
+ * D = number of active axes.
  */
 #ifndef CZC_ORACLE_H
 #define CZC_ORACLE_H

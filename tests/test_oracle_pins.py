@@ -447,3 +447,84 @@ class TestFloat64:
         assert abs(d["grad_mae"] - np.mean(np.abs(grad))) < 1e-9 * np.mean(np.abs(grad)) + 1e-15
         s, nw = orc.ssim(x, y, [3, 3, 3])
         assert nw == 4 * 5 * 7 and 0.0 < s <= 1.0
+
+
+# ------------------------------------------------------------------------ 4-D fields (NEXT f3)
+class TestFourD:
+    """4-D fields (L92: "easily extended to other dimensions (including 1D, 2D, and 4D)"): the
+    same definitions over four axes, pinned by closed forms, numpy and an invariant tying 4-D
+    windows to 3-D ones."""
+
+    def test_ramp_and_quadratic_closed_forms(self, orc):
+        shape = (5, 6, 7, 8)
+        p = np.indices(shape).astype(np.float64)
+        c = np.array([2 ** -2, 2 ** -3, -(2 ** -4), 2 ** -5])
+        q = np.array([2 ** -4, -(2 ** -5), 2 ** -3, 2 ** -6])
+        x = np.tensordot(c, p, 1).astype(np.float32)
+        y = (np.tensordot(c, p, 1) + np.tensordot(q, p ** 2, 1)).astype(np.float32)
+        r = orc.deriv(x, y)
+        assert r["n_interior"] == 3 * 4 * 5 * 6
+        assert r["der1_f_min"] == r["der1_f_max"] == 2 * np.abs(c).sum()
+        assert r["div_f_max"] == c.sum() and r["lap_f_max"] == 0
+        assert r["grad_f_max"] == pytest.approx(math.sqrt((c ** 2).sum()), abs=1e-15)
+        assert r["lap_maxabs"] == 2 * q.sum() and r["lap_mse"] == (2 * q.sum()) ** 2
+
+    def test_against_numpy_gradient(self, orc):
+        r4 = np.random.default_rng(5)
+        x = r4.standard_normal((6, 7, 8, 9)).astype(np.float32)
+        y = (x + 1e-3 * r4.standard_normal(x.shape)).astype(np.float32)
+        r = orc.deriv(x, y)
+        xd, yd = x.astype(np.float64), y.astype(np.float64)
+        inner = (slice(1, -1),) * 4
+        gx = np.sqrt(sum(g ** 2 for g in np.gradient(xd)))[inner]
+        gy = np.sqrt(sum(g ** 2 for g in np.gradient(yd)))[inner]
+        assert abs(r["grad_mae"] - np.mean(np.abs(gy - gx))) < 1e-12
+        lap = lambda f: sum(np.roll(f, 1, a) - 2 * f + np.roll(f, -1, a) for a in range(4))[inner]
+        assert abs(r["lap_mse"] - np.mean((lap(yd) - lap(xd)) ** 2)) < 1e-12 * r["lap_mse"] + 1e-18
+        assert r["der1_f_max"] == pytest.approx(
+            sum(np.abs(np.roll(xd, -1, a) - np.roll(xd, 1, a)) for a in range(4))[inner].max(), rel=1e-15)
+
+    def test_autocorr_checkerboard_and_axis(self, orc):
+        shape = (8, 9, 10, 11)
+        i = np.indices(shape).sum(0)
+        x = np.zeros(shape, np.float32)
+        y = np.where(i % 2 == 0, 1.0, -1.0).astype(np.float32)
+        ac, cnt = orc.autocorr(x, y, 5)
+        # e = (-1)^(i0+i1+i2+i3) has mean ~0 but not exactly (odd extent): compare with numpy
+        e = y.astype(np.float64)
+        mu, var = e.mean(), e.var()
+        for t in range(1, 6):
+            hi = tuple(slice(0, n - t) for n in shape)
+            s = 0.0
+            for a in range(4):
+                sh = [slice(0, n - t) for n in shape]
+                sh[a] = slice(t, shape[a])
+                s += np.sum((e[hi] - mu) * (e[tuple(sh)] - mu))
+            want = s / 4 / np.prod([n - t for n in shape]) / var
+            assert abs(ac[t] - want) < 1e-12, (t, ac[t], want)
+            assert cnt[t] == np.prod([n - t for n in shape])
+        assert ac[1] < -0.99 and ac[2] > 0.99
+
+    def test_ssim_zero_error_brute_force_and_replication(self, orc):
+        r4 = np.random.default_rng(9)
+        x = (280 + r4.standard_normal((5, 6, 7, 8))).astype(np.float32)
+        assert orc.ssim(x, x, [3, 3, 3, 3]) == (1.0, 3 * 4 * 5 * 6)
+        y = (x + 1e-2 * r4.standard_normal(x.shape)).astype(np.float32)
+        # per-window numpy (np.var / np.cov definitions) at two origins
+        for o in ((0, 1, 2, 3), (2, 3, 0, 1)):
+            w = (3, 3, 4, 5)
+            sl = tuple(slice(a, a + b) for a, b in zip(o, w))
+            xw, yw = x[sl].astype(np.float64).ravel(), y[sl].astype(np.float64).ravel()
+            L = xw.max() - xw.min()
+            C1, C2 = (0.01 * L) ** 2, (0.03 * L) ** 2
+            cov = np.cov(xw, yw, bias=True)
+            want = ((2 * xw.mean() * yw.mean() + C1) * (2 * cov[0, 1] + C2) /
+                    ((xw.mean() ** 2 + yw.mean() ** 2 + C1) * (cov[0, 0] + cov[1, 1] + C2)))
+            assert abs(orc.ssim_window(x, y, o, w) - want) < 1e-12
+        # a 4-D field replicating a 3-D one along axis 0, windows spanning that axis: every 4-D
+        # window holds w0 copies of a 3-D window -> the same local SSIM, the same mean
+        x3, y3 = x[0], y[0]
+        x4, y4 = np.repeat(x3[None], 3, 0), np.repeat(y3[None], 3, 0)
+        s3, n3 = orc.ssim(x3, y3, [3, 4, 5])
+        s4, n4 = orc.ssim(x4, y4, [3, 3, 4, 5])
+        assert n3 == n4 and abs(s3 - s4) < 1e-13
