@@ -18,8 +18,10 @@
  * Metric definitions and every reading taken where the paper is silent: DESIGN.md §2.
  *
  * Conventions (all entry points):
- *   - Shapes: ndim 1..3, dims slowest-first, C order; the last axis is contiguous.  An axis of
- *     extent 1 is inactive (no stencil neighbour, no lag, window extent 1).
+ *   - Shapes: ndim 1..4, dims slowest-first, C order; the last axis is contiguous.  An axis of
+ *     extent 1 is inactive (no stencil neighbour, no lag, window extent 1).  Fields with at most
+ *     three active axes run on the streamed 3-D engines; four active axes (L92: "easily extended
+ *     to ... 4D"; NEXT row f3) run generic grid-stride kernels (single GPU, no slab mode).
  *   - Every function returns czc_status; nothing aborts and no C++ exception crosses the ABI.
  *     On error, out->computed_mask = 0 and nothing else in *out is meaningful.
  *   - Undefined metrics are NaN (e.g. Pearson with zero variance, AC with sigma_e^2 = 0, pwr
@@ -37,7 +39,8 @@
 extern "C" {
 #endif
 
-#define CZC_ABI_VERSION 3
+#define CZC_ABI_VERSION 4
+#define CZC_MAX_DIMS 4           /* ndim 1..3 on the streamed engines; 4-D fields (NEXT row f3)    */
 #define CZC_MAX_LAG 16           /* largest supported autocorrelation lag (paper uses <= 10, L345) */
 #define CZC_PDF_MAX_BINS 256     /* largest number of error-PDF bins                              */
 
@@ -78,8 +81,8 @@ typedef struct czc_config {
   void* stream;                  /* cudaStream_t to run on; NULL = a BLOCKING stream owned by the */
                                  /* context (ordered after the caller's legacy-default-stream    */
                                  /* work, e.g. PyTorch's default stream, handle 0)               */
-  int ssim_window[3];            /* window extent per input axis (index i <-> dims[i]); 0 -> 8   */
-  int ssim_step[3];              /* window step per input axis; 0 -> 1 (L352: w = 8, step 1)     */
+  int ssim_window[CZC_MAX_DIMS]; /* window extent per input axis (index i <-> dims[i]); 0 -> 8   */
+  int ssim_step[CZC_MAX_DIMS];   /* window step per input axis; 0 -> 1 (L352: w = 8, step 1)     */
   int ssim_range_mode;           /* 0: L = max - min of the original window (reading R15)        */
                                  /* 1: L = value range of the whole original field               */
   int ac_max_lag;                /* autocorrelation lags 1..ac_max_lag (<= CZC_MAX_LAG); 0 -> 10 */
@@ -101,7 +104,7 @@ typedef struct czc_config {
  * Slab mode: dims are GLOBAL; this rank's buffers hold planes [z0, z0 + nz_local) of axis 0. */
 typedef struct czc_shape {
   int ndim;
-  int64_t dims[3];
+  int64_t dims[CZC_MAX_DIMS];
   int64_t z0;
   int64_t nz_local;
 } czc_shape;
@@ -131,7 +134,7 @@ typedef struct czc_result {
   double ac[CZC_MAX_LAG + 1];                         /* ac[0] = 1                               */
   uint64_t ac_count[CZC_MAX_LAG + 1];                 /* ne_tau = prod_a (n_a - tau)             */
   /* ---- P3 SSIM (L139-L146) ------------------------------------------------------------------- */
-  int32_t ssim_window[3], ssim_step[3];               /* as used, per input axis                 */
+  int32_t ssim_window[CZC_MAX_DIMS], ssim_step[CZC_MAX_DIMS];   /* as used, per input axis      */
   uint64_t n_windows;
   double ssim;
   uint64_t n_ssim_exact;         /* windows whose fast-path error bound failed and were          */

@@ -27,6 +27,7 @@ F32, F64 = 0, 1      # czc_dtype
 M_ALL = 0xF          # the four pattern groups (bench.py's step)
 M_FULL = 0x1F        # + the error / pwr-error PDFs (Table I Category I)
 MAX_LAG = 16
+MAX_DIMS = 4         # ndim 1..4 (4-D fields: NEXT row f3)
 PDF_MAX_BINS = 256
 DERIV_FIELDS = ("der1", "der2", "grad", "div", "lap")
 DERIV_STATS = ("maxabs", "mae", "mse", "rmse", "f_min", "f_max", "psnr")
@@ -42,14 +43,14 @@ class CzcError(RuntimeError):
 
 class Config(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("stream", ctypes.c_void_p),
-                ("ssim_window", ctypes.c_int * 3), ("ssim_step", ctypes.c_int * 3),
+                ("ssim_window", ctypes.c_int * MAX_DIMS), ("ssim_step", ctypes.c_int * MAX_DIMS),
                 ("ssim_range_mode", ctypes.c_int), ("ac_max_lag", ctypes.c_int), ("timing", ctypes.c_int),
                 ("rank", ctypes.c_int), ("nranks", ctypes.c_int), ("nccl_uid", ctypes.c_void_p),
                 ("debug_wssim", ctypes.c_void_p), ("loopback_slabs", ctypes.c_int), ("pdf_bins", ctypes.c_int)]
 
 
 class Shape(ctypes.Structure):
-    _fields_ = [("ndim", ctypes.c_int), ("dims", ctypes.c_int64 * 3), ("z0", ctypes.c_int64),
+    _fields_ = [("ndim", ctypes.c_int), ("dims", ctypes.c_int64 * MAX_DIMS), ("z0", ctypes.c_int64),
                 ("nz_local", ctypes.c_int64)]
 
 
@@ -69,7 +70,7 @@ class Result(ctypes.Structure):
                    ("n_interior", ctypes.c_uint64), ("deriv", DerivStats * 5),
                    ("ac_max_lag", ctypes.c_int32), ("_pad0", ctypes.c_int32),
                    ("ac", ctypes.c_double * (MAX_LAG + 1)), ("ac_count", ctypes.c_uint64 * (MAX_LAG + 1)),
-                   ("ssim_window", ctypes.c_int32 * 3), ("ssim_step", ctypes.c_int32 * 3),
+                   ("ssim_window", ctypes.c_int32 * MAX_DIMS), ("ssim_step", ctypes.c_int32 * MAX_DIMS),
                    ("n_windows", ctypes.c_uint64), ("ssim", ctypes.c_double),
                    ("n_ssim_exact", ctypes.c_uint64),
                    ("pdf_bins", ctypes.c_int32), ("_pad1", ctypes.c_int32),
@@ -133,9 +134,9 @@ EXPORTED = ("czc_init", "czc_assess", "czc_assess_host", "czc_combine", "czc_fre
 
 def _per_axis(v, ndim) -> Sequence[int]:
     if isinstance(v, int):
-        return [v] * ndim + [0] * (3 - ndim)
+        return [v] * ndim + [0] * (MAX_DIMS - ndim)
     v = list(v)
-    return v + [0] * (3 - len(v))
+    return v + [0] * (MAX_DIMS - len(v))
 
 
 def make_config(ndim: int = 3, device: int = -1, stream: Optional[int] = None, ssim_window=8, ssim_step=1,

@@ -19,7 +19,7 @@ CSRC = os.path.join(HERE, "csrc")
 OBJ = os.path.join(HERE, "build_obj")
 SO = os.path.join(HERE, "libczc.so")
 ROOT = os.path.dirname(HERE)
-SOURCES = ["czc_api.cu", "czc_comm.cu", "p1_reduce.cu", "p2_stencil.cu", "p3_ssim.cu"]
+SOURCES = ["czc_api.cu", "czc_comm.cu", "p1_reduce.cu", "p2_stencil.cu", "p3_ssim.cu", "p4_generic.cu"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 

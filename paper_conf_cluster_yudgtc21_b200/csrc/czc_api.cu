@@ -42,6 +42,17 @@ template <typename E>
 cudaError_t launch_ssim(int kind, int W, const Field3<E>& f, const SsimParams& p,
                         double* parts, DevResults* res, unsigned int* ticket, double* dbg,
                         cudaStream_t st, int64_t* nblocks_out);
+// 4-D fields (p4_generic.cu)
+int64_t g4_max_blocks(int sms);
+template <typename E>
+cudaError_t launch_deriv4(const E* x, const E* y, const int64_t n[4], int sms, double* parts, DevResults* res,
+                          unsigned int* ticket, cudaStream_t st);
+template <typename E>
+cudaError_t launch_ac4(const E* x, const E* y, const int64_t n[4], int T, int sms, double* parts, DevResults* res,
+                       unsigned int* ticket, cudaStream_t st);
+template <typename E>
+cudaError_t launch_ssim4(const E* x, const E* y, const int64_t n[4], const int w[4], const int stp[4], int range_mode,
+                         int sms, double* parts, DevResults* res, unsigned int* ticket, double* dbg, cudaStream_t st);
 }  // namespace czc
 
 using namespace czc;
@@ -111,7 +122,7 @@ static czc_status cuda_fail(czc_ctx* ctx, cudaError_t e, const char* where) {
 static czc_status validate_config(const czc_config& c) {
   if (c.ac_max_lag < 0 || c.ac_max_lag > CZC_MAX_LAG) return CZC_ERR_INVALID;
   if (c.ssim_range_mode < 0 || c.ssim_range_mode > 1) return CZC_ERR_INVALID;
-  for (int i = 0; i < 3; i++)
+  for (int i = 0; i < CZC_MAX_DIMS; i++)
     if (c.ssim_window[i] < 0 || c.ssim_step[i] < 0) return CZC_ERR_INVALID;
   if (c.nranks > 1 && (c.rank < 0 || c.rank >= c.nranks || !c.nccl_uid)) return CZC_ERR_INVALID;
   if (c.nccl_uid && (c.nranks < 1 || c.rank < 0 || c.rank >= c.nranks)) return CZC_ERR_INVALID;
@@ -219,29 +230,33 @@ extern "C" void czc_free(czc_ctx* ctx) {
 namespace {
 struct Plan {
   int64_t g3[3] = {1, 1, 1};      // GLOBAL field, extent-1 axes squeezed, right-aligned (nz, ny, nx)
+  int64_t g4[4] = {1, 1, 1, 1};   // the same right-aligned into four axes (D = 4: all active)
   int D = 0;                      // active axes
+  int win4[4] = {1, 1, 1, 1}, step4[4] = {1, 1, 1, 1};   // SSIM per right-aligned axis (D = 4)
   int W = 8, step[3] = {1, 1, 1}; // SSIM (per 3-D axis)
   int win3[3] = {1, 1, 1};
   int kind = 0;                   // 3, 2, 1 (active axes of the SSIM window)
   int T = 10;
   int nb = 100;                   // PDF bins
   bool run_p1 = false, run_deriv = false, run_ac = false, run_ssim = false, run_pdf = false;
-  int32_t win_in[3] = {0, 0, 0}, step_in[3] = {0, 0, 0};  // reported per input axis
+  int32_t win_in[4] = {0, 0, 0, 0}, step_in[4] = {0, 0, 0, 0};  // reported per input axis
 };
 
 czc_status make_plan(const czc_config& c, int ndim, const int64_t* dims, uint64_t mask, Plan& P, std::string& why) {
-  if (ndim < 1 || ndim > 3) { why = "ndim must be 1..3"; return CZC_ERR_SHAPE; }
-  int64_t gd[3];
+  if (ndim < 1 || ndim > CZC_MAX_DIMS) { why = "ndim must be 1..4"; return CZC_ERR_SHAPE; }
+  int64_t gd[CZC_MAX_DIMS];
   for (int i = 0; i < ndim; i++) {
     if (dims[i] < 1) { why = "dims must be >= 1"; return CZC_ERR_SHAPE; }
     gd[i] = dims[i];
   }
   // squeeze inactive (extent-1) axes; the C-order layout is unchanged by it
-  int act_in[3], na = 0;
+  int act_in[CZC_MAX_DIMS], na = 0;
   for (int i = 0; i < ndim; i++)
     if (gd[i] > 1) act_in[na++] = i;
   P.D = na;
-  for (int k = 0; k < na; k++) P.g3[3 - na + k] = gd[act_in[k]];
+  for (int k = 0; k < na; k++) P.g4[4 - na + k] = gd[act_in[k]];
+  if (na <= 3)
+    for (int k = 0; k < na; k++) P.g3[3 - na + k] = gd[act_in[k]];
   P.T = c.ac_max_lag ? c.ac_max_lag : 10;
   P.run_ssim = (mask & CZC_M_SSIM) != 0;
   P.run_deriv = (mask & CZC_M_DERIV) != 0;
@@ -263,8 +278,12 @@ czc_status make_plan(const czc_config& c, int ndim, const int64_t* dims, uint64_
       if (W < 0) W = w;
       if (w != W) { why = "SSIM fast path needs the same window extent on every active axis"; return CZC_ERR_UNSUPPORTED; }
       if (w > gd[act_in[k]]) { why = "SSIM window larger than the field"; return CZC_ERR_SHAPE; }
-      P.win3[3 - na + k] = w;
-      P.step[3 - na + k] = P.step_in[act_in[k]];
+      P.win4[4 - na + k] = w;
+      P.step4[4 - na + k] = P.step_in[act_in[k]];
+      if (na <= 3) {
+        P.win3[3 - na + k] = w;
+        P.step[3 - na + k] = P.step_in[act_in[k]];
+      }
     }
     if (W < 2 || W > kMaxWin) { why = "SSIM window extent must be 2..16"; return CZC_ERR_UNSUPPORTED; }
     P.W = W;
@@ -329,8 +348,8 @@ void combine_and_finish(const Plan& P, const Record* recs, int nrec, uint64_t ma
   if (P.run_p1 && (mask & CZC_M_P1)) { finish_p1(R.p1, out); done |= CZC_M_P1; }
   if (P.run_deriv) {
     int64_t nI = P.D > 0 ? 1 : 0;
-    for (int a = 0; a < 3; a++)
-      if (P.g3[a] > 1) nI *= std::max<int64_t>(P.g3[a] - 2, 0);
+    for (int a = 0; a < 4; a++)
+      if (P.g4[a] > 1) nI *= std::max<int64_t>(P.g4[a] - 2, 0);
     out->n_interior = (uint64_t)nI;
     for (int f = 0; f < CZC_NDERIV; f++) {
       const double* r = R.deriv + f * kDerivStats;
@@ -354,14 +373,14 @@ void combine_and_finish(const Plan& P, const Record* recs, int nrec, uint64_t ma
     out->ac_max_lag = P.T;
     const double var = R.p1.m2e / R.p1.n;
     int64_t nmin = INT64_MAX;
-    for (int a = 0; a < 3; a++)
-      if (P.g3[a] > 1) nmin = std::min(nmin, P.g3[a]);
+    for (int a = 0; a < 4; a++)
+      if (P.g4[a] > 1) nmin = std::min(nmin, P.g4[a]);
     out->ac[0] = 1.0;
-    out->ac_count[0] = (uint64_t)(P.g3[0] * P.g3[1] * P.g3[2]);
+    out->ac_count[0] = (uint64_t)(P.g4[0] * P.g4[1] * P.g4[2] * P.g4[3]);
     for (int t = 1; t <= CZC_MAX_LAG; t++) {
       if (t > P.T || P.D == 0 || t >= nmin) { out->ac[t] = NAN; out->ac_count[t] = 0; continue; }
       int64_t ne = 1;
-      for (int a = 0; a < 3; a++) ne *= P.g3[a] > 1 ? P.g3[a] - t : 1;
+      for (int a = 0; a < 4; a++) ne *= P.g4[a] > 1 ? P.g4[a] - t : 1;
       out->ac_count[t] = (uint64_t)ne;
       const double S = R.ac[0][t - 1] + R.ac[1][t - 1] + R.ac[2][t - 1];   // z, y, x walks
       out->ac[t] = var > 0 ? S / (double)P.D / (double)ne / var : NAN;
@@ -369,7 +388,7 @@ void combine_and_finish(const Plan& P, const Record* recs, int nrec, uint64_t ma
     done |= CZC_M_AUTOCORR;
   }
   if (P.run_ssim) {
-    for (int i = 0; i < 3; i++) { out->ssim_window[i] = P.win_in[i]; out->ssim_step[i] = P.step_in[i]; }
+    for (int i = 0; i < CZC_MAX_DIMS; i++) { out->ssim_window[i] = P.win_in[i]; out->ssim_step[i] = P.step_in[i]; }
     out->n_windows = (uint64_t)R.ssim[1];
     out->ssim = R.ssim[1] > 0 ? R.ssim[0] / R.ssim[1] : NAN;
     out->n_ssim_exact = (uint64_t)R.ssim[2];
@@ -760,9 +779,48 @@ static czc_status check_common(czc_ctx* ctx, const void* orig, const void* recon
   return CZC_OK;
 }
 
+// Four active axes (NEXT row f3): P1 / PDF on the flat pair, then the generic 4-D stencil,
+// autocorrelation and window kernels (p4_generic.cu); single GPU only.
+template <typename E>
+static czc_status assess_4d(czc_ctx* ctx, const Plan& P, const E* x, const E* y, czc_result* out, uint64_t mask) {
+  const cudaStream_t s = ctx->stream;
+  const bool timing = ctx->cfg.timing != 0;
+  const int64_t N = P.g4[0] * P.g4[1] * P.g4[2] * P.g4[3];
+  const size_t need = std::max((size_t)ctx->p1_grid_cap * sizeof(P1State),
+                               (size_t)g4_max_blocks(ctx->sm_count) * kAcSlots * sizeof(double));
+  czc_status st = ensure_buf(ctx, &ctx->parts, &ctx->parts_cap, need);
+  if (st != CZC_OK) return st;
+  double* parts = (double*)ctx->parts;
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
+  if ((st = p1_local(ctx, P, x, y, N)) != CZC_OK) return st;
+  if (P.run_pdf) CZC_CUDA(ctx, launch_pdf(x, y, N, P.nb, ctx->p1_grid_cap, ctx->dres, s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
+  if (P.run_deriv) CZC_CUDA(ctx, launch_deriv4(x, y, P.g4, ctx->sm_count, parts, ctx->dres, ctx->tickets + TICKET_DERIV, s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
+  if (P.run_ac) CZC_CUDA(ctx, launch_ac4(x, y, P.g4, P.T, ctx->sm_count, parts, ctx->dres, ctx->tickets + TICKET_ACZ, s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));
+  if (P.run_ssim)
+    CZC_CUDA(ctx, launch_ssim4(x, y, P.g4, P.win4, P.step4, ctx->cfg.ssim_range_mode, ctx->sm_count, parts, ctx->dres,
+                               ctx->tickets + TICKET_SSIM, ctx->cfg.debug_wssim, s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
+  CZC_CUDA(ctx, copy_records(ctx->hrec, &ctx->dres->rec, 1, P.run_pdf, s));
+  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[5], s));
+  CZC_CUDA(ctx, cudaStreamSynchronize(s));
+  combine_and_finish(P, ctx->hrec, 1, mask, out);
+  finish_timing(ctx, out);
+  return CZC_OK;
+}
+
 template <typename E>
 static czc_status assess_dispatch(czc_ctx* ctx, const Plan& P, const E* x, const E* y, const czc_shape* shape,
                                   czc_result* out, uint64_t mask) {
+  if (P.D == 4) {
+    if (ctx->comm || ctx->cfg.loopback_slabs > 1) {
+      ctx->last_error = "4-D fields run on one GPU (no slab mode)";
+      return CZC_ERR_UNSUPPORTED;
+    }
+    return assess_4d(ctx, P, x, y, out, mask);
+  }
   if (ctx->comm) return assess_ranks(ctx, P, x, y, shape, out, mask);
   if (ctx->cfg.loopback_slabs > 1) return assess_loopback(ctx, P, x, y, out, mask);
   return assess_single(ctx, P, x, y, out, mask);
@@ -893,7 +951,7 @@ extern "C" czc_status czc_assess_host(czc_ctx* ctx, const void* orig, const void
                                       czc_dtype dtype, uint64_t metric_mask, czc_result* out) {
   czc_status st = check_common(ctx, orig, recon, shape, dtype, out);
   if (st != CZC_OK) return st;
-  if (shape->ndim < 1 || shape->ndim > 3) return CZC_ERR_SHAPE;
+  if (shape->ndim < 1 || shape->ndim > CZC_MAX_DIMS) return CZC_ERR_SHAPE;
   int64_t n = 1;
   for (int i = 0; i < shape->ndim; i++) {
     if (shape->dims[i] < 1) return CZC_ERR_SHAPE;

@@ -633,3 +633,55 @@ def test_f64_dtype_errors(czc):
         r = czc.Result()
         assert czc.lib.czc_assess(a.ctx, x.data_ptr(), x.data_ptr(), ctypes.byref(czc.make_shape([4, 5, 6])),
                                   2, czc.M_P1, ctypes.byref(r)) == 3
+
+
+# ----------------------------------------------------------------- 4-D fields (NEXT row f3, L92)
+def pair4(cfg, shape4, dtype=np.float32):
+    """A 4-D pair: the `cfg` recipe generated as a 3-D field (n0 n1, n2, n3) and viewed in 4-D."""
+    x, y = synth.make_pair(synth.config(cfg, dims=(shape4[0] * shape4[1],) + tuple(shape4[2:])))
+    return (x.numpy().reshape(shape4).astype(dtype), y.numpy().reshape(shape4).astype(dtype))
+
+
+@pytest.mark.parametrize("cfg,shape,w,step,lag", [("C1", (7, 9, 10, 12), 3, 1, 4), ("C2", (6, 8, 20, 24), 4, (1, 2, 1, 3), 6),
+                                                  ("C2q", (5, 6, 17, 19), 5, 1, 10), ("C3", (8, 5, 9, 33), 2, 2, 3)])
+def test_4d_parity(czc, orc, cfg, shape, w, step, lag):
+    x, y = pair4(cfg, shape)
+    g, o = run_both(czc, orc, x, y, window=w, step=step, lag=lag)
+    assert g["computed_mask"] == czc.M_ALL and g["n_interior"] == np.prod([n - 2 for n in shape])
+    full_check(g, o)
+
+
+def test_4d_float64_pdf_debug_and_modes(czc, orc):
+    x, y = pair4("C2", (6, 7, 11, 13), np.float64)
+    y = y + 1e-7 * np.random.default_rng(3).standard_normal(y.shape)
+    g, o = run_both(czc, orc, x, y, window=3, lag=5)
+    full_check(g, o)
+    nw = [n - 3 + 1 for n in x.shape]
+    dbg = torch.empty(nw, dtype=torch.float64, device="cuda")
+    with czc.Assessor(ndim=4, ssim_window=3, pdf_bins=40, ssim_range_mode=1, debug_wssim=dbg.data_ptr()) as a:
+        g = a.assess(torch.from_numpy(x).cuda(), torch.from_numpy(y).cuda(), czc.M_FULL)
+    pdf_check(g, orc.pdf(x.ravel(), y.ravel(), 40), 40)
+    s, n = orc.ssim(x, y, [3] * 4, None, 1)
+    assert g["n_windows"] == n and abs(g["ssim"] - s) < 1e-6
+    d = dbg.cpu().numpy()
+    R = float(x.max() - x.min())
+    for o4 in ((0, 0, 0, 0), (3, 4, 8, 10), (1, 2, 5, 7)):
+        assert abs(d[o4] - orc.ssim_window(x, y, o4, [3] * 4, 1, R)) < 1e-9
+
+
+def test_4d_squeezed_and_unsupported(czc, orc):
+    """A 4-D shape with an extent-1 axis is a 3-D field (streamed engines, identical results);
+    four active axes refuse slab mode."""
+    x, y = synth.make_pair(synth.config("C1", dims=(12, 14, 16)))
+    with czc.Assessor(ndim=3, ssim_window=4) as a:
+        g3 = a.assess(x.cuda(), y.cuda())
+    with czc.Assessor(ndim=4, ssim_window=4) as a:
+        g4 = a.assess(x.cuda().reshape(12, 1, 14, 16), y.cuda().reshape(12, 1, 14, 16))
+    for k in ("x_min", "err_max", "mse", "ssim", "n_windows", "der1_mae", "n_interior"):
+        assert g3[k] == g4[k], k
+    assert np.array_equal(g3["ac"], g4["ac"])
+    x4 = x.cuda().reshape(3, 4, 14, 16)
+    with czc.Assessor(ndim=4, ssim_window=3, loopback_slabs=2) as a:
+        with pytest.raises(czc.CzcError) as ei:
+            a.assess(x4, x4)
+        assert ei.value.status == 7
