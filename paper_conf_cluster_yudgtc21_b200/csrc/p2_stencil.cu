@@ -46,32 +46,47 @@ __device__ __forceinline__ double dmin(double a, double b) { return a < b ? a : 
 // Derived fields of one point.  ZA / YA: the streamed (slow) axis / the in-plane y axis are
 // active; x is always active.  Axis order slow, y, x (slowest first) as in the oracle.  A 2-D
 // field is streamed along its rows: its y axis plays the slow axis (ZA, !YA).
-// The /2 of the central differences D_a = delta_a / 2 is applied once per point: sum D_a =
-// 0.5 sum delta_a and sum D_a^2 = 0.25 sum delta_a^2 hold exactly (power-of-two scaling).
+// The /2 of the central differences D_a = delta_a / 2 is NOT applied per point: F[GRAD] and
+// F[DIV] hold 2 Grad = sqrt(sum delta_a^2) and 2 Div = sum delta_a, and the block's statistics of
+// those two fields are scaled once by scale_halved() (power-of-two scaling is exact).  The sums
+// start from the first active axis (0 + v is not foldable in IEEE arithmetic: -0).
 template <bool ZA, bool YA>
 __device__ __forceinline__ void deriv_fields(const double c, const double zp, const double zm,
                                              const double yp, const double ym, const double xp,
                                              const double xm, double F[CZC_NDERIV]) {
-  double der1 = 0, der2 = 0, d2 = 0, dsum = 0, lap = 0;
-#define CZC_AXIS(P, M)                          \
-  {                                             \
-    const double delta = (P) - (M);             \
-    const double l = (P) - 2.0 * c + (M);       \
-    der1 += fabs(delta);                        \
-    der2 += fabs(l);                            \
-    d2 = fma(delta, delta, d2);                 \
-    dsum += delta;                              \
-    lap += l;                                   \
-  }
-  if (ZA) CZC_AXIS(zp, zm)
-  if (YA) CZC_AXIS(yp, ym)
-  CZC_AXIS(xp, xm)
-#undef CZC_AXIS
+  double der1, der2, d2, dsum, lap;
+  bool first = true;
+  auto axis = [&](const double P, const double M) {
+    const double delta = P - M;
+    const double l = P - 2.0 * c + M;
+    if (first) {
+      der1 = fabs(delta); der2 = fabs(l); d2 = delta * delta; dsum = delta; lap = l;
+    } else {
+      der1 += fabs(delta); der2 += fabs(l); d2 = fma(delta, delta, d2); dsum += delta; lap += l;
+    }
+    first = false;
+  };
+  if (ZA) axis(zp, zm);
+  if (YA) axis(yp, ym);
+  axis(xp, xm);
   F[CZC_DER1] = der1;
   F[CZC_DER2] = der2;
-  F[CZC_GRAD] = 0.5 * fast_sqrt(d2);
-  F[CZC_DIV] = 0.5 * dsum;
+  F[CZC_GRAD] = fast_sqrt(d2);
+  F[CZC_DIV] = dsum;
   F[CZC_LAP] = lap;
+}
+
+// Undo the factor 2 of F[GRAD] / F[DIV] (deriv_fields) in a block's accumulators:
+// max |dF|, sum |dF|, min F, max F scale by 1/2, sum dF^2 by 1/4 — exact.
+__device__ __forceinline__ void scale_halved(double (&acc)[kDerivSlots]) {
+#pragma unroll
+  for (int f : {CZC_GRAD, CZC_DIV}) {
+    acc[f * kDerivStats + 0] *= 0.5;
+    acc[f * kDerivStats + 1] *= 0.5;
+    acc[f * kDerivStats + 2] *= 0.25;
+    acc[f * kDerivStats + 3] *= 0.5;
+    acc[f * kDerivStats + 4] *= 0.5;
+  }
 }
 
 struct DerivOp {
@@ -165,6 +180,7 @@ deriv_kernel(Field3<T> s, int zchunk, double* __restrict__ parts, DevResults* __
     xm = x0; x0 = xp; ym = y0; y0 = yp;
   }
   __syncthreads();
+  scale_halved(acc);
   const unsigned bid = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
   block_reduce_slots<kDerivSlots>(acc, DerivOp{}, parts + (size_t)bid * kDerivSlots);
   if (!last_block_arrive(ticket)) return;
@@ -286,6 +302,7 @@ deriv3_kernel(Field3<T> s, int zchunk, double* __restrict__ parts, DevResults* _
     for (int p = 0; p < PTS; p++) { xm[p] = x0[p]; x0[p] = xp[p]; ym[p] = y0[p]; y0[p] = yp[p]; }
   }
   __syncthreads();
+  scale_halved(acc);
   const unsigned bid = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
   block_reduce_slots<kDerivSlots>(acc, DerivOp{}, parts + (size_t)bid * kDerivSlots);
   if (!last_block_arrive(ticket)) return;

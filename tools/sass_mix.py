@@ -10,8 +10,8 @@ h, data = rows[hi], rows[hi + 1:]
 ie, st = h.index("Instructions Executed"), h.index("Warp Stall Sampling (All Samples)")
 cnt, stall = collections.Counter(), collections.Counter()
 for r in data:
-    if len(r) <= ie or not r[ie]:
-        continue
+    if len(r) <= ie or not r[ie] or not r[ie].replace(",", "").isdigit():
+        continue                       # blank rows, repeated headers of further launches
     op = r[1].split()
     if not op:
         continue
