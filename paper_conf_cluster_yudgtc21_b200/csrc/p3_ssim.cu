@@ -316,15 +316,39 @@ static cudaError_t launch_t(const Field3<T>& f, const SsimParams& p, double* par
                             DevResults* res, unsigned int* ticket, double* dbg, cudaStream_t st,
                             int64_t* nblocks_out) {
   using Gm = SsimGeom<T, WX, WY, WZ, G>;
-  int64_t zhi = f.zown1 < f.nz - WZ + 1 ? f.zown1 : f.nz - WZ + 1;
-  const int64_t noz = zhi > f.zown0 ? zhi - f.zown0 : 1;
-  dim3 grid((unsigned)cdiv(f.nx - WX + 1, Gm::TX), (unsigned)cdiv(f.ny - WY + 1, Gm::TY),
-            (unsigned)cdiv(noz, p.zchunk));
-  if (nblocks_out) { *nblocks_out = (int64_t)grid.x * grid.y * grid.z; return cudaSuccess; }
-  if (f.ny * f.nx >= (int64_t)1 << 31) return cudaErrorInvalidValue;   // 32-bit in-plane offsets
+  auto kern = p3_kernel<T, WX, WY, WZ, G>;
   cudaError_t e = set_smem_once<p3_kernel<T, WX, WY, WZ, G>>((int)Gm::smem);
   if (e != cudaSuccess) return e;
-  p3_kernel<T, WX, WY, WZ, G><<<grid, kP3Threads, Gm::smem, st>>>(f, p, parts, res, ticket, dbg);
+  int64_t zhi = f.zown1 < f.nz - WZ + 1 ? f.zown1 : f.nz - WZ + 1;
+  const int64_t noz = zhi > f.zown0 ? zhi - f.zown0 : 1;
+  const int64_t tiles = cdiv(f.nx - WX + 1, Gm::TX) * cdiv(f.ny - WY + 1, Gm::TY);
+  // z-chunking: a block walks zc + WZ - 1 planes for zc window planes; blocks run in waves of
+  // `slots` (SMs x resident blocks).  Pick the chunk count that minimises waves x planes per
+  // block around the nominal chunk (equal chunks: the longest block walks as few planes as it
+  // can), e.g. C2: 3 chunks of 31 instead of 32 + 32 + 29.
+  static int occ = 0, sms = 0;
+  if (!occ) {
+    int d = 0;
+    cudaGetDevice(&d);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, d);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kP3Threads, Gm::smem) != cudaSuccess || occ < 1) occ = 1;
+  }
+  const int64_t slots = (int64_t)(sms > 0 ? sms : 148) * occ;
+  const int64_t n0 = cdiv(noz, p.zchunk);
+  int64_t best_n = n0, best_cost = INT64_MAX;
+  for (int64_t nch = n0 > 2 ? n0 - 2 : 1; nch <= n0 + 2 && nch <= noz; nch++) {
+    const int64_t zc = cdiv(noz, nch);
+    if (cdiv(noz, zc) != nch) continue;               // the same chunking as a smaller count
+    const int64_t cost = cdiv(tiles * nch, slots) * (zc + WZ - 1);
+    if (cost < best_cost) { best_cost = cost; best_n = nch; }
+  }
+  SsimParams q = p;
+  q.zchunk = (int)cdiv(noz, best_n);
+  dim3 grid((unsigned)cdiv(f.nx - WX + 1, Gm::TX), (unsigned)cdiv(f.ny - WY + 1, Gm::TY),
+            (unsigned)cdiv(noz, q.zchunk));
+  if (nblocks_out) { *nblocks_out = (int64_t)grid.x * grid.y * grid.z; return cudaSuccess; }
+  if (f.ny * f.nx >= (int64_t)1 << 31) return cudaErrorInvalidValue;   // 32-bit in-plane offsets
+  kern<<<grid, kP3Threads, Gm::smem, st>>>(f, q, parts, res, ticket, dbg);
   return cudaGetLastError();
 }
 
