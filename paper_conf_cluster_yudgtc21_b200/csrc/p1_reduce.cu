@@ -11,13 +11,13 @@
 
 namespace czc {
 
-// Per-thread accumulator: sums about the thread's first element (kx, ky, ke).  The element count
+// Per-thread accumulator: sums about the thread's first element (kx, ke).  The element count
 // is implicit (counted per vector), so no per-element work is spent on it.
 
 template <typename T>
 struct P1Acc {
-  double kx, ky, ke;
-  double sa, sb, sc, saa, sbb, sab, scc, sae;
+  double kx, ke;
+  double sa, sc, saa, sac, scc, sae;   // d_a = x - kx, d_c = e - ke (d_b = y - (kx + ke) = d_a + d_c)
   double emin, emax, pmin, pmax, spwr;
   double pthr_hi, pthr_lo;          // candidate thresholds for the exact pwr extrema
   unsigned npwr;                    // count of x != 0 (per thread, < 2^32)
@@ -26,8 +26,8 @@ struct P1Acc {
 
 template <typename T>
 __device__ __forceinline__ void acc_init(P1Acc<T>& a, T kxf, T kyf) {
-  a.kx = kxf; a.ky = kyf; a.ke = (double)kyf - (double)kxf;
-  a.sa = a.sb = a.sc = a.saa = a.sbb = a.sab = a.scc = a.sae = 0;
+  a.kx = kxf; a.ke = (double)kyf - (double)kxf;
+  a.sa = a.sc = a.saa = a.sac = a.scc = a.sae = 0;
   a.emin = dinf(); a.emax = -dinf(); a.pmin = dinf(); a.pmax = -dinf(); a.spwr = 0;
   a.pthr_hi = -dinf(); a.pthr_lo = dinf();
   a.npwr = 0;
@@ -51,11 +51,12 @@ template <typename T>
 __device__ __forceinline__ bool acc_elem(P1Acc<T>& a, T xf, T yf, double& ae_out, double& ax_out) {
   const double x = xf, y = yf;
   const double e = y - x;
-  const double da = x - a.kx, db = y - a.ky, dc = e - a.ke;
-  a.sa += da; a.sb += db; a.sc += dc;
+  // y - (kx + ke) = (x - kx) + (e - ke): the recon moments follow from d_a, d_c and their cross
+  // sum (6 accumulators instead of 8)
+  const double da = x - a.kx, dc = e - a.ke;
+  a.sa += da; a.sc += dc;
   a.saa = fma(da, da, a.saa);
-  a.sbb = fma(db, db, a.sbb);
-  a.sab = fma(da, db, a.sab);
+  a.sac = fma(da, dc, a.sac);
   a.scc = fma(dc, dc, a.scc);
   const double ae = fabs(e);
   a.sae += ae;
@@ -129,11 +130,12 @@ __device__ __forceinline__ P1State acc_to_state(const P1Acc<T>& a, double n) {
   if (n > 0) {
     s.n = n;
     s.mx = a.kx + a.sa / n;
-    s.my = a.ky + a.sb / n;
+    const double sb = a.sa + a.sc, sbb = a.saa + 2.0 * a.sac + a.scc, sab = a.saa + a.sac;
+    s.my = (a.kx + a.ke) + sb / n;
     s.me = a.ke + a.sc / n;
     s.m2x = a.saa - a.sa * (a.sa / n);
-    s.m2y = a.sbb - a.sb * (a.sb / n);
-    s.cxy = a.sab - a.sa * (a.sb / n);
+    s.m2y = sbb - sb * (sb / n);
+    s.cxy = sab - a.sa * (sb / n);
     s.m2e = a.scc - a.sc * (a.sc / n);
   }
   return s;
