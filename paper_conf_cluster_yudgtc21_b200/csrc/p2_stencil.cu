@@ -377,28 +377,29 @@ __device__ __forceinline__ void walk_line(Next next, int64_t lo, int64_t hi, int
 }
 
 // ---- TMA line walks (rows 16-byte aligned: nx % 4 == 0 and aligned segment bases) ------------
-// A block's 256 threads own 256 consecutive x of a line family (a row y for the z-walk, a plane z
-// for the y-walk) and walk positions i in [lo, end).  Thread 0 streams the contiguous row segment
-// of each position (<= 1 KB per field) into a ring of S = 2 TM shared-memory slots with one bulk
+// A block's 256 threads own CPT x 256 consecutive x of a row y (thread t: columns t, t + 256, ...)
+// and walk positions (planes) i in [lo, end).  Lanes of warp 0 stream the contiguous row segment
+// of each position (<= CPT KB per field) into a ring of S = 2 TM shared-memory slots with one bulk
 // copy per field, completing on the slot's mbarrier; after every TM positions the block
-// synchronises once and the consumed half of the ring is refilled S positions ahead.  Threads past
-// the row end read stale slot data; their products are discarded by walk_mask (lim = 0).
+// synchronises once and the consumed half of the ring is refilled S positions ahead.  Columns past
+// the row end read stale slot data; their products are discarded by walk_mask (lim = 0).  CPT = 2
+// halves the per-position cost of the waits and barriers per element (float32).
 constexpr int kWalkThreads = 256;
-template <typename T, int TM>
+template <typename T, int TM, int CPT>
 struct BulkWalkSmem {
   static constexpr int S = 2 * TM;
-  T x[S][kWalkThreads];
-  T y[S][kWalkThreads];
+  T x[S][CPT * kWalkThreads];
+  T y[S][CPT * kWalkThreads];
   uint64_t bar[S];
 };
 
 // RowPtr(i) -> (const T* xrow, const T* yrow) for position i (already offset to x0).
 // Positions are tracked relative to lo in 32 bits.  Lane v < S of warp 0 issues slot v's copies
 // (after the barrier that frees the slot), so the refill costs one bulk copy pair per lane.
-template <typename T, int TM, typename RowPtr>
-__device__ __forceinline__ void bulk_walk(BulkWalkSmem<T, TM>& sm, RowPtr row_ptr, uint32_t bytes, int64_t lo,
+template <typename T, int TM, int CPT, typename RowPtr>
+__device__ __forceinline__ void bulk_walk(BulkWalkSmem<T, TM, CPT>& sm, RowPtr row_ptr, uint32_t bytes, int64_t lo,
                                           int64_t hi, int64_t end, double mu,
-                                          double (&ring)[TM], double (&acc)[TM]) {
+                                          double (&ring)[CPT][TM], double (&acc)[CPT][TM]) {
   constexpr int S = 2 * TM;
   const int tid = threadIdx.x;
   const int jend = (int)(end - lo), jhi = (int)(hi - lo);
@@ -424,8 +425,12 @@ __device__ __forceinline__ void bulk_walk(BulkWalkSmem<T, TM>& sm, RowPtr row_pt
       const int j = j0 + u;
       if (j < jend) {                                  // block-uniform
         mbar_wait(&sm.bar[u], parity);
-        const double eps = ((double)sm.y[u][tid] - (double)sm.x[u][tid]) - mu;
-        walk_step<TM>(ring, acc, eps, j < jhi, u % TM);
+#pragma unroll
+        for (int c = 0; c < CPT; c++) {
+          const int col = tid + c * kWalkThreads;
+          const double eps = ((double)sm.y[u][col] - (double)sm.x[u][col]) - mu;
+          walk_step<TM>(ring[c], acc[c], eps, j < jhi, u % TM);
+        }
       }
       if (u == TM - 1 || u == S - 1) {                 // half of the ring consumed
         __syncthreads();
@@ -437,34 +442,43 @@ __device__ __forceinline__ void bulk_walk(BulkWalkSmem<T, TM>& sm, RowPtr row_pt
   }
 }
 
-// z-walk, TMA: block = 256 consecutive x of row y; grid (x tiles, ny, z chunks).
-template <typename E, int TM>
-__global__ void __launch_bounds__(kWalkThreads, 3)
+// z-walk, TMA: block = CPT x 256 consecutive x of row y; grid (x tiles, ny, z chunks).
+template <typename E, int TM, int CPT>
+__global__ void __launch_bounds__(kWalkThreads, CPT == 1 ? 3 : 2)
 ac_zwalk_tma(Field3<E> s, int T, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
              unsigned int* __restrict__ ticket) {
   extern __shared__ __align__(128) unsigned char walk_smem[];
-  BulkWalkSmem<E, TM>& sm = *reinterpret_cast<BulkWalkSmem<E, TM>*>(walk_smem);
-  const int64_t x0 = (int64_t)blockIdx.x * kWalkThreads, gy = blockIdx.y;
-  const int64_t gx = x0 + threadIdx.x;
+  BulkWalkSmem<E, TM, CPT>& sm = *reinterpret_cast<BulkWalkSmem<E, TM, CPT>*>(walk_smem);
+  const int64_t x0 = (int64_t)blockIdx.x * (CPT * kWalkThreads), gy = blockIdx.y;
   const double mu = res->p1g.me;
-  const bool own = gx < s.nx;
-  int64_t m = T;
-  if (s.ny > 1 && s.ny - 1 - gy < m) m = s.ny - 1 - gy;
-  if (s.nx > 1 && s.nx - 1 - gx < m) m = s.nx - 1 - gx;
+  int64_t mrow = T;
+  if (s.ny > 1 && s.ny - 1 - gy < mrow) mrow = s.ny - 1 - gy;
   const int64_t lo = s.zown0 + (int64_t)blockIdx.z * zchunk;
   int64_t hi = lo + zchunk;
   if (hi > s.zown1) hi = s.zown1;
   int64_t end = hi + T;
   if (end > s.nz) end = s.nz;
-  const int64_t ncols = (s.nx - x0) < kWalkThreads ? (s.nx - x0) : kWalkThreads;
+  const int64_t ncols = (s.nx - x0) < CPT * kWalkThreads ? (s.nx - x0) : CPT * kWalkThreads;
   const int64_t off = gy * s.nx + x0;
-  double ring[TM], acc[TM];
+  double ring[CPT][TM], acc[CPT][TM];
 #pragma unroll
-  for (int t = 0; t < TM; t++) ring[t] = acc[t] = 0;
-  bulk_walk<E, TM>(sm, [&](int64_t z, const E*& xr, const E*& yr) { xr = s.xp(z) + off; yr = s.yp(z) + off; },
-                   (uint32_t)(ncols * sizeof(E)), lo, hi, end, mu, ring, acc);
-  walk_mask<TM>(acc, own ? (int)m : 0);
-  ac_finish<TM>(acc, parts, res->rec.ac[0], ticket);
+  for (int c = 0; c < CPT; c++)
+#pragma unroll
+    for (int t = 0; t < TM; t++) ring[c][t] = acc[c][t] = 0;
+  bulk_walk<E, TM, CPT>(sm, [&](int64_t z, const E*& xr, const E*& yr) { xr = s.xp(z) + off; yr = s.yp(z) + off; },
+                        (uint32_t)(ncols * sizeof(E)), lo, hi, end, mu, ring, acc);
+  // per column: the R_tau bound from y and x (lim = 0 past the row end), then one sum
+#pragma unroll
+  for (int c = 0; c < CPT; c++) {
+    const int64_t gx = x0 + threadIdx.x + c * kWalkThreads;
+    int64_t m = mrow;
+    if (s.nx > 1 && s.nx - 1 - gx < m) m = s.nx - 1 - gx;
+    walk_mask<TM>(acc[c], gx < s.nx ? (int)m : 0);
+    if (c > 0)
+#pragma unroll
+      for (int t = 0; t < TM; t++) acc[0][t] += acc[c][t];
+  }
+  ac_finish<TM>(acc[0], parts, res->rec.ac[0], ticket);
 }
 
 // z-walk: thread <-> column (y, x); block 32 x 8 columns; grid.z chunks of owned planes.
@@ -885,6 +899,10 @@ cudaError_t launch_deriv(const Field3<T>& s0, int zchunk, double* parts, DevResu
 // Autocorrelation: the z-walk (3-D fields) and the in-plane tile kernel (x and y lags, ny > 1),
 // or the x-walk alone for 1-D fields; each launch has its own partial-buffer slice and ticket and
 // writes its own record slot (z -> ac[0], in-plane -> ac[1], x-walk -> ac[2]); the finish sums them.
+// columns per thread of the TMA z-walk: 2 for float32 (2 KB row segments), 1 for float64
+template <typename E>
+constexpr int kWalkCPT = sizeof(E) == 4 ? 2 : 1;
+
 struct AcGrids {
   dim3 z, zt, pl, x, xvec;
   bool rz, ry, rx;
@@ -894,14 +912,25 @@ template <typename E>
 static AcGrids ac_grids(const Field3<E>& s, int T) {
   AcGrids g{};
   const int64_t nzo = s.zown1 - s.zown0;
-  g.zc = 50; g.xc = 128;    // xc % 4 == 0 for the vector x-walk
+  g.xc = 128;                // xc % 4 == 0 for the vector x-walk
+  // z-walk chunks: long walks amortise the T halo planes every chunk re-reads (measured: 50 ->
+  // 100 -> 256 planes made the C3 walk 0.99 -> 0.91 -> 0.86 ms, and C2's 100 planes in one chunk
+  // beat two chunks of 50: 0.209 vs 0.226 ms); shorter only when the grid would not fill the 2
+  // resident blocks per SM once; equal chunks
+  {
+    const int64_t xy = cdiv(s.nx, kWalkCPT<E> * kWalkThreads) * s.ny;
+    int64_t zc = 256;
+    while (zc > 16 && xy * cdiv(nzo, zc) < 2 * (int64_t)sm_count()) zc /= 2;
+    zc = cdiv(nzo, cdiv(nzo, zc));
+    g.zc = (int)(zc > 0 ? zc : 1);
+  }
   g.rz = s.nz > 1; g.ry = s.ny > 1; g.rx = s.nx > 1;
   // persistent in-plane grid: the resident block count (3 per SM for TM <= 10, else 2)
   const int64_t W = cdiv(s.nx, kPlTX) * cdiv(s.ny, kPlTY) * nzo;
   const int64_t G = (int64_t)sm_count() * (T <= 10 ? 3 : 2);
   g.pzc = 0;
   g.z = dim3((unsigned)cdiv(s.nx, kTX), (unsigned)cdiv(s.ny, kTY), (unsigned)cdiv(nzo, g.zc));
-  g.zt = dim3((unsigned)cdiv(s.nx, kWalkThreads), (unsigned)s.ny, (unsigned)cdiv(nzo, g.zc));
+  g.zt = dim3((unsigned)cdiv(s.nx, kWalkCPT<E> * kWalkThreads), (unsigned)s.ny, (unsigned)cdiv(nzo, g.zc));
   g.pl = dim3((unsigned)(W < G ? W : G), 1, 1);
   g.x = dim3((unsigned)cdiv(nzo * s.ny, kXWarps * 32), (unsigned)cdiv(s.nx, g.xc), 1);
   g.xvec = dim3((unsigned)cdiv(nzo * s.ny, 256), (unsigned)cdiv(s.nx, g.xc), 1);
@@ -931,9 +960,10 @@ static cudaError_t launch_ac_t(const Field3<E>& s, int T, double* parts, DevResu
   cudaError_t e = cudaMemsetAsync(res->rec.ac, 0, sizeof(res->rec.ac), st);
   if (e != cudaSuccess) return e;
   if (g.rz && vec) {
-    constexpr int wsm = (int)sizeof(BulkWalkSmem<E, TM>);
-    if ((e = set_smem_once<ac_zwalk_tma<E, TM>>(wsm)) != cudaSuccess) return e;
-    ac_zwalk_tma<E, TM><<<g.zt, kWalkThreads, wsm, st>>>(s, T, g.zc, pz, res, tickets + 0);
+    constexpr int C = kWalkCPT<E>;
+    constexpr int wsm = (int)sizeof(BulkWalkSmem<E, TM, C>);
+    if ((e = set_smem_once<ac_zwalk_tma<E, TM, C>>(wsm)) != cudaSuccess) return e;
+    ac_zwalk_tma<E, TM, C><<<g.zt, kWalkThreads, wsm, st>>>(s, T, g.zc, pz, res, tickets + 0);
   } else if (g.rz) {
     ac_zwalk<E, TM><<<g.z, dim3(kTX, kTY), 0, st>>>(s, T, g.zc, pz, res, tickets + 0);
   }
