@@ -91,7 +91,7 @@ __device__ __forceinline__ T lane_window_ext(T v) {
 // T = float: the x ring and the exchanged extrema are floats (exact); T = double: doubles, one
 // block per SM for the larger register ring.
 template <typename T, int WX, int WY, int WZ, int G>
-__global__ void __launch_bounds__(kP3Threads, (SsimGeom<T, WX, WY, WZ, G>::KC * WZ * sizeof(T) <= 96) ? 2 : 1)
+__global__ void __launch_bounds__(kP3Threads, (kP3Warps <= 8 && SsimGeom<T, WX, WY, WZ, G>::KC * WZ * sizeof(T) <= 96) ? 2 : 1)
 p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __restrict__ res,
           unsigned int* __restrict__ ticket, double* __restrict__ dbg) {
   using Gm = SsimGeom<T, WX, WY, WZ, G>;
@@ -132,10 +132,14 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
   if (nsteps > 0) { cin.init(f, zb); cold.init(f, zb); }
   Pair<T> nxt[KC];                                       // prefetched next plane
   T nyo[KC];                                             // ... and its leaving y sample
+  // footprint row warp + kP3Warps k exists (r < FY); warp-uniform, and constant for every k but
+  // the last, so rows past the footprint cost nothing
+  auto row_live = [&](const int k) { return kP3Warps * (k + 1) <= FY || warp + kP3Warps * k < FY; };
   auto load = [&](int n, bool has_old) {                 // has_old: n >= WZ (constant per call site)
     if (n < nsteps) {                                    // block-uniform
 #pragma unroll
       for (int k = 0; k < KC; k++) {
+        if (!row_live(k)) continue;
         nxt[k].x = __ldg(cin.x + off[k]);
         nxt[k].y = __ldg(cin.y + off[k]);
         nyo[k] = has_old ? __ldg(cold.y + off[k]) : (T)0;
@@ -183,6 +187,7 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
     // ---- (a) z-walk --------------------------------------------------------------------
 #pragma unroll
     for (int k = 0; k < KC; k++) {
+      if (!row_live(k)) continue;
       {
         const double xd = nxt[k].x, yd = nxt[k].y;
         const double a = xd - K, b = yd - K, e = yd - xd;
@@ -195,7 +200,7 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
       }
       ring[k][s] = nxt[k].x;
       const int r = warp + kP3Warps * k;
-      if (full && (kP3Warps * (k + 1) <= FY || r < FY)) {
+      if (full) {
         T mn = ring[k][0], mx = ring[k][0];
 #pragma unroll
         for (int t = 1; t < WZ; t++) { mn = tmin(mn, ring[k][t]); mx = tmax(mx, ring[k][t]); }
