@@ -252,6 +252,21 @@ def run_ours(args, rank, world, local):
     shares = {name: statistics.mean(k[i] for k in kms)
               for i, name in enumerate(("P1", "P2_deriv", "P2_autocorr", "P3_ssim"))}
     dom = max(shares, key=shares.get)
+    # secondary ceiling: every pattern is FP64-arithmetic / issue bound, so the
+    # algorithmic FP64 operations of the method (per element / interior point /
+    # window) are also set against the FP64 pipe rate measured on this GPU model
+    # (profiles/r01_pipes2.txt: DFMA 61.6 lanes/clk/SM; 148 SMs at 1.965 GHz)
+    fp64_peak = 61.6 * 148 * 1.965                     # G FP64 instructions / s
+    units = {"P1": (12, int(r["n"]), "element: e, 6 moment sums, |e| sum, 2 extrema, pwr quotient + sum"),
+             "P2_deriv": (74, int(r["n_interior"]), "interior point: 2 x 22 stencil ops, 2 sqrt, 5 x 6 statistics"),
+             "P2_autocorr": (31, int(r["n"]), "element: eps, 10 lags x 3 axes FMAs"),
+             "P3_ssim": (42, int(r["n_windows"]), "window: 24 running-sum adds, 2 products, 16 mix ops")}
+    fp64 = {}
+    for k, (ops, n_units, what) in units.items():
+        if shares.get(k, 0) > 0:
+            a_g = ops * n_units / world / (shares[k] * 1e-3) / 1e9    # per GPU (units are global)
+            fp64[k] = {"achieved": round(a_g, 1), "frac": round(a_g / fp64_peak, 4), "ops_per_unit": ops,
+                       "units_per_launch": n_units, "unit": what}
     peak, peak_src = measured_peak()
     alg_bytes = nbytes_rank                              # each pattern reads the pair once (+ halos)
     achieved = alg_bytes / (shares[dom] * 1e-3) / 1e9
@@ -347,6 +362,10 @@ def run_ours(args, rank, world, local):
                          "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
                          "peak_source": peak_src, "traffic_source": traffic_src,
                          "algorithmic_bytes_per_launch": alg_bytes},
+            "roofline_fp64": {"bound": "alu", "kernel": dom, "achieved": fp64[dom]["achieved"],
+                              "peak": round(fp64_peak, 1), "unit": "G FP64 ops/s", "frac": fp64[dom]["frac"],
+                              "peak_source": "measured DFMA issue rate (profiles/r01_pipes2.txt) x 148 SMs x 1.965 GHz",
+                              "per_pattern": fp64},
             "cpu_baseline": cpu, "e2e": e2e, "float64_inputs": f64,
             "gpu_launches": launches_per_step * args.steps,
             "clocks": clocks, "wall_s_timed_region": round(t_wall, 4),

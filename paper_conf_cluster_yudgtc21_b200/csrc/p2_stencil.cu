@@ -807,21 +807,26 @@ ac_plane(Field3<T> s, double* __restrict__ parts, DevResults* __restrict__ res, 
       cp_async_wait_all();
       __syncthreads();                     // plane z staged; previous walks done with sm.e
       {
-        // all 16-byte groups of the staged window, 256 at a time (row r, group g of the row)
-        int r = r0, g = g0;
-        for (int i = tid; i < HY * NV; i += kPlThreads) {
-          const Vec16<T> a = *reinterpret_cast<const Vec16<T>*>(&sm.fx[r][EPG * g]);
-          const Vec16<T> b = *reinterpret_cast<const Vec16<T>*>(&sm.fy[r][EPG * g]);
-          double* er = &sm.e[r][EPG * g];
+        // all 16-byte groups of the staged window, 256 at a time (row r, group g of the row);
+        // tiles away from the field ends (xy_inner, block-uniform) need no zero fill
+        auto convert = [&](const bool inner) {
+          int r = r0, g = g0;
+          for (int i = tid; i < HY * NV; i += kPlThreads) {
+            const Vec16<T> a = *reinterpret_cast<const Vec16<T>*>(&sm.fx[r][EPG * g]);
+            const Vec16<T> b = *reinterpret_cast<const Vec16<T>*>(&sm.fy[r][EPG * g]);
+            double* er = &sm.e[r][EPG * g];
 #pragma unroll
-          for (int j = 0; j < EPG; j++) {
-            const double ej = ((double)b.e[j] - (double)a.e[j]) - mu;
-            er[j] = (xy_inner || (r < rv && EPG * g + j < cv)) ? ej : 0.0;
+            for (int j = 0; j < EPG; j++) {
+              const double ej = ((double)b.e[j] - (double)a.e[j]) - mu;
+              er[j] = (inner || (r < rv && EPG * g + j < cv)) ? ej : 0.0;
+            }
+            r += kPlThreads / NV;
+            g += kPlThreads % NV;
+            if (g >= NV) { g -= NV; r++; }
           }
-          r += kPlThreads / NV;
-          g += kPlThreads % NV;
-          if (g >= NV) { g -= NV; r++; }
-        }
+        };
+        if (xy_inner) convert(true);
+        else convert(false);
       }
       __syncthreads();                     // eps ready, staging buffer free
       if (z + 1 < ze) {
