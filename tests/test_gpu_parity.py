@@ -685,3 +685,23 @@ def test_4d_squeezed_and_unsupported(czc, orc):
         with pytest.raises(czc.CzcError) as ei:
             a.assess(x4, x4)
         assert ei.value.status == 7
+
+
+def test_graph_replay_sees_new_contents_and_plans(czc, orc):
+    """The single-GPU sequence replays as a CUDA graph while the call signature repeats: new
+    contents in the same buffers must be read, and a different mask / window (new signature)
+    must re-capture, then returning to the first signature must be right again."""
+    x, y = synth.make_pair(synth.config("C2", dims=(20, 40, 48)))
+    xd, yd = x.cuda(), y.cuda()
+    with czc.Assessor(ssim_window=5) as a:
+        for it in range(3):
+            if it:
+                yd.copy_(xd + (yd - xd) * (1.0 + it))             # same buffers, new contents
+            g = a.assess(xd, yd)
+            xn, yn = xd.cpu().numpy(), yd.cpu().numpy()
+            errors = []
+            check_p1(g, orc.p1(xn, yn), errors)
+            check_ssim(g["ssim"], g["n_windows"], *orc.ssim(xn, yn, [5] * 3), errors)
+            report(errors)
+            gp = a.assess(xd, yd, czc.M_P1 | czc.M_PDF)           # another signature in between
+            assert gp["computed_mask"] == czc.M_P1 | czc.M_PDF and gp["mse"] == g["mse"]
