@@ -280,9 +280,9 @@ def run_ours(args, rank, world, local):
     # end-to-end through the public host-buffer entry point (H2D + kernels + D2H inside)
     e2e = None
     if not args.no_e2e:
-        # czc_assess_host pipelines K = min(8, nz / halo) z-chunks (halo = max(1, T, W - 1) = 10)
-        # and copies back one record prefix per chunk (czc_sizeof(4) bytes each)
-        K = min(8, nz_local // 10) if world == 1 else world
+        # czc_assess_host pipelines K = min(8, nz / 4) z-chunks and copies back one record
+        # prefix per chunk (czc_sizeof(4) bytes each)
+        K = min(8, nz_local // 4) if world == 1 else world
         d2h_host = int(czc.get_lib().czc_sizeof(4)) * (K if K >= 2 else 1)
         xp = xh.pin_memory()
         yp = yh.pin_memory()

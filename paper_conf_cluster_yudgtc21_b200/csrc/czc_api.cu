@@ -58,6 +58,7 @@ cudaError_t launch_ssim4(const E* x, const E* y, const int64_t n[4], const int w
 using namespace czc;
 
 static constexpr int kMaxHostChunks = 16;   // z-chunks of the pipelined czc_assess_host
+static constexpr int kHostChunks = 8;       // default chunk count
 
 struct czc_ctx {
   czc_config cfg;
@@ -874,7 +875,6 @@ static czc_status assess_host_pipelined(czc_ctx* ctx, const Plan& P, const E* hx
   }
   std::vector<int64_t> b(K + 1);
   for (int k = 0; k <= K; k++) b[k] = nz * k / K;
-  const int64_t H = halo_depth(P);
   // the copy streams start after everything already queued on the compute stream (which may
   // still read the device buffers of the previous call)
   CZC_CUDA(ctx, cudaEventRecord(ctx->copy_ev[0][0], s));
@@ -885,12 +885,6 @@ static czc_status assess_host_pipelined(czc_ctx* ctx, const Plan& P, const E* hx
     CZC_CUDA(ctx, cudaMemcpyAsync(y + b[k] * plane, hy + b[k] * plane, bytes, cudaMemcpyHostToDevice, ctx->copy_stream[0]));
     CZC_CUDA(ctx, cudaEventRecord(ctx->copy_ev[0][k], ctx->copy_stream[0]));
   }
-  // index of the last chunk that must be resident before chunk k's stencils / windows can run
-  auto ready_for = [&](int k) {
-    int j = k;
-    while (j + 1 < K && b[j + 1] < std::min(nz, b[k + 1] + H)) j++;
-    return j;
-  };
   Field3<E> F{};
   F.nz = nz; F.ny = P.g3[1]; F.nx = P.g3[2];
   F.nseg = 1; F.xs[0] = x; F.ys[0] = y; F.zs[0] = 0; F.zs[1] = nz;
@@ -898,30 +892,43 @@ static czc_status assess_host_pipelined(czc_ctx* ctx, const Plan& P, const E* hx
   Record* drec = (Record*)ctx->dgather;
   P1State* dst = (P1State*)ctx->dstates;
   CZC_CUDA(ctx, cudaMemsetAsync(drec, 0, (size_t)K * sizeof(Record), s));
-  Plan P23 = P;                                       // per chunk: derivatives + SSIM only
-  P23.run_ac = false;
+  // Per arrived chunk k (planes < b[k+1] resident): P1 of the chunk, then the derivative points
+  // and SSIM window origins whose whole stencil / window is resident — owned ranges
+  // [done, b[k+1] - 1) and [done, b[k+1] - W + 1) (the whole rest for the last chunk), so no
+  // chunk waits for the next one and only the last chunk's share runs after the last copy.
+  Plan Pd = P, Ps = P;
+  Pd.run_ac = Pd.run_ssim = false;
+  Ps.run_ac = Ps.run_deriv = false;
+  int64_t d_done = 0, s_done = 0;
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
-  int waited = -1;
   for (int k = 0; k < K; k++) {
-    const int need = (P.run_deriv || P.run_ssim) ? ready_for(k) : k;
-    for (int j = waited + 1; j <= need; j++) CZC_CUDA(ctx, cudaStreamWaitEvent(s, ctx->copy_ev[0][j], 0));
-    waited = std::max(waited, need);
+    CZC_CUDA(ctx, cudaStreamWaitEvent(s, ctx->copy_ev[0][k], 0));
+    const bool last = k == K - 1;
     if (P.run_p1) {
       czc_status st = p1_local(ctx, P, x + b[k] * plane, y + b[k] * plane, (b[k + 1] - b[k]) * plane);
       if (st != CZC_OK) return st;
       CZC_CUDA(ctx, cudaMemcpyAsync(dst + k, &ctx->dres->rec.p1, sizeof(P1State), cudaMemcpyDeviceToDevice, s));
       CZC_CUDA(ctx, cudaMemcpyAsync(&drec[k].p1, &ctx->dres->rec.p1, sizeof(P1State), cudaMemcpyDeviceToDevice, s));
     }
-    if (P.run_deriv || P.run_ssim) {
-      F.zown0 = b[k];
-      F.zown1 = b[k + 1];
-      czc_status st = run_p23(ctx, P23, F, sp);
+    if (P.run_deriv) {                                 // possibly empty: the record then holds identities
+      const int64_t hi = std::max(d_done, last ? nz : b[k + 1] - 1);
+      F.zown0 = d_done;
+      F.zown1 = hi;
+      czc_status st = run_p23(ctx, Pd, F, sp);
       if (st != CZC_OK) return st;
       CZC_CUDA(ctx, cudaMemcpyAsync(drec[k].deriv, ctx->dres->rec.deriv, sizeof(drec[k].deriv), cudaMemcpyDeviceToDevice, s));
+      d_done = hi;
+    }
+    if (P.run_ssim) {
+      const int64_t hi = std::max(s_done, last ? nz : b[k + 1] - (P.W - 1));
+      F.zown0 = s_done;
+      F.zown1 = hi;
+      czc_status st = run_p23(ctx, Ps, F, sp);
+      if (st != CZC_OK) return st;
       CZC_CUDA(ctx, cudaMemcpyAsync(drec[k].ssim, ctx->dres->rec.ssim, sizeof(drec[k].ssim), cudaMemcpyDeviceToDevice, s));
+      s_done = hi;
     }
   }
-  for (int j = waited + 1; j < K; j++) CZC_CUDA(ctx, cudaStreamWaitEvent(s, ctx->copy_ev[0][j], 0));
   if (P.run_p1) CZC_CUDA(ctx, launch_p1_combine(dst, K, ctx->dres, s));
   if (P.run_pdf) {
     CZC_CUDA(ctx, launch_pdf(x, y, nz * plane, P.nb, ctx->p1_grid_cap, ctx->dres, s));
@@ -975,8 +982,10 @@ extern "C" czc_status czc_assess_host(czc_ctx* ctx, const void* orig, const void
                      make_plan(ctx->cfg, shape->ndim, shape->dims, metric_mask, P, why) == CZC_OK && P.D == 3 &&
                      (shape->nz_local == 0 || shape->nz_local == shape->dims[0]);
   if (plain) {
-    const int64_t H = std::max<int64_t>(halo_depth(P), 1);
-    const int K = (int)std::min<int64_t>(std::min<int64_t>(8, kMaxHostChunks), P.g3[0] / H);
+    // chunks of >= 4 planes, at most kHostChunks (CZC_HOST_CHUNKS overrides: A/B timing only)
+    int kc = kHostChunks;
+    if (const char* e = getenv("CZC_HOST_CHUNKS")) kc = std::max(2, std::min(kMaxHostChunks, atoi(e)));
+    const int K = (int)std::min<int64_t>(kc, P.g3[0] / 4);
     if (K >= 2) {
       st = dtype == CZC_F64
                ? assess_host_pipelined(ctx, P, (const double*)orig, (const double*)recon, out, metric_mask, K)
