@@ -232,7 +232,12 @@ def run_ours(args, rank, world, local):
     barrier()
     t_wall = time.perf_counter() - t_wall
     clocks = sampler.stop()
-    with czc.Assessor(ndim=3, device=local, stream=stream, timing=True, **cfg) as at:
+    cfg_t = dict(cfg)
+    if world > 1:                       # a second communicator needs its own ncclUniqueId
+        obj = [czc_nccl_uid() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        cfg_t["nccl_uid"] = obj[0]
+    with czc.Assessor(ndim=3, device=local, stream=stream, timing=True, **cfg_t) as at:
         for i in range(args.warmup + args.steps):
             flush.zero_()
             clean.sum()
