@@ -91,7 +91,7 @@ __device__ __forceinline__ T lane_window_ext(T v) {
 // T = float: the x ring and the exchanged extrema are floats (exact); T = double: doubles, one
 // block per SM for the larger register ring.
 template <typename T, int WX, int WY, int WZ, int G>
-__global__ void __launch_bounds__(kP3Threads, (kP3Warps <= 8 && SsimGeom<T, WX, WY, WZ, G>::KC * WZ * sizeof(T) <= 96) ? 2 : 1)
+__global__ void __launch_bounds__(kP3Threads, (kP3Warps <= 8 && SsimGeom<T, WX, WY, WZ, G>::KC * WZ * sizeof(T) <= 128) ? 2 : 1)
 p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __restrict__ res,
           unsigned int* __restrict__ ticket, double* __restrict__ dbg) {
   using Gm = SsimGeom<T, WX, WY, WZ, G>;
@@ -361,7 +361,9 @@ static cudaError_t launch_t(const Field3<T>& f, const SsimParams& p, double* par
 template <typename T, int W>
 static cudaError_t dispatch_w(int kind, const Field3<T>& f, const SsimParams& p, double* parts,
                               DevResults* res, unsigned int* ticket, double* dbg, cudaStream_t st, int64_t* nb) {
-  constexpr int G = W <= 8 ? 2 : 1;                     // keep the z-walk state in registers
+  // keep the z-walk state in registers: float rows of a 2-row origin tile (W <= 8), one origin
+  // row per warp otherwise and for double rings (2 blocks per SM instead of 1)
+  constexpr int G = (W <= 8 && sizeof(T) == 4) ? 2 : 1;
   if (kind == 3) return launch_t<T, W, W, W, G>(f, p, parts, res, ticket, dbg, st, nb);
   if (kind == 2) return launch_t<T, W, W, 1, 2>(f, p, parts, res, ticket, dbg, st, nb);
   return launch_t<T, W, 1, 1, 1>(f, p, parts, res, ticket, dbg, st, nb);
