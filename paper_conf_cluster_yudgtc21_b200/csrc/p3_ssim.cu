@@ -357,6 +357,134 @@ static cudaError_t launch_t(const Field3<T>& f, const SsimParams& p, double* par
   return cudaGetLastError();
 }
 
+// ------------------------------------------------------------------------------------------------
+// 2-D fields (square W x W windows): the rows stream like the planes of the 3-D kernel, and the
+// y-window is the running sum of that stream, so no shared-memory exchange and no barrier are
+// needed: warp w of a block owns its own tile of 32 - W + 1 x-origins (lane = footprint column),
+// keeps FP64 running sums of the four anchored moments over the last W rows plus the rows' x in
+// a register ring (static rotation, warm-up peeled), re-reads the leaving row's y from L2, and
+// per row does the x-pass by shuffles and the mix.  (The 3-D kernel on a one-plane field ran one
+// plane per block: 0.29 ms for the 1800 x 3600 CESM-shaped pair.)
+constexpr int kRowWarps = 8;
+template <typename T, int W>
+__global__ void __launch_bounds__(kRowWarps * 32)
+p3_rows_kernel(Field3<T> f, SsimParams p, int rchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+               unsigned int* __restrict__ ticket, double* __restrict__ dbg) {
+  constexpr int TX = 32 - W + 1;
+  constexpr double invM = 1.0 / (double)(W * W);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t ny = f.ny, nx = f.nx;
+  const T* __restrict__ X = f.xp(0);
+  const T* __restrict__ Y = f.yp(0);
+  const int64_t x0 = ((int64_t)blockIdx.x * kRowWarps + warp) * TX;
+  const int64_t gx = x0 + lane, gxc = gx < nx ? gx : nx - 1;   // clamped columns feed masked windows only
+  const int64_t rb = (int64_t)blockIdx.y * rchunk;
+  int64_t ro_end = rb + rchunk;                                 // origin rows [rb, ro_end)
+  if (ro_end > ny - W + 1) ro_end = ny - W + 1;
+  const int nsteps = ro_end > rb ? (int)(ro_end + W - 1 - rb) : 0;
+  const int64_t kx = x0 + 16 < nx ? x0 + 16 : nx - 1, ky = rb + W / 2 < ny ? rb + W / 2 : ny - 1;
+  const double K = (double)X[ky * nx + kx];                     // anchor of this warp's tile
+  const double Lglob = res->p1g.xmax - res->p1g.xmin;
+  const bool range_global = p.range_mode != 0;
+  const bool xok = lane < TX && gx <= nx - W && (gx % p.sx) == 0;
+  const T* px = X + rb * nx + gxc;                              // row cursor (next row to load)
+  const T* py = Y + rb * nx + gxc;
+  const T* pyo = py;                                            // row leaving the window
+  T nx_ = 0, ny_ = 0, nyo = 0;
+  auto load = [&](int n, bool has_old) {
+    if (n < nsteps) {
+      nx_ = __ldg(px); ny_ = __ldg(py); px += nx; py += nx;
+      if (has_old) { nyo = __ldg(pyo); pyo += nx; }
+    }
+  };
+  double sm0 = 0, sm1 = 0, sm2 = 0, sm3 = 0;
+  T ring[W];
+#pragma unroll
+  for (int t = 0; t < W; t++) ring[t] = 0;
+  double ssum = 0;
+  unsigned scnt = 0;
+  int rph = (int)(rb % p.sy);
+  load(0, false);
+  auto step_body = [&](const int step, const int s, const bool warm) {
+    const bool full = warm || s == W - 1;
+    {
+      const double xd = nx_, yd = ny_;
+      const double a = xd - K, b = yd - K, e = yd - xd;
+      sm0 += a; sm1 += e; sm2 = fma(a, b, sm2); sm3 = fma(e, e, sm3);
+    }
+    if (warm) {
+      const double xd = ring[s], yd = nyo;
+      const double a = xd - K, b = yd - K, e = yd - xd;
+      sm0 -= a; sm1 -= e; sm2 = fma(-a, b, sm2); sm3 = fma(-e, e, sm3);
+    }
+    ring[s] = nx_;
+    load(step + 1, warm || s == W - 1);
+    if (!full) return;
+    T mn = ring[0], mx = ring[0];
+#pragma unroll
+    for (int t = 1; t < W; t++) { mn = tmin(mn, ring[t]); mx = tmax(mx, ring[t]); }
+    const double S0 = lane_window_sum<W>(sm0), S1 = lane_window_sum<W>(sm1);
+    const double S2 = lane_window_sum<W>(sm2), S3 = lane_window_sum<W>(sm3);
+    const T wmn = lane_window_ext<W, false>(mn), wmx = lane_window_ext<W, true>(mx);
+    const bool ok = xok && rph == 0;                            // origin row rb + step - W + 1
+    rph = rph + 1 == p.sy ? 0 : rph + 1;
+    const double mua = S0 * invM, mue = S1 * invM;
+    const double mux = K + mua, muy = mux + mue;
+    const double sxy = S2 * invM - mua * (mua + mue);
+    const double see = S3 * invM - mue * mue;
+    double L = range_global ? Lglob : (double)wmx - (double)wmn;
+    L = (L == 0.0) ? 1.0 : L;
+    const double C1 = (0.01 * L) * (0.01 * L), C2 = (0.03 * L) * (0.03 * L);
+    const double A = 2.0 * mux * muy + C1, B = 2.0 * sxy + C2;
+    const double ssim = (A * B) * fast_rcp((A + mue * mue) * (B + see));
+    ssum += ok ? ssim : 0.0;
+    scnt += ok ? 1u : 0u;
+    if (dbg && ok) dbg[((rb + step - W + 1) / p.sy) * p.nwx + gx / p.sx] = ssim;
+  };
+#pragma unroll
+  for (int s = 0; s < W; s++) {
+    if (s >= nsteps) break;                                     // block-uniform
+    step_body(s, s, false);
+  }
+  for (int s0 = W; s0 < nsteps; s0 += W) {
+#pragma unroll
+    for (int s = 0; s < W; s++) {
+      if (s0 + s >= nsteps) break;
+      step_body(s0 + s, s, true);
+    }
+  }
+  double rec[kSsimSlots] = {ssum, (double)scnt, 0.0};
+  struct Sum { __device__ int operator()(int) const { return OP_SUM; } };
+  const unsigned bid = blockIdx.x + gridDim.x * blockIdx.y;
+  block_reduce_slots<kSsimSlots>(rec, Sum{}, parts + (size_t)bid * kSsimSlots);
+  if (!last_block_arrive(ticket)) return;
+  finish_slots<kSsimSlots>(parts, gridDim.x * gridDim.y, Sum{}, res->rec.ssim);
+  if (threadIdx.x == 0) *ticket = 0;
+}
+
+template <typename T, int W>
+static cudaError_t launch_rows(const Field3<T>& f, const SsimParams& p, double* parts, DevResults* res,
+                               unsigned int* ticket, double* dbg, cudaStream_t st, int64_t* nblocks_out) {
+  constexpr int TX = 32 - W + 1;
+  const int64_t tiles = cdiv(f.nx - W + 1, TX), bx = cdiv(tiles, kRowWarps);
+  const int64_t nro = f.ny - W + 1 > 0 ? f.ny - W + 1 : 1;
+  // row chunks: as long as possible (each chunk re-reads W - 1 rows) while the grid still fills
+  // about four blocks per SM
+  int64_t rc = nro;
+  int sms = 148;
+  {
+    int d = 0;
+    cudaGetDevice(&d);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, d);
+  }
+  while (rc > 4 * W && bx * cdiv(nro, rc) < 4 * (int64_t)sms) rc = cdiv(rc, 2);
+  rc = cdiv(nro, cdiv(nro, rc));
+  const dim3 grid((unsigned)bx, (unsigned)cdiv(nro, rc), 1);
+  if (nblocks_out) { *nblocks_out = (int64_t)grid.x * grid.y; return cudaSuccess; }
+  p3_rows_kernel<T, W><<<grid, kRowWarps * 32, 0, st>>>(f, p, (int)rc, parts, res, ticket, dbg);
+  return cudaGetLastError();
+}
+
 // kind 3: cubic window (3-D); 2: square window, z inactive (2-D); 1: x only (1-D).
 template <typename T, int W>
 static cudaError_t dispatch_w(int kind, const Field3<T>& f, const SsimParams& p, double* parts,
@@ -365,7 +493,7 @@ static cudaError_t dispatch_w(int kind, const Field3<T>& f, const SsimParams& p,
   // row per warp otherwise and for double rings (2 blocks per SM instead of 1)
   constexpr int G = (W <= 8 && sizeof(T) == 4) ? 2 : 1;
   if (kind == 3) return launch_t<T, W, W, W, G>(f, p, parts, res, ticket, dbg, st, nb);
-  if (kind == 2) return launch_t<T, W, W, 1, 2>(f, p, parts, res, ticket, dbg, st, nb);
+  if (kind == 2) return launch_rows<T, W>(f, p, parts, res, ticket, dbg, st, nb);
   return launch_t<T, W, 1, 1, 1>(f, p, parts, res, ticket, dbg, st, nb);
 }
 
