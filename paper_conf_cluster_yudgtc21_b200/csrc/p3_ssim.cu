@@ -13,8 +13,8 @@
 //   (a) z-walk — keeps FP64 running sums over the last WZ planes of four anchored moments
 //         a = x - K,  e = y - x,  a*b (b = y - K),  e*e
 //       in registers; the leaving plane's x sits in a per-thread register ring (the paper's
-//       FIFO, moved from window partials to raw samples; the ring rotates statically because
-//       the plane loop is unrolled by WZ), which also gives the z-window min/max of x, and its
+//       FIFO, moved from window partials to raw samples; a shifting ring, so the plane loop
+//       needs no unrolling), which also gives the z-window min/max of x, and its
 //       y is re-read from L2; the next plane is prefetched into registers one plane ahead;
 //   (b) y-pass — after ONE __syncthreads on a double-buffered shared-memory exchange of the
 //       z-sums, each warp forms running sums over WY rows for its G origin rows;
@@ -174,9 +174,9 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
   }
   int zph = (int)(zb % p.sz);                            // phase of origin plane zb
 
-  // One plane step; s = step mod WZ (the ring slot) and warm = (step >= WZ: a plane leaves the
-  // z-window) are compile-time constants at every call site, so the ring rotates statically and
-  // the warm-up planes carry no per-step tests.
+  // One plane step; warm = (step >= WZ: a plane leaves the z-window) and, in the warm-up, s =
+  // step are compile-time constants at every call site, so the warm-up planes carry no per-step
+  // tests.
   auto step_body = [&](const int step, const int s, const bool warm) {
     // the prefetched plane is consumed by the z-walk below, then the next one is requested
     // into the same registers (no copies; its latency hides behind the y / x passes)
@@ -194,11 +194,17 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
         sm[k][0] += a; sm[k][1] += e; sm[k][2] = fma(a, b, sm[k][2]); sm[k][3] = fma(e, e, sm[k][3]);
       }
       if (warm) {
-        const double xd = ring[k][s], yd = nyo[k];
+        const double xd = ring[k][0], yd = nyo[k];
         const double a = xd - K, b = yd - K, e = yd - xd;
         sm[k][0] -= a; sm[k][1] -= e; sm[k][2] = fma(-a, b, sm[k][2]); sm[k][3] = fma(-e, e, sm[k][3]);
       }
-      ring[k][s] = nxt[k].x;
+      // shifting ring (oldest plane first; WZ - 1 register moves per row): the main loop is not
+      // unrolled, so one copy of the step (~4.4 K instructions for the kernel instead of 10.3 K
+      // with a static-slot ring unrolled by WZ) stays in the instruction cache — the
+      // `no_instruction` stalls of the unrolled version cost more than the moves (0.475 -> 0.445 ms)
+#pragma unroll
+      for (int t = 0; t + 1 < WZ; t++) ring[k][t] = ring[k][t + 1];
+      ring[k][WZ - 1] = nxt[k].x;
       const int r = warp + kP3Warps * k;
       if (full) {
         T mn = ring[k][0], mx = ring[k][0];
@@ -295,14 +301,8 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
     if (s >= nsteps) break;                              // block-uniform
     step_body(s, s, false);
   }
-  for (int s0 = WZ; s0 < nsteps; s0 += WZ) {
-#pragma unroll
-    for (int s = 0; s < WZ; s++) {
-      const int step = s0 + s;                           // == s (mod WZ)
-      if (step >= nsteps) break;                         // block-uniform
-      step_body(step, s, true);
-    }
-  }
+#pragma unroll 1
+  for (int step = WZ; step < nsteps; step++) step_body(step, 0, true);
 
   double rec[kSsimSlots] = {ssum, (double)scnt, 0.0};
   const unsigned bid = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
