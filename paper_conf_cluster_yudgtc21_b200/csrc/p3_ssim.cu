@@ -362,7 +362,7 @@ static cudaError_t launch_t(const Field3<T>& f, const SsimParams& p, double* par
 // y-window is the running sum of that stream, so no shared-memory exchange and no barrier are
 // needed: warp w of a block owns its own tile of 32 - W + 1 x-origins (lane = footprint column),
 // keeps FP64 running sums of the four anchored moments over the last W rows plus the rows' x in
-// a register ring (static rotation, warm-up peeled), re-reads the leaving row's y from L2, and
+// a shifting register ring (warm-up peeled), re-reads the leaving row's y from L2, and
 // per row does the x-pass by shuffles and the mix.  (The 3-D kernel on a one-plane field ran one
 // plane per block: 0.29 ms for the 1800 x 3600 CESM-shaped pair.)
 constexpr int kRowWarps = 8;
@@ -413,11 +413,13 @@ p3_rows_kernel(Field3<T> f, SsimParams p, int rchunk, double* __restrict__ parts
       sm0 += a; sm1 += e; sm2 = fma(a, b, sm2); sm3 = fma(e, e, sm3);
     }
     if (warm) {
-      const double xd = ring[s], yd = nyo;
+      const double xd = ring[0], yd = nyo;
       const double a = xd - K, b = yd - K, e = yd - xd;
       sm0 -= a; sm1 -= e; sm2 = fma(-a, b, sm2); sm3 = fma(-e, e, sm3);
     }
-    ring[s] = nx_;
+#pragma unroll
+    for (int t = 0; t + 1 < W; t++) ring[t] = ring[t + 1];     // shifting ring, oldest first
+    ring[W - 1] = nx_;
     load(step + 1, warm || s == W - 1);
     if (!full) return;
     T mn = ring[0], mx = ring[0];
@@ -446,13 +448,8 @@ p3_rows_kernel(Field3<T> f, SsimParams p, int rchunk, double* __restrict__ parts
     if (s >= nsteps) break;                                     // block-uniform
     step_body(s, s, false);
   }
-  for (int s0 = W; s0 < nsteps; s0 += W) {
-#pragma unroll
-    for (int s = 0; s < W; s++) {
-      if (s0 + s >= nsteps) break;
-      step_body(s0 + s, s, true);
-    }
-  }
+#pragma unroll 1
+  for (int step = W; step < nsteps; step++) step_body(step, 0, true);
   double rec[kSsimSlots] = {ssum, (double)scnt, 0.0};
   struct Sum { __device__ int operator()(int) const { return OP_SUM; } };
   const unsigned bid = blockIdx.x + gridDim.x * blockIdx.y;
