@@ -97,8 +97,8 @@ struct SumOp {
 };
 
 // grid: (ceil(nx/BX), ceil(ny/BY), zchunks); block (BX, BY), BX * BY = 256.
-//   3-D: <true, true, 32, 8>; 2-D row view (slow axis = rows): <true, false, 256, 1>;
-//   1-D: <false, false, 256, 1>.
+//   3-D fields with nz <= 2: <true, true, 32, 8>; 1-D: <false, false, 256, 1> (3-D fields use
+//   deriv3_kernel, 2-D row views deriv2_kernel).
 template <typename T, bool ZA, bool YA, int BX, int BY>
 __global__ void __launch_bounds__(BX * BY, 2)
 deriv_kernel(Field3<T> s, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
@@ -186,6 +186,77 @@ deriv_kernel(Field3<T> s, int zchunk, double* __restrict__ parts, DevResults* __
   if (!last_block_arrive(ticket)) return;
   finish_slots<kDerivSlots>(parts, gridDim.x * gridDim.y * gridDim.z, DerivOp{}, res->rec.deriv);
   if (tid == 0) *ticket = 0;
+}
+
+// 2-D fields (row view: the rows stream as the slow axis, ny = 1): lane = column, the row
+// neighbours are the previous / next streamed rows in registers, the column neighbours come from
+// the adjacent lanes by shuffles (the two warp-edge lanes load their outer neighbour directly),
+// so there is no shared-memory plane and no barrier.  One point per thread, 256 columns per block.
+template <typename T>
+__global__ void __launch_bounds__(256)
+deriv2_kernel(Field3<T> s, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+              unsigned int* __restrict__ ticket) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gx = (int64_t)blockIdx.x * 256 + threadIdx.x;
+  const int64_t nx = s.nx, nrow = s.nz;
+  const int64_t gxc = gx < nx ? gx : nx - 1;
+  const bool inx = gx >= 1 && gx < nx - 1;
+  int64_t zlo = 1, zhi = nrow - 1;
+  if (zlo < s.zown0) zlo = s.zown0;
+  if (zhi > s.zown1) zhi = s.zown1;
+  const int64_t zb = zlo + (int64_t)blockIdx.z * zchunk;       // grid: (column tiles, 1, row chunks)
+  int64_t ze = zb + zchunk;
+  if (ze > zhi) ze = zhi;
+  double acc[kDerivSlots];
+#pragma unroll
+  for (int k = 0; k < kDerivSlots; k++) acc[k] = op_identity(deriv_op(k));
+  const int n = ze > zb ? (int)(ze - zb) : 0;
+  if (n > 0) {
+    const T* X = s.xp(0);
+    const T* Y = s.yp(0);
+    // edge lanes also read the column just outside the warp (clamped inside the row)
+    const int64_t ox = lane == 0 ? (gxc > 0 ? gxc - 1 : 0) : (lane == 31 ? (gxc + 1 < nx ? gxc + 1 : nx - 1) : gxc);
+    const T* px = X + (zb - 1) * nx;
+    const T* py = Y + (zb - 1) * nx;
+    double xm = px[gxc], ym = py[gxc];
+    px += nx; py += nx;
+    double x0 = px[gxc], y0 = py[gxc], xo = px[ox], yo = py[ox];
+    px += nx; py += nx;
+    T nxv = px[gxc], nyv = py[gxc], nxo = px[ox], nyo = py[ox];   // row zb + 1 (interior rows end at nrow - 2)
+    for (int i = 0; i < n; i++) {
+      const double xp = nxv, yp = nyv, xpo = nxo, ypo = nyo;
+      if (i + 1 < n) {
+        px += nx; py += nx;
+        nxv = __ldg(px + gxc); nyv = __ldg(py + gxc); nxo = __ldg(px + ox); nyo = __ldg(py + ox);
+      }
+      // column neighbours of the centre row: lanes +-1, the edge lanes' outer ones from xo / yo
+      double xw = __shfl_up_sync(0xffffffffu, x0, 1), yw = __shfl_up_sync(0xffffffffu, y0, 1);
+      double xe = __shfl_down_sync(0xffffffffu, x0, 1), ye = __shfl_down_sync(0xffffffffu, y0, 1);
+      if (lane == 0) { xw = xo; yw = yo; }
+      if (lane == 31) { xe = xo; ye = yo; }
+      if (inx) {
+        double Fx[CZC_NDERIV], Fy[CZC_NDERIV];
+        deriv_fields<true, false>(x0, xp, xm, 0.0, 0.0, xe, xw, Fx);
+        deriv_fields<true, false>(y0, yp, ym, 0.0, 0.0, ye, yw, Fy);
+#pragma unroll
+        for (int fi = 0; fi < CZC_NDERIV; fi++) {
+          const double d = Fy[fi] - Fx[fi];
+          acc[fi * kDerivStats + 0] = dmax(acc[fi * kDerivStats + 0], fabs(d));
+          acc[fi * kDerivStats + 1] += fabs(d);
+          acc[fi * kDerivStats + 2] = fma(d, d, acc[fi * kDerivStats + 2]);
+          acc[fi * kDerivStats + 3] = dmin(acc[fi * kDerivStats + 3], Fx[fi]);
+          acc[fi * kDerivStats + 4] = dmax(acc[fi * kDerivStats + 4], Fx[fi]);
+        }
+      }
+      xm = x0; ym = y0; x0 = xp; y0 = yp; xo = xpo; yo = ypo;
+    }
+  }
+  scale_halved(acc);
+  const unsigned bid = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
+  block_reduce_slots<kDerivSlots>(acc, DerivOp{}, parts + (size_t)bid * kDerivSlots);
+  if (!last_block_arrive(ticket)) return;
+  finish_slots<kDerivSlots>(parts, gridDim.x * gridDim.y * gridDim.z, DerivOp{}, res->rec.deriv);
+  if (threadIdx.x == 0) *ticket = 0;
 }
 
 // 3-D variant with two points per thread: threads (32, 4) cover a 32 x 8 tile, thread (tx, ty)
@@ -897,7 +968,7 @@ cudaError_t launch_deriv(const Field3<T>& s0, int zchunk, double* parts, DevResu
   const dim3 grid = deriv_grid(s, zchunk, &zc);
   if (s.ny > 1 && s.nz > 2) deriv3_kernel<T, 2><<<grid, dim3(kTX, kTY / 2), 0, st>>>(s, zc, parts, res, ticket);
   else if (s.ny > 1) deriv_kernel<T, true, true, kTX, kTY><<<grid, dim3(kTX, kTY), 0, st>>>(s, zc, parts, res, ticket);
-  else if (s.nz > 1) deriv_kernel<T, true, false, 256, 1><<<grid, dim3(256, 1), 0, st>>>(s, zc, parts, res, ticket);
+  else if (s.nz > 1) deriv2_kernel<T><<<grid, 256, 0, st>>>(s, zc, parts, res, ticket);
   else deriv_kernel<T, false, false, 256, 1><<<grid, dim3(256, 1), 0, st>>>(s, zc, parts, res, ticket);
   return cudaGetLastError();
 }
