@@ -705,3 +705,29 @@ def test_graph_replay_sees_new_contents_and_plans(czc, orc):
             report(errors)
             gp = a.assess(xd, yd, czc.M_P1 | czc.M_PDF)           # another signature in between
             assert gp["computed_mask"] == czc.M_P1 | czc.M_PDF and gp["mse"] == g["mse"]
+
+
+def test_full_size_hurricane_float64(czc, orc):
+    """BASELINE configs[1] shape with float64 inputs (the field widened with a 1e-9 relative
+    perturbation, 400 MB pair): P1, derivatives and AC against the float64 oracle over all 25 M
+    elements, the exact mean of the per-window SSIM values, 200 sampled windows."""
+    spec = synth.CONFIGS["C2"]
+    x, y = synth.make_pair(spec)
+    r = np.random.default_rng(17)
+    xn = x.numpy().astype(np.float64) * (1.0 + 1e-9 * r.standard_normal(spec.dims))
+    yn = xn + (y.numpy().astype(np.float64) - x.numpy().astype(np.float64))
+    nw = [n - 8 + 1 for n in xn.shape]
+    dbg = torch.empty(nw, dtype=torch.float64, device="cuda")
+    with czc.Assessor(ssim_window=8, debug_wssim=dbg.data_ptr()) as a:
+        g = a.assess(torch.from_numpy(xn).cuda(), torch.from_numpy(yn).cuda())
+    errors = []
+    check_p1(g, orc.p1(xn, yn), errors)
+    check_deriv(g, orc.deriv(xn, yn), errors)
+    ac, cnt = orc.autocorr(xn, yn, 10)
+    check_ac(g["ac"], g["ac_count"], ac, cnt, errors)
+    report(errors)
+    d = dbg.cpu().numpy()
+    assert g["n_windows"] == np.prod(nw) and abs(d.mean() - g["ssim"]) < 1e-12
+    for _ in range(200):
+        o = [int(r.integers(0, k)) for k in nw]
+        assert abs(d[tuple(o)] - orc.ssim_window(xn, yn, o, [8, 8, 8])) < 1e-6, o
