@@ -30,8 +30,25 @@ def _nvcc() -> str:
     raise RuntimeError("nvcc not found: the CUDA extension cannot be built")
 
 
+def _torch_nccl():
+    """(include dir, lib dir) of the NCCL that PyTorch loads (the `nvidia-nccl` wheel), or None.
+    libczc.so links that one, not the system libnccl: both carry the soname libnccl.so.2, and
+    whichever a process loads first serves both, so an older system copy loaded through libczc
+    before torch would leave torch's newer NCCL symbols unresolved."""
+    import importlib.util
+    try:
+        spec = importlib.util.find_spec("nvidia.nccl")
+    except (ImportError, ValueError):
+        spec = None
+    for loc in (list(spec.submodule_search_locations) if spec else []):
+        inc, lib = os.path.join(loc, "include"), os.path.join(loc, "lib")
+        if os.path.exists(os.path.join(inc, "nccl.h")) and os.path.exists(os.path.join(lib, "libnccl.so.2")):
+            return inc, lib
+    return None
+
+
 def _have_nccl() -> bool:
-    return os.path.exists("/usr/include/nccl.h")
+    return _torch_nccl() is not None or os.path.exists("/usr/include/nccl.h")
 
 
 def _flags():
@@ -39,6 +56,9 @@ def _flags():
                 "-I" + os.path.join(ROOT, "include")]
     if _have_nccl():
         f.append("-DCZC_WITH_NCCL")
+        tn = _torch_nccl()
+        if tn:
+            f.append("-I" + tn[0])
     return f
 
 
@@ -76,7 +96,10 @@ def build(force: bool = False, verbose: bool = False) -> str:
     objs = [os.path.join(OBJ, s.replace(".cu", ".o")) for s in SOURCES]
     if force or jobs or _stale(SO, objs):
         cmd = [nvcc] + ARCH + ["-shared", "-o", SO + ".tmp"] + objs + ["-lcudart_static"]
-        if _have_nccl():
+        tn = _torch_nccl()
+        if tn:
+            cmd += ["-L" + tn[1], "-l:libnccl.so.2", "-Xlinker", "-rpath=" + tn[1]]
+        elif _have_nccl():
             cmd.append("-lnccl")
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
