@@ -363,6 +363,8 @@ def run_ours(args, rank, world, local):
                                  "outside the step events); the pair (200 MB) is also larger than L2"},
             "per_pattern_ms": {k: round(v, 4) for k, v in shares.items()},
             "per_pattern_gbs": {k: round(alg_bytes / (v * 1e-3) / 1e9, 2) for k, v in shares.items() if v > 0},
+            "per_pattern_hbm_frac": {k: round(alg_bytes / (v * 1e-3) / 1e9 / peak, 4)
+                                     for k, v in shares.items() if v > 0},
             "roofline": {"bound": "hbm", "kernel": dom, "achieved": round(achieved, 2), "peak": peak,
                          "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
                          "peak_source": peak_src, "traffic_source": traffic_src,
