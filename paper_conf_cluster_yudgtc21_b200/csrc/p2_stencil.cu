@@ -717,7 +717,7 @@ ac_xwalk_smem(Field3<E> s, int T, int xchunk, double* __restrict__ parts, DevRes
 // other two axes give one bound per thread segment (lim), applied to the segment's lag sums.
 // Tiles far from the field ends (all t <= TM valid) skip even that.  The next plane's copies
 // overlap the walks of the current one.
-// Work split: the (tile, plane) pairs in tile-major order are cut into gridDim.x equal ranges,
+// Work split: the (tile, plane) pairs in plane-major order are cut into gridDim.x equal ranges,
 // one per block (a persistent grid of the resident block count): no tail wave, and the
 // assignment is static, so the result is deterministic.
 constexpr int kPlTX = 64, kPlTY = 32, kPlThreads = 256, kPlSeg = 8;
