@@ -720,11 +720,16 @@ ac_xwalk_smem(Field3<E> s, int T, int xchunk, double* __restrict__ parts, DevRes
 // Work split: the (tile, plane) pairs in plane-major order are cut into gridDim.x equal ranges,
 // one per block (a persistent grid of the resident block count): no tail wave, and the
 // assignment is static, so the result is deterministic.
-constexpr int kPlTX = 64, kPlTY = 32, kPlThreads = 256, kPlSeg = 8;
+constexpr int kPlTX = 64, kPlThreads = 256, kPlSeg = 8;
+// Tile height: 64 rows where two blocks of the 64 x 64 tile fit an SM (float32, TM <= 10: halo
+// 1.34x instead of 1.52x, half the barriers per element), else 32 rows.
+template <typename T, int TM> constexpr int pl_ty() { return (sizeof(T) == 4 && TM <= 10) ? 64 : 32; }
+template <typename T, int TM> constexpr int pl_bps() { return pl_ty<T, TM>() == 64 ? 2 : (TM <= 10 ? 3 : 2); }
 template <typename T, int TM>
 struct PlaneTile {
   static_assert(TM % 2 == 0, "even lag templates only");
-  static constexpr int HX = kPlTX + TM, HY = kPlTY + TM;
+  static constexpr int TY = pl_ty<T, TM>();
+  static constexpr int HX = kPlTX + TM, HY = TY + TM;
   static constexpr int EPG = 16 / (int)sizeof(T);        // elements per 16-byte group
   static constexpr int NV = (HX + EPG - 1) / EPG;        // 16-byte groups per staged row
   static constexpr int PF = EPG * NV;            // staged row pitch (elements), 16-byte multiple
@@ -820,26 +825,32 @@ __device__ __forceinline__ void seg_products(const double (&v)[kPlSeg + TM], int
 // limx: R_t bound of the y-role's column (from x), limy: of the x-role's row (from y), both
 // already capped by the plane's z bound.
 template <typename T, int TM, bool LIM>
-__device__ __forceinline__ void plane_walks(const PlaneTile<T, TM>& sm, int tid, int limx, int limy, double (&acc)[TM]) {
+__device__ __forceinline__ void plane_walks(const PlaneTile<T, TM>& sm, int tid, int limx, const int (&limy)[PlaneTile<T, TM>::TY / 32],
+                                            double (&acc)[TM]) {
+  constexpr int NH = PlaneTile<T, TM>::TY / 32;     // 32-row halves of the tile
+  static_assert(NH == 1 || NH == 2, "tile heights 32 and 64");
   double v[kPlSeg + TM];
-  {  // y-role
-    const int c = tid & (kPlTX - 1), ys = (tid / kPlTX) * kPlSeg;
+#pragma unroll 1
+  for (int h = 0; h < NH; h++) {
+    {  // y-role
+      const int c = tid & (kPlTX - 1), ys = (tid / kPlTX) * kPlSeg + 32 * h;
 #pragma unroll
-    for (int j = 0; j < kPlSeg + TM; j++) v[j] = sm.e[ys + j][c];
-    seg_products<TM, LIM>(v, limx, acc);
-  }
-  {  // x-role
-    const int r = tid & 31, xs = (tid / 32) * kPlSeg;
+      for (int j = 0; j < kPlSeg + TM; j++) v[j] = sm.e[ys + j][c];
+      seg_products<TM, LIM>(v, limx, acc);
+    }
+    {  // x-role
+      const int r = (tid & 31) + 32 * h, xs = (tid / 32) * kPlSeg;
 #pragma unroll
-    for (int j = 0; j < kPlSeg + TM; j++) v[j] = sm.e[r][xs + j];
-    seg_products<TM, LIM>(v, limy, acc);
+      for (int j = 0; j < kPlSeg + TM; j++) v[j] = sm.e[r][xs + j];
+      seg_products<TM, LIM>(v, h == 0 ? limy[0] : limy[NH - 1], acc);   // NH <= 2: no local array
+    }
   }
 }
 
 // grid: persistent (gridDim.x blocks); block 256; requires ny > 1.
 // VEC: rows 16-byte aligned (nx % 4 == 0, aligned plane segments) and (32 + TM) * nx < 2^31.
 template <typename T, int TM, bool VEC>
-__global__ void __launch_bounds__(kPlThreads, TM <= 10 ? 3 : 2)
+__global__ void __launch_bounds__(kPlThreads, pl_bps<T, TM>())
 ac_plane(Field3<T> s, double* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket) {
   extern __shared__ __align__(128) unsigned char plane_smem[];
   using PT = PlaneTile<T, TM>;
@@ -850,7 +861,8 @@ ac_plane(Field3<T> s, double* __restrict__ parts, DevResults* __restrict__ res, 
   const int r0 = tid / NV, g0 = tid % NV;          // this thread's first conversion group
   const double mu = res->p1g.me;
   const int64_t nzo = s.zown1 - s.zown0, ntx = (s.nx + kPlTX - 1) / kPlTX;
-  const int64_t ntiles = ntx * ((s.ny + kPlTY - 1) / kPlTY), W = ntiles * nzo;
+  constexpr int TY = PT::TY, NH = TY / 32;
+  const int64_t ntiles = ntx * ((s.ny + TY - 1) / TY), W = ntiles * nzo;
   const int64_t jb = W * blockIdx.x / gridDim.x, je = W * (blockIdx.x + 1) / gridDim.x;
   double acc[TM];
 #pragma unroll
@@ -865,13 +877,13 @@ ac_plane(Field3<T> s, double* __restrict__ parts, DevResults* __restrict__ res, 
     const int64_t q = jb / ntiles, tile = jb - q * ntiles;
     z = s.zown0 + q;
     x0 = (tile % ntx) * kPlTX;
-    y0 = (tile / ntx) * kPlTY;
+    y0 = (tile / ntx) * TY;
   }
   auto next_org = [&](int64_t& nz, int64_t& nx0, int64_t& ny0) {
     nx0 += kPlTX;
     if (nx0 >= s.nx) {
       nx0 = 0;
-      ny0 += kPlTY;
+      ny0 += TY;
       if (ny0 >= s.ny) { ny0 = 0; ++nz; }
     }
   };
@@ -883,13 +895,19 @@ ac_plane(Field3<T> s, double* __restrict__ parts, DevResults* __restrict__ res, 
   };
   if (jb < je) stage_item(z, x0, y0);
   for (int64_t j = jb; j < je; j++) {
-    const bool xy_inner = x0 + kPlTX + TM <= s.nx && y0 + kPlTY + TM <= s.ny;
+    const bool xy_inner = x0 + kPlTX + TM <= s.nx && y0 + TY + TM <= s.ny;
     // staged cells outside the field hold eps = 0
     const int rv = (int)(s.ny - y0 < HY ? s.ny - y0 : HY);
     const int cv = (int)(s.nx - x0 < PT::PF ? s.nx - x0 : PT::PF);
     // per-segment R_t bounds from x (y-role column) and y (x-role row)
-    const int64_t mx = s.nx - 1 - (x0 + (tid & (kPlTX - 1))), my = s.ny - 1 - (y0 + (tid & 31));
-    const int limx0 = mx < TM ? (int)(mx < -1 ? -1 : mx) : TM, limy0 = my < TM ? (int)(my < -1 ? -1 : my) : TM;
+    const int64_t mx = s.nx - 1 - (x0 + (tid & (kPlTX - 1)));
+    const int limx0 = mx < TM ? (int)(mx < -1 ? -1 : mx) : TM;
+    int limy0[NH];
+#pragma unroll
+    for (int h = 0; h < NH; h++) {
+      const int64_t my = s.ny - 1 - (y0 + (tid & 31) + 32 * h);
+      limy0[h] = my < TM ? (int)(my < -1 ? -1 : my) : TM;
+    }
     {
       cp_async_wait_all();
       __syncthreads();                     // plane z staged; previous walks done with sm.e
@@ -922,8 +940,17 @@ ac_plane(Field3<T> s, double* __restrict__ parts, DevResults* __restrict__ res, 
       // R_t bound from the z axis (active only for 3-D fields)
       const int64_t mz64 = s.nz > 1 ? s.nz - 1 - z : TM;
       const int mz = mz64 > TM ? TM : (int)mz64;
-      if (xy_inner && mz >= TM) plane_walks<T, TM, false>(sm, tid, TM, TM, acc);
-      else plane_walks<T, TM, true>(sm, tid, limx0 < mz ? limx0 : mz, limy0 < mz ? limy0 : mz, acc);
+      if (xy_inner && mz >= TM) {
+        int full[NH];
+#pragma unroll
+        for (int h = 0; h < NH; h++) full[h] = TM;
+        plane_walks<T, TM, false>(sm, tid, TM, full, acc);
+      } else {
+        int ly[NH];
+#pragma unroll
+        for (int h = 0; h < NH; h++) ly[h] = limy0[h] < mz ? limy0[h] : mz;
+        plane_walks<T, TM, true>(sm, tid, limx0 < mz ? limx0 : mz, ly, acc);
+      }
       z = nz; x0 = nx0; y0 = ny0;
     }
   }
@@ -1019,8 +1046,10 @@ static AcGrids ac_grids(const Field3<E>& s, int T) {
   }
   g.rz = s.nz > 1; g.ry = s.ny > 1; g.rx = s.nx > 1;
   // persistent in-plane grid: the resident block count (3 per SM for TM <= 10, else 2)
-  const int64_t W = cdiv(s.nx, kPlTX) * cdiv(s.ny, kPlTY) * nzo;
-  const int64_t G = (int64_t)sm_count() * (T <= 10 ? 3 : 2);
+  // (tile height and blocks per SM as pl_ty / pl_bps of the lag template chosen for T)
+  const int ty = (sizeof(E) == 4 && T <= 10) ? 64 : 32;
+  const int64_t W = cdiv(s.nx, kPlTX) * cdiv(s.ny, ty) * nzo;
+  const int64_t G = (int64_t)sm_count() * (ty == 64 ? 2 : (T <= 10 ? 3 : 2));
   g.pzc = 0;
   g.z = dim3((unsigned)cdiv(s.nx, kTX), (unsigned)cdiv(s.ny, kTY), (unsigned)cdiv(nzo, g.zc));
   g.zt = dim3((unsigned)cdiv(s.nx, kWalkCPT<E> * kWalkThreads), (unsigned)s.ny, (unsigned)cdiv(nzo, g.zc));
@@ -1063,7 +1092,7 @@ static cudaError_t launch_ac_t(const Field3<E>& s, int T, double* parts, DevResu
   if (g.ry) {
     constexpr int psm = (int)sizeof(PlaneTile<E, TM>);
     // 16-byte staging needs aligned rows; tile-relative offsets are 32-bit
-    const bool pvec = vec && (int64_t)(kPlTY + TM) * s.nx < ((int64_t)1 << 31);
+    const bool pvec = vec && (int64_t)(pl_ty<E, TM>() + TM) * s.nx < ((int64_t)1 << 31);
     auto kern = pvec ? ac_plane<E, TM, true> : ac_plane<E, TM, false>;
     if ((e = pvec ? set_smem_once<ac_plane<E, TM, true>>(psm) : set_smem_once<ac_plane<E, TM, false>>(psm)) != cudaSuccess)
       return e;
