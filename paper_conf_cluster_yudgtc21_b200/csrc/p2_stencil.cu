@@ -463,6 +463,10 @@ struct BulkWalkSmem {
   T y[S][CPT * kWalkThreads];
   uint64_t bar[S];
 };
+template <typename T, int TM, int CPT>
+__host__ __device__ constexpr int zwalk_tot_offset() { return (int)((sizeof(BulkWalkSmem<T, TM, CPT>) + 15) / 16 * 16); }
+template <typename T, int TM, int CPT>
+__host__ __device__ constexpr int zwalk_smem() { return zwalk_tot_offset<T, TM, CPT>() + TM * kWalkThreads * (int)sizeof(double); }
 
 // RowPtr(i) -> (const T* xrow, const T* yrow) for position i (already offset to x0).
 // Positions are tracked relative to lo in 32 bits.  Lane v < S of warp 0 issues slot v's copies
@@ -470,16 +474,12 @@ struct BulkWalkSmem {
 template <typename T, int TM, int CPT, typename RowPtr>
 __device__ __forceinline__ void bulk_walk(BulkWalkSmem<T, TM, CPT>& sm, RowPtr row_ptr, uint32_t bytes, int64_t lo,
                                           int64_t hi, int64_t end, double mu,
-                                          double (&ring)[CPT][TM], double (&acc)[CPT][TM]) {
+                                          double (&ring)[CPT][TM], double (&acc)[CPT][TM], uint32_t& phase) {
   constexpr int S = 2 * TM;
+  static_assert(S <= 32, "one phase bit per slot");
   const int tid = threadIdx.x;
   const int jend = (int)(end - lo), jhi = (int)(hi - lo);
-  if (tid == 0) {
-#pragma unroll
-    for (int v = 0; v < S; v++) mbar_init(&sm.bar[v], 1);
-    fence_mbar_init();
-  }
-  __syncthreads();
+  __syncthreads();                                     // barriers initialised; previous line's slots consumed
   auto issue = [&](int slot, int j) {
     const T* xr;
     const T* yr;
@@ -489,13 +489,13 @@ __device__ __forceinline__ void bulk_walk(BulkWalkSmem<T, TM, CPT>& sm, RowPtr r
     bulk_g2s(sm.y[slot], yr, bytes, &sm.bar[slot]);
   };
   if (tid < S && tid < jend) issue(tid, tid);
-  uint32_t parity = 0;
   for (int j0 = 0; j0 < jend; j0 += S) {
 #pragma unroll
     for (int u = 0; u < S; u++) {
       const int j = j0 + u;
       if (j < jend) {                                  // block-uniform
-        mbar_wait(&sm.bar[u], parity);
+        mbar_wait(&sm.bar[u], (phase >> u) & 1u);
+        phase ^= 1u << u;
 #pragma unroll
         for (int c = 0; c < CPT; c++) {
           const int col = tid + c * kWalkThreads;
@@ -509,47 +509,73 @@ __device__ __forceinline__ void bulk_walk(BulkWalkSmem<T, TM, CPT>& sm, RowPtr r
         if (tid < TM && j0 + v + S < jend) issue(v, j0 + v + S);
       }
     }
-    parity ^= 1u;
   }
 }
 
-// z-walk, TMA: block = CPT x 256 consecutive x of row y; grid (x tiles, ny, z chunks).
+// z-walk, TMA: a line = CPT x 256 consecutive x of row y; persistent grid (the resident block
+// count), the (line, owned plane) units in line-major order cut into gridDim.x equal ranges, so
+// every block walks ~the same number of planes (a grid of (line, z-chunk) blocks ran 1.7 waves on
+// C2) and a range's pieces of two lines each pay their own T halo planes.  The per-line sums are
+// masked with the line's R_tau bound and folded into a per-thread total in shared memory.
 template <typename E, int TM, int CPT>
 __global__ void __launch_bounds__(kWalkThreads, CPT == 1 ? 3 : 2)
-ac_zwalk_tma(Field3<E> s, int T, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
+ac_zwalk_tma(Field3<E> s, int T, int, double* __restrict__ parts, DevResults* __restrict__ res,
              unsigned int* __restrict__ ticket) {
   extern __shared__ __align__(128) unsigned char walk_smem[];
-  BulkWalkSmem<E, TM, CPT>& sm = *reinterpret_cast<BulkWalkSmem<E, TM, CPT>*>(walk_smem);
-  const int64_t x0 = (int64_t)blockIdx.x * (CPT * kWalkThreads), gy = blockIdx.y;
+  using SM = BulkWalkSmem<E, TM, CPT>;
+  SM& sm = *reinterpret_cast<SM*>(walk_smem);
+  double* tot = reinterpret_cast<double*>(walk_smem + zwalk_tot_offset<E, TM, CPT>());   // [TM][kWalkThreads]
+  const int tid = threadIdx.x;
   const double mu = res->p1g.me;
-  int64_t mrow = T;
-  if (s.ny > 1 && s.ny - 1 - gy < mrow) mrow = s.ny - 1 - gy;
-  const int64_t lo = s.zown0 + (int64_t)blockIdx.z * zchunk;
-  int64_t hi = lo + zchunk;
-  if (hi > s.zown1) hi = s.zown1;
-  int64_t end = hi + T;
-  if (end > s.nz) end = s.nz;
-  const int64_t ncols = (s.nx - x0) < CPT * kWalkThreads ? (s.nx - x0) : CPT * kWalkThreads;
-  const int64_t off = gy * s.nx + x0;
-  double ring[CPT][TM], acc[CPT][TM];
+  constexpr int LW = CPT * kWalkThreads;
+  const int64_t nzo = s.zown1 - s.zown0, ntx = (s.nx + LW - 1) / LW;
+  const int64_t W = ntx * s.ny * nzo;
+  const int64_t jb = W * blockIdx.x / gridDim.x, je = W * (blockIdx.x + 1) / gridDim.x;
 #pragma unroll
-  for (int c = 0; c < CPT; c++)
+  for (int t = 0; t < TM; t++) tot[t * kWalkThreads + tid] = 0.0;
+  if (tid == 0) {
 #pragma unroll
-    for (int t = 0; t < TM; t++) ring[c][t] = acc[c][t] = 0;
-  bulk_walk<E, TM, CPT>(sm, [&](int64_t z, const E*& xr, const E*& yr) { xr = s.xp(z) + off; yr = s.yp(z) + off; },
-                        (uint32_t)(ncols * sizeof(E)), lo, hi, end, mu, ring, acc);
-  // per column: the R_tau bound from y and x (lim = 0 past the row end), then one sum
-#pragma unroll
-  for (int c = 0; c < CPT; c++) {
-    const int64_t gx = x0 + threadIdx.x + c * kWalkThreads;
-    int64_t m = mrow;
-    if (s.nx > 1 && s.nx - 1 - gx < m) m = s.nx - 1 - gx;
-    walk_mask<TM>(acc[c], gx < s.nx ? (int)m : 0);
-    if (c > 0)
-#pragma unroll
-      for (int t = 0; t < TM; t++) acc[0][t] += acc[c][t];
+    for (int v = 0; v < 2 * TM; v++) mbar_init(&sm.bar[v], 1);
+    fence_mbar_init();
   }
-  ac_finish<TM>(acc[0], parts, res->rec.ac[0], ticket);
+  uint32_t phase = 0;
+  for (int64_t j = jb; j < je;) {
+    const int64_t line = j / nzo, dz = j - line * nzo;
+    const int64_t run = (je - j) < (nzo - dz) ? (je - j) : (nzo - dz);
+    j += run;
+    const int64_t gy = line / ntx, x0 = (line - gy * ntx) * LW;
+    int64_t mrow = T;
+    if (s.ny > 1 && s.ny - 1 - gy < mrow) mrow = s.ny - 1 - gy;
+    const int64_t lo = s.zown0 + dz, hi = lo + run;
+    int64_t end = hi + T;
+    if (end > s.nz) end = s.nz;
+    const int64_t ncols = (s.nx - x0) < LW ? (s.nx - x0) : LW;
+    const int64_t off = gy * s.nx + x0;
+    double ring[CPT][TM], acc[CPT][TM];
+#pragma unroll
+    for (int c = 0; c < CPT; c++)
+#pragma unroll
+      for (int t = 0; t < TM; t++) ring[c][t] = acc[c][t] = 0;
+    bulk_walk<E, TM, CPT>(sm, [&](int64_t z, const E*& xr, const E*& yr) { xr = s.xp(z) + off; yr = s.yp(z) + off; },
+                          (uint32_t)(ncols * sizeof(E)), lo, hi, end, mu, ring, acc, phase);
+    // per column: the R_tau bound from y and x (lim = 0 past the row end), then one sum
+#pragma unroll
+    for (int c = 0; c < CPT; c++) {
+      const int64_t gx = x0 + tid + c * kWalkThreads;
+      int64_t m = mrow;
+      if (s.nx > 1 && s.nx - 1 - gx < m) m = s.nx - 1 - gx;
+      walk_mask<TM>(acc[c], gx < s.nx ? (int)m : 0);
+      if (c > 0)
+#pragma unroll
+        for (int t = 0; t < TM; t++) acc[0][t] += acc[c][t];
+    }
+#pragma unroll
+    for (int t = 0; t < TM; t++) tot[t * kWalkThreads + tid] += acc[0][t];
+  }
+  double fin[TM];
+#pragma unroll
+  for (int t = 0; t < TM; t++) fin[t] = tot[t * kWalkThreads + tid];
+  ac_finish<TM>(fin, parts, res->rec.ac[0], ticket);
 }
 
 // z-walk: thread <-> column (y, x); block 32 x 8 columns; grid.z chunks of owned planes.
@@ -1052,7 +1078,17 @@ static AcGrids ac_grids(const Field3<E>& s, int T) {
   const int64_t G = (int64_t)sm_count() * (ty == 64 ? 2 : (T <= 10 ? 3 : 2));
   g.pzc = 0;
   g.z = dim3((unsigned)cdiv(s.nx, kTX), (unsigned)cdiv(s.ny, kTY), (unsigned)cdiv(nzo, g.zc));
-  g.zt = dim3((unsigned)cdiv(s.nx, kWalkCPT<E> * kWalkThreads), (unsigned)s.ny, (unsigned)cdiv(nzo, g.zc));
+  {  // persistent TMA z-walk: the resident block count (register bound 3 / 2 per SM, shared-memory bound)
+    const int tm = T <= 10 ? (T + 1) / 2 * 2 : (T <= 12 ? 12 : 16), cpt = kWalkCPT<E>;
+    const int64_t smem = (int64_t)2 * tm * cpt * kWalkThreads * 2 * (int64_t)sizeof(E) + 2 * tm * 8 + 16 +
+                         (int64_t)tm * kWalkThreads * 8 + 1024;
+    int64_t bps = (227 * 1024 + 1024) / smem;
+    const int64_t rb = cpt == 1 ? 3 : 2;
+    if (bps > rb) bps = rb;
+    if (bps < 1) bps = 1;
+    const int64_t Wz = cdiv(s.nx, kWalkCPT<E> * kWalkThreads) * s.ny * nzo, Gz = (int64_t)sm_count() * bps;
+    g.zt = dim3((unsigned)(Wz < Gz ? Wz : Gz), 1, 1);
+  }
   g.pl = dim3((unsigned)(W < G ? W : G), 1, 1);
   g.x = dim3((unsigned)cdiv(nzo * s.ny, kXWarps * 32), (unsigned)cdiv(s.nx, g.xc), 1);
   g.xvec = dim3((unsigned)cdiv(nzo * s.ny, 256), (unsigned)cdiv(s.nx, g.xc), 1);
@@ -1083,7 +1119,7 @@ static cudaError_t launch_ac_t(const Field3<E>& s, int T, double* parts, DevResu
   if (e != cudaSuccess) return e;
   if (g.rz && vec) {
     constexpr int C = kWalkCPT<E>;
-    constexpr int wsm = (int)sizeof(BulkWalkSmem<E, TM, C>);
+    constexpr int wsm = zwalk_smem<E, TM, C>();
     if ((e = set_smem_once<ac_zwalk_tma<E, TM, C>>(wsm)) != cudaSuccess) return e;
     ac_zwalk_tma<E, TM, C><<<g.zt, kWalkThreads, wsm, st>>>(s, T, g.zc, pz, res, tickets + 0);
   } else if (g.rz) {
