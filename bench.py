@@ -37,7 +37,12 @@ def parse():
     p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    p.add_argument("--config", default="C2")
+    p.add_argument("--config", default="C5", help="BASELINE workload (C5 2048^3 = configs[4]; C2, C3)")
+    p.add_argument("--scaling", default="strong", choices=["strong", "weak"],
+                   help="strong: the config's fixed field cut into slabs; weak: one field per rank")
+    p.add_argument("--extra", default="C2,C3", help="other configs timed at N=1 for context")
+    p.add_argument("--no-extra", action="store_true")
+    p.add_argument("--cpu-planes", type=int, default=0)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-f64", action="store_true", help="skip the float64-input measurement")
@@ -168,8 +173,103 @@ def run_reference(args, rank, world):
 
 
 # ------------------------------------------------------------------------------------ our leg
+def host_info():
+    """Host cores the oracle can use (cpu_baseline.cores is what it actually used)."""
+    info = {"nproc": os.cpu_count(), "omp_num_threads": os.environ.get("OMP_NUM_THREADS")}
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            k, _, v = ln.partition(":")
+            if k.strip() in ("Model name", "Socket(s)", "Core(s) per socket", "Thread(s) per core"):
+                info[k.strip()] = v.strip()
+    except Exception:
+        pass
+    return info
+
+
+def slab_bounds(nz: int, rank: int, world: int, scaling: str):
+    """Planes [z0, z1) of this rank: strong scaling cuts the fixed global field into equal slabs
+    (SURVEY.md §8(e)); weak scaling stacks one whole config field per rank."""
+    if scaling == "strong":
+        return nz * rank // world, nz * (rank + 1) // world, nz
+    return nz * rank, nz * (rank + 1), nz * world
+
+
+def make_slab_device(spec, z0: int, z1: int, dev, world: int):
+    """(x, y) float32 of planes [z0, z1) generated ON THE DEVICE, a few planes at a time (no
+    68.7 GB host buffer for C5): x first, then the GLOBAL value range (min / max over all ranks)
+    that a relative error bound needs, then y from x.  synth's recipe; bit-identical to the CPU
+    generation except for exp() kinds (synth docstring)."""
+    import torch
+    import torch.distributed as dist
+    import synth
+    rest = tuple(spec.dims[1:])
+    plane = 1
+    for d in rest:
+        plane *= d
+    ch = max(1, (1 << 27) // plane)                      # ~134 M elements per generation chunk
+    x = torch.empty((z1 - z0,) + rest, dtype=torch.float32, device=dev)
+    lo = torch.tensor([float("inf")], dtype=torch.float64, device=dev)
+    hi = torch.tensor([-float("inf")], dtype=torch.float64, device=dev)
+    for c0 in range(z0, z1, ch):
+        c1 = min(z1, c0 + ch)
+        xc = synth.make_field(spec, c0, c1, device=dev)
+        x[c0 - z0:c1 - z0] = xc
+        lo = torch.minimum(lo, xc.min().double().reshape(1))
+        hi = torch.maximum(hi, xc.max().double().reshape(1))
+        del xc
+    if world > 1:
+        dist.all_reduce(lo, op=dist.ReduceOp.MIN)
+        dist.all_reduce(hi, op=dist.ReduceOp.MAX)
+    rng = float(hi.item() - lo.item())
+    y = torch.empty_like(x)
+    for c0 in range(z0, z1, ch):
+        c1 = min(z1, c0 + ch)
+        y[c0 - z0:c1 - z0] = synth.make_recon(spec, x[c0 - z0:c1 - z0], c0, range_hint=rng)
+    torch.cuda.synchronize(dev)
+    return x, y
+
+
+PATTERNS = ("P1", "P2_deriv", "P2_autocorr", "P3_ssim")
+
+
+def time_steps(czc, a, xd, yd, kw, steps, warmup, stream, flush, clean, barrier=None):
+    """Device time (ms) of each of `steps` czc_assess calls after `warmup` untimed ones, L2
+    flushed between them (outside the events)."""
+    import torch
+    for _ in range(warmup):
+        a.assess(xd, yd, czc.M_ALL, **kw)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    if barrier:
+        barrier()
+    for i in range(steps):
+        flush.zero_()                                   # L2 flush between timed steps (not timed):
+        clean.sum()                                     # write 256 MB, then read ANOTHER 256 MB so
+                                                        # the dirty lines are written back before the
+                                                        # step starts and L2 holds only clean lines
+        ev[i][0].record(stream)
+        r = a.assess(xd, yd, czc.M_ALL, **kw)
+        ev[i][1].record(stream)
+    if barrier:
+        barrier()
+    torch.cuda.synchronize()
+    return [s.elapsed_time(e) for s, e in ev], r
+
+
+def pattern_split(czc, xd, yd, kw, cfg, steps, warmup, stream, flush, clean, local):
+    """Per-kernel device time (library events on the launching stream, per-kernel timing mode)."""
+    kms = []
+    with czc.Assessor(ndim=3, device=local, stream=stream, timing=True, **cfg) as at:
+        for i in range(warmup + steps):
+            flush.zero_()
+            clean.sum()
+            r = at.assess(xd, yd, czc.M_ALL, **kw)
+            if i >= warmup:
+                kms.append(r["kernel_ms"])
+    return {name: statistics.mean(k[i] for k in kms) for i, name in enumerate(PATTERNS)}
+
+
 def run_ours(args, rank, world, local):
-    import numpy as np
     import torch
     import torch.distributed as dist
 
@@ -179,22 +279,20 @@ def run_ours(args, rank, world, local):
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     spec = synth.CONFIGS[args.config]
-    nz_local = spec.dims[0]
-    gdims = (nz_local * world,) + tuple(spec.dims[1:])
+    scaling = args.scaling
+    z0, z1, gnz = slab_bounds(spec.dims[0], rank, world, scaling)
+    gdims = (gnz,) + tuple(spec.dims[1:])
     gspec = synth.config(args.config, dims=gdims)
-    z0 = rank * nz_local
-    # generate this rank's slab on the host (bit-identical recipe), copy once to HBM
-    xh, yh = synth.make_pair(gspec, z0, z0 + nz_local, device="cpu",
-                             range_hint=None)
-    xd, yd = xh.to(dev), yh.to(dev)
-    nbytes_rank = 2 * xh.numel() * 4
-
     uid = None
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
         obj = [czc_nccl_uid() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         uid = obj[0]
+    t_gen = time.perf_counter()
+    xd, yd = make_slab_device(gspec, z0, z1, dev, world)
+    t_gen = time.perf_counter() - t_gen
+    nbytes_rank = 2 * xd.numel() * 4
     stream = torch.cuda.current_stream(dev)
     cfg = dict(ssim_window=8, ssim_step=1, ac_max_lag=10)
     if world > 1:
@@ -212,55 +310,46 @@ def run_ours(args, rank, world, local):
 
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)   # 256 MB > L2
     clean = torch.zeros(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)   # read-only after this
+    sampler = ClockSampler(local)
     for _ in range(args.warmup):
         a.assess(xd, yd, czc.M_ALL, **kw)
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    kms = []
-    sampler = ClockSampler(local)
     barrier()
     sampler.start()
     time.sleep(0.3)
     t_wall = time.perf_counter()
-    for i in range(args.steps):
-        flush.zero_()                                   # L2 flush between timed steps (not timed):
-        clean.sum()                                     # write 256 MB, then read ANOTHER 256 MB so
-                                                        # the dirty lines are written back before the
-                                                        # step starts and L2 holds only clean lines
-        ev[i][0].record(stream)
-        a.assess(xd, yd, czc.M_ALL, **kw)
-        ev[i][1].record(stream)
-    barrier()
+    step_ms, r = time_steps(czc, a, xd, yd, kw, args.steps, 0, stream, flush, clean, barrier)
     t_wall = time.perf_counter() - t_wall
     clocks = sampler.stop()
-    cfg_t = dict(cfg)
-    if world > 1:                       # a second communicator needs its own ncclUniqueId
-        obj = [czc_nccl_uid() if rank == 0 else None]
-        dist.broadcast_object_list(obj, src=0)
-        cfg_t["nccl_uid"] = obj[0]
-    with czc.Assessor(ndim=3, device=local, stream=stream, timing=True, **cfg_t) as at:
-        for i in range(args.warmup + args.steps):
-            flush.zero_()
-            clean.sum()
-            r = at.assess(xd, yd, czc.M_ALL, **kw)
-            if i >= args.warmup:
-                kms.append(r["kernel_ms"])
-    step_ms = [s.elapsed_time(e) for s, e in ev]
     tot_ms = sum(step_ms)
     if world > 1:
         t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         tot_ms = float(t.item())
-    value = world * nbytes_rank * args.steps / (tot_ms * 1e-3) / 1e9
+    total_bytes = 2 * 4 * int(np_prod(gdims))            # the whole field, all ranks
+    value = total_bytes * args.steps / (tot_ms * 1e-3) / 1e9
 
-    # per-kernel device time (library events on the launching stream), averaged over timed steps:
-    # P1, P2 derivatives, P2 autocorrelation (3 walk launches), P3 SSIM
-    shares = {name: statistics.mean(k[i] for k in kms)
-              for i, name in enumerate(("P1", "P2_deriv", "P2_autocorr", "P3_ssim"))}
+    cfg_t = dict(cfg)
+    if world > 1:                       # a second communicator needs its own ncclUniqueId
+        obj = [czc_nccl_uid() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        cfg_t["nccl_uid"] = obj[0]
+    shares = pattern_split(czc, xd, yd, kw, cfg_t, max(3, args.steps // 2), min(args.warmup, 3), stream,
+                           flush, clean, local)
     dom = max(shares, key=shares.get)
-    # secondary ceiling: every pattern is FP64-arithmetic / issue bound, so the
+    peak, peak_src = measured_peak()
+    alg_bytes = nbytes_rank                              # each pattern reads the pair once (+ halos)
+    per_gbs = {k: alg_bytes / (v * 1e-3) / 1e9 for k, v in shares.items() if v > 0}
+    achieved = per_gbs[dom]
+    tr = ncu_traffic()
+    traffic, traffic_src = None, None
+    if tr and tr.get("kernel_pattern") == dom and tr.get("dram_bytes_per_alg_byte"):
+        traffic = round(tr["dram_bytes_per_alg_byte"] * alg_bytes, 0)
+        traffic_src = (f"{tr.get('source')}: {tr['dram_bytes_per_alg_byte']:.4f} DRAM bytes per algorithmic byte "
+                       f"measured on {tr.get('workload')}, times this launch's algorithmic bytes")
+    # secondary ceiling: the patterns are FP64-arithmetic / issue bound: the
     # algorithmic FP64 operations of the method (per element / interior point /
-    # window) are also set against the FP64 pipe rate measured on this GPU model
-    # (profiles/r01_pipes2.txt: DFMA 61.6 lanes/clk/SM; 148 SMs at 1.965 GHz)
+    # window) against the FP64 pipe rate measured on this GPU model (profiles/r01_pipes2.txt:
+    # DFMA 61.6 lanes/clk/SM; 148 SMs at 1.965 GHz)
     fp64_peak = 61.6 * 148 * 1.965                     # G FP64 instructions / s
     units = {"P1": (12, int(r["n"]), "element: e, 6 moment sums, |e| sum, 2 extrema, pwr quotient + sum"),
              "P2_deriv": (74, int(r["n_interior"]), "interior point: 2 x 22 stencil ops, 2 sqrt, 5 x 6 statistics"),
@@ -272,99 +361,112 @@ def run_ours(args, rank, world, local):
             a_g = ops * n_units / world / (shares[k] * 1e-3) / 1e9    # per GPU (units are global)
             fp64[k] = {"achieved": round(a_g, 1), "frac": round(a_g / fp64_peak, 4), "ops_per_unit": ops,
                        "units_per_launch": n_units, "unit": what}
-    peak, peak_src = measured_peak()
-    alg_bytes = nbytes_rank                              # each pattern reads the pair once (+ halos)
-    achieved = alg_bytes / (shares[dom] * 1e-3) / 1e9
-    tr = ncu_traffic()
-    traffic = tr.get("dram_bytes_per_launch") if tr and tr.get("kernel_pattern") == dom else None
-    traffic_src = tr.get("source") if tr and traffic else None
     # kernels of ours per step: P1, derivatives, AC z-walk + in-plane tile kernel, SSIM
     # (slab mode adds the on-device P1 state merge); the record memset is not counted
     launches_per_step = (1 + 1 + 2 + 1) if world == 1 else (2 + 1 + 2 + 1)
 
-    # end-to-end through the public host-buffer entry point (H2D + kernels + D2H inside)
+    # end-to-end through the public host-buffer entry point (H2D + kernels + D2H inside): the
+    # same slab copied once into pinned host memory, then the device copies are released
     e2e = None
     if not args.no_e2e:
-        # czc_assess_host pipelines K = min(8, nz / 4) z-chunks and copies back one record
-        # prefix per chunk (czc_sizeof(4) bytes each)
-        K = min(8, nz_local // 4) if world == 1 else world
-        d2h_host = int(czc.get_lib().czc_sizeof(4)) * (K if K >= 2 else 1)
-        xp = xh.pin_memory()
-        yp = yh.pin_memory()
-        for _ in range(max(3, args.warmup)):            # the H2D path keeps speeding up over the
-            a.assess_host(xp, yp, czc.M_ALL, **kw)      # first calls (4.39 -> 4.23 ms); warm it like the kernels
-        barrier()
-        t0 = time.perf_counter()
-        e_tot = 0.0
-        for _ in range(max(3, args.steps // 2)):
-            s_ev, e_ev = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            s_ev.record(stream)
-            a.assess_host(xp, yp, czc.M_ALL, **kw)
-            e_ev.record(stream)
-            e_ev.synchronize()
-            e_tot += s_ev.elapsed_time(e_ev)
-        nsteps_e2e = max(3, args.steps // 2)
-        if world > 1:
-            t = torch.tensor([e_tot], dtype=torch.float64, device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            e_tot = float(t.item())
-        e2e = {"value": round(world * nbytes_rank * nsteps_e2e / (e_tot * 1e-3) / 1e9, 3), "unit": UNIT,
-               "h2d_bytes_per_step": nbytes_rank, "d2h_bytes_per_step": d2h_host,
-               "ms_per_step": round(e_tot / nsteps_e2e, 4)}
-
-    # float64 inputs (NEXT row f3): the same field widened to double, 16 B per element pair
-    f64 = None
-    if world == 1 and not args.no_f64:
-        xd64, yd64 = xd.double(), yd.double()
-        n64 = 2 * xd64.numel() * 8
-        with czc.Assessor(ndim=3, device=local, stream=stream, **cfg) as a64, \
-                czc.Assessor(ndim=3, device=local, stream=stream, timing=True, **cfg) as t64:
-            for _ in range(args.warmup):
-                a64.assess(xd64, yd64, czc.M_ALL)
-            tot64, k64 = 0.0, []
-            for i in range(args.steps):
-                flush.zero_()
-                clean.sum()
+        try:
+            xp = torch.empty(xd.shape, dtype=torch.float32, pin_memory=True)
+            yp = torch.empty(yd.shape, dtype=torch.float32, pin_memory=True)
+            xp.copy_(xd)
+            yp.copy_(yd)
+            torch.cuda.synchronize(dev)
+        except Exception as ex:                          # not enough pinnable host memory
+            xp = yp = None
+            e2e = {"value": None, "unit": UNIT, "skipped": f"pinned host copy of the slab failed: {ex!r}"[:300]}
+        if xp is not None:
+            del xd, yd
+            torch.cuda.empty_cache()
+            K = min(8, (z1 - z0) // 4) if world == 1 else world
+            d2h_host = int(czc.get_lib().czc_sizeof(4)) * (K if K >= 2 else 1)
+            nsteps_e2e = max(3, args.steps // 4)
+            for _ in range(max(2, min(3, args.warmup))):   # the H2D path speeds up over the first calls
+                a.assess_host(xp, yp, czc.M_ALL, **kw)
+            barrier()
+            e_tot = 0.0
+            for _ in range(nsteps_e2e):
                 s_ev, e_ev = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 s_ev.record(stream)
-                a64.assess(xd64, yd64, czc.M_ALL)
+                a.assess_host(xp, yp, czc.M_ALL, **kw)
                 e_ev.record(stream)
                 e_ev.synchronize()
-                tot64 += s_ev.elapsed_time(e_ev)
-                flush.zero_()
-                clean.sum()
-                k64.append(t64.assess(xd64, yd64, czc.M_ALL)["kernel_ms"])
-        sh64 = {name: statistics.mean(k[i] for k in k64)
-                for i, name in enumerate(("P1", "P2_deriv", "P2_autocorr", "P3_ssim"))}
-        f64 = {"value": round(n64 * args.steps / (tot64 * 1e-3) / 1e9, 3), "unit": UNIT,
-               "ms_per_step": round(tot64 / args.steps, 4), "dtype": "f64",
-               "workload": f"the same field widened to float64 ({n64 / 1e6:.0f} MB pair)",
+                e_tot += s_ev.elapsed_time(e_ev)
+            if world > 1:
+                t = torch.tensor([e_tot], dtype=torch.float64, device=dev)
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                e_tot = float(t.item())
+            e2e = {"value": round(total_bytes * nsteps_e2e / (e_tot * 1e-3) / 1e9, 3), "unit": UNIT,
+                   "h2d_bytes_per_step": nbytes_rank, "d2h_bytes_per_step": d2h_host,
+                   "ms_per_step": round(e_tot / nsteps_e2e, 4), "steps": nsteps_e2e}
+            del xp, yp
+    a.close()
+    if "xd" in locals():
+        del xd, yd
+    torch.cuda.empty_cache()
+
+    # context configurations at N = 1 (rank 0): the other BASELINE shapes, same protocol
+    others = {}
+    if world == 1 and not args.no_extra:
+        for name in [c for c in args.extra.split(",") if c and c != args.config]:
+            sp = synth.CONFIGS[name]
+            xo, yo = make_slab_device(sp, 0, sp.dims[0], dev, 1)
+            nb = 2 * xo.numel() * 4
+            with czc.Assessor(ndim=xo.dim(), device=local, stream=stream, **cfg) as ao:
+                ms, _ = time_steps(czc, ao, xo, yo, {}, args.steps, args.warmup, stream, flush, clean)
+            sh = pattern_split(czc, xo, yo, {}, cfg, max(3, args.steps // 2), 3, stream, flush, clean, local) \
+                if xo.dim() == 3 else {}
+            others[name] = {"workload": sp.name, "dims": list(sp.dims), "value": round(nb * len(ms) / (sum(ms) * 1e-3) / 1e9, 3),
+                            "unit": UNIT, "ms_per_step": round(sum(ms) / len(ms), 4),
+                            "per_pattern_ms": {k: round(v, 4) for k, v in sh.items()},
+                            "per_pattern_hbm_frac": {k: round(nb / (v * 1e-3) / 1e9 / peak, 4) for k, v in sh.items() if v > 0}}
+            del xo, yo
+            torch.cuda.empty_cache()
+
+    # float64 inputs (NEXT row f3): C3 widened to double, 16 B per element pair
+    f64 = None
+    if world == 1 and not args.no_f64:
+        sp = synth.CONFIGS["C3"]
+        xo, yo = make_slab_device(sp, 0, sp.dims[0], dev, 1)
+        x64, y64 = xo.double(), yo.double()
+        del xo, yo
+        n64 = 2 * x64.numel() * 8
+        with czc.Assessor(ndim=3, device=local, stream=stream, **cfg) as a64:
+            ms, _ = time_steps(czc, a64, x64, y64, {}, max(3, args.steps // 2), 3, stream, flush, clean)
+        sh64 = pattern_split(czc, x64, y64, {}, cfg, max(3, args.steps // 2), 3, stream, flush, clean, local)
+        f64 = {"value": round(n64 * len(ms) / (sum(ms) * 1e-3) / 1e9, 3), "unit": UNIT,
+               "ms_per_step": round(sum(ms) / len(ms), 4), "dtype": "f64",
+               "workload": f"{sp.name} widened to float64 ({n64 / 1e6:.0f} MB pair)",
                "per_pattern_ms": {k: round(v, 4) for k, v in sh64.items()},
                "per_pattern_gbs": {k: round(n64 / (v * 1e-3) / 1e9, 2) for k, v in sh64.items() if v > 0}}
-        del xd64, yd64
+        del x64, y64
+        torch.cuda.empty_cache()
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        v, dt, cores, desc = oracle_sample(spec, planes=spec.dims[0])
+        v, dt, cores, desc = oracle_sample(spec, planes=args.cpu_planes or default_planes(spec))
         cpu = {"value": round(v, 6), "unit": UNIT, "cores": cores, "kind": "oracle", "sample": desc,
-               "seconds": round(dt, 3)}
+               "seconds": round(dt, 3), "host": host_info()}
 
     if rank == 0:
+        wl = (f"{spec.name}: {'x'.join(map(str, gdims))} float32 pair ({total_bytes / 1e9:.1f} GB), "
+              f"{'abs' if not spec.eb_relative else 'range-relative'} eb {spec.eb:g}, full metric set (P1, "
+              f"derivatives, AC lags 1..10, SSIM 8^3 step 1)")
         line = {
             "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(tot_ms / args.steps, 4),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-            "data": "synthetic",
-            "config": {"workload": f"{gspec.name.split('-')[0]} Hurricane-shaped {'x'.join(map(str, gdims))} "
-                                   f"float32 pair, abs eb {spec.eb:g}, full metric set (P1, derivatives, "
-                                   f"AC lags 1..10, SSIM 8^3 step 1)",
-                       "per_rank_planes": nz_local, "parallelism": f"slab{world}",
+            "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic (seeded synth recipe, generated on the device per rank)",
+            "config": {"workload": wl, "per_rank_planes": z1 - z0, "parallelism": f"slab{world}",
                        "l2": "flushed between timed steps (256 MB write + 256 MB read of another buffer, "
-                                 "outside the step events); the pair (200 MB) is also larger than L2"},
+                             "outside the step events); the pair is also larger than L2",
+                       "generation_s": round(t_gen, 2)},
             "per_pattern_ms": {k: round(v, 4) for k, v in shares.items()},
-            "per_pattern_gbs": {k: round(alg_bytes / (v * 1e-3) / 1e9, 2) for k, v in shares.items() if v > 0},
-            "per_pattern_hbm_frac": {k: round(alg_bytes / (v * 1e-3) / 1e9 / peak, 4)
-                                     for k, v in shares.items() if v > 0},
+            "per_pattern_gbs": {k: round(v, 2) for k, v in per_gbs.items()},
+            "per_pattern_hbm_frac": {k: round(v / peak, 4) for k, v in per_gbs.items()},
             "roofline": {"bound": "hbm", "kernel": dom, "achieved": round(achieved, 2), "peak": peak,
                          "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
                          "peak_source": peak_src, "traffic_source": traffic_src,
@@ -373,14 +475,26 @@ def run_ours(args, rank, world, local):
                               "peak": round(fp64_peak, 1), "unit": "G FP64 ops/s", "frac": fp64[dom]["frac"],
                               "peak_source": "measured DFMA issue rate (profiles/r01_pipes2.txt) x 148 SMs x 1.965 GHz",
                               "per_pattern": fp64},
-            "cpu_baseline": cpu, "e2e": e2e, "float64_inputs": f64,
+            "ssim_exact_windows": int(r.get("n_ssim_exact", 0)),
+            "cpu_baseline": cpu, "e2e": e2e, "float64_inputs": f64, "other_configs": others,
             "gpu_launches": launches_per_step * args.steps,
             "clocks": clocks, "wall_s_timed_region": round(t_wall, 4),
         }
         print(json.dumps(line), flush=True)
-    a.close()
     if world > 1:
         dist.destroy_process_group()
+
+
+def np_prod(v):
+    p = 1
+    for d in v:
+        p *= int(d)
+    return p
+
+
+def default_planes(spec):
+    """Planes of the bounded oracle sample: ~10-30 s of CPU work on the box's cores."""
+    return min(spec.dims[0], {"C5": 16, "C3": 24}.get(spec.name.split("-")[0], 25))
 
 
 def czc_nccl_uid() -> bytes:

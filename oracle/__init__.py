@@ -78,8 +78,10 @@ def _load():
         DP = ctypes.POINTER(ctypes.c_double)
         UP = ctypes.POINTER(ctypes.c_uint64)
         lib.czco_pdf.argtypes = [P, P, ctypes.c_uint64, ctypes.c_int, DP, DP, UP, DP, DP, UP, UP]
+        lib.czco_ssim_windows.argtypes = [P, P, ctypes.c_int, I64P, I64P, I64P, ctypes.c_int, P]
         lib.czco_threads.restype = ctypes.c_int
-        for name in ("czco_p1", "czco_deriv", "czco_autocorr", "czco_ssim_window", "czco_ssim", "czco_pdf"):
+        for name in ("czco_p1", "czco_deriv", "czco_autocorr", "czco_ssim_window", "czco_ssim", "czco_pdf",
+                     "czco_ssim_windows"):
             f32, f64 = getattr(lib, name), getattr(lib, name + "_f64")
             f64.argtypes = f32.argtypes
             f64.restype = f32.restype
@@ -175,6 +177,24 @@ def ssim(x, y, window, step=None, range_mode: int = 0, dims=None):
     if rc:
         raise ValueError(f"czco_ssim failed ({rc})")
     return out.value, int(nw.value)
+
+
+def ssim_windows(x, y, window, step=None, range_mode: int = 0, dims=None) -> np.ndarray:
+    """Local SSIM of every valid window (czco_ssim_windows), shaped like the window-origin grid
+    (one value per origin, slowest axis first); its mean is ssim()."""
+    x, y = _pair(x, y)
+    nd, d = _dims(x, dims)
+    shp = tuple(x.shape) if dims is None else tuple(int(v) for v in dims)
+    if step is None:
+        step = [1] * nd
+    nw = [((n - w) // s + 1) if (n > 1 and w <= n) else (1 if n == 1 else 0)
+          for n, w, s in zip(shp, window, step)]
+    out = np.empty(int(np.prod(nw)), dtype=np.float64)
+    rc = _fn("czco_ssim_windows", x)(x.ctypes.data, y.ctypes.data, nd, d, _i64(window), _i64(step), range_mode,
+                                     out.ctypes.data)
+    if rc:
+        raise ValueError(f"czco_ssim_windows failed ({rc})")
+    return out.reshape(nw)
 
 
 def pdf(x, y, nbins: int = 100) -> Dict:

@@ -29,6 +29,7 @@ int czco_threads(void) {
 /* Shapes: ndim 1..4 (4-D is NEXT row f3), right-aligned into NA = 4 axes with leading 1s (an
  * axis of extent 1 is inactive).  Returns 0 if invalid. */
 #define NA 4
+#define CZCO_P1_CHUNK 65536   /* P1: fixed element chunks, combined in chunk order */
 static int shape4(int ndim, const int64_t* dims, int64_t n[NA]) {
   if (ndim < 1 || ndim > NA || !dims) return 0;
   for (int a = 0; a < NA; a++) n[a] = 1;

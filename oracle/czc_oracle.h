@@ -62,6 +62,13 @@ double czco_ssim_window(const float* x, const float* y, int ndim, const int64_t*
 int czco_ssim(const float* x, const float* y, int ndim, const int64_t* dims, const int64_t* window,
               const int64_t* step, int range_mode, double* ssim, uint64_t* n_windows);
 
+/* Local SSIM of every valid window, C order of the window-origin grid (out: n_windows doubles);
+ * returns 3 when there is no valid window. */
+int czco_ssim_windows(const float* x, const float* y, int ndim, const int64_t* dims, const int64_t* window,
+                      const int64_t* step, int range_mode, double* out);
+int czco_ssim_windows_f64(const double* x, const double* y, int ndim, const int64_t* dims, const int64_t* window,
+                          const int64_t* step, int range_mode, double* out);
+
 /* Error PDF and pwr-error PDF (Table I Category I, L107: "Error PDF", "Pwr error PDF"; the paper
  * gives no bin rule — reading R24): nbins equal-width bins over [min, max] of the
  * values (the error e = y - x over all n elements; |e|/|x| over x != 0), bin of v =

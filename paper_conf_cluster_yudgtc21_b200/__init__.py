@@ -247,6 +247,7 @@ class Assessor:
         dev = torch.cuda.current_device() if device is None else int(device)
         if stream is None:
             stream = torch.cuda.current_stream(dev)
+        self.device = dev
         self.stream = stream
         self.cfg = make_config(ndim=ndim, device=dev, stream=stream.cuda_stream, **cfg)
         self.ctx = czc_init(self.cfg)
@@ -263,6 +264,9 @@ class Assessor:
             raise TypeError("orig and recon must have the same dtype")
         if orig.shape != recon.shape:
             raise ValueError("orig and recon must have the same shape")
+        for t in (orig, recon):               # kernels of this context run on self.device only
+            if t.device.index != self.device:
+                raise ValueError(f"tensor on cuda:{t.device.index}, context bound to cuda:{self.device}")
         gdims = list(orig.shape) if dims is None else list(dims)
         shape = make_shape(gdims, z0, orig.shape[0] if dims is not None else 0)
         return czc_assess(self.ctx, orig.data_ptr(), recon.data_ptr(), shape, mask, dtype=dts[orig.dtype])
@@ -299,5 +303,6 @@ class Assessor:
 
 def assess(orig, recon, mask: int = M_ALL, **cfg) -> Dict:
     """One-shot assessment of two CUDA float32 / float64 tensors (creates and frees a context)."""
+    cfg.setdefault("device", orig.device.index if orig.is_cuda else None)
     with Assessor(ndim=orig.dim(), **cfg) as a:
         return a.assess(orig, recon, mask)

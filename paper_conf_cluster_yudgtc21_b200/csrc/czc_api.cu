@@ -827,11 +827,36 @@ static czc_status assess_dispatch(czc_ctx* ctx, const Plan& P, const E* x, const
   return assess_single(ctx, P, x, y, out, mask);
 }
 
+// The fields must be memory the context's device can read: device memory of that device (or
+// managed / mapped host memory).  Unregistered host memory or another device's allocation would
+// fault inside a kernel and leave a sticky error in the CUDA context, so it is a
+// status code here instead.
+static czc_status check_device_ptr(czc_ctx* ctx, const void* p, const char* what) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    (void)cudaGetLastError();
+    ctx->last_error = std::string(what) + ": not a CUDA-accessible pointer";
+    return CZC_ERR_INVALID;
+  }
+  if (a.type == cudaMemoryTypeUnregistered) {
+    ctx->last_error = std::string(what) + ": host memory (czc_assess takes device pointers; see czc_assess_host)";
+    return CZC_ERR_INVALID;
+  }
+  if (a.type == cudaMemoryTypeDevice && a.device != ctx->device) {
+    ctx->last_error = std::string(what) + ": memory of device " + std::to_string(a.device) +
+                      ", context bound to device " + std::to_string(ctx->device);
+    return CZC_ERR_INVALID;
+  }
+  return CZC_OK;
+}
+
 extern "C" czc_status czc_assess(czc_ctx* ctx, const void* orig, const void* recon, const czc_shape* shape,
                                  czc_dtype dtype, uint64_t metric_mask, czc_result* out) {
   czc_status st = check_common(ctx, orig, recon, shape, dtype, out);
   if (st != CZC_OK) return st;
   if (cudaSetDevice(ctx->device) != cudaSuccess) return cuda_fail(ctx, cudaGetLastError(), "cudaSetDevice");
+  if ((st = check_device_ptr(ctx, orig, "orig")) != CZC_OK || (st = check_device_ptr(ctx, recon, "recon")) != CZC_OK)
+    return st;
   Plan P;
   st = make_plan(ctx->cfg, shape->ndim, shape->dims, metric_mask, P, ctx->last_error);
   if (st == CZC_OK) {

@@ -1,4 +1,4 @@
-// p3_ssim.cu — Pattern 3: sliding-window SSIM.
+// p3_ssim.cu — Pattern 3: sliding-window SSIM with a certified fast path.
 //
 // Paper (L139-L146, Fig. 5, Alg. 3): a w^3 window slides with a fixed step over both
 // fields; at each position the window's min, max, sum and power sums are reduced, "mixed (by some
@@ -10,27 +10,43 @@
 // B200 design.  A block = 8 warps owns a tile of (32 - WX + 1) x (8 G) window
 // origins and a chunk of origin planes, and streams z.  Lane l of warp w owns the footprint
 // columns (rows w, w+8, ...; column l) of the tile and, per plane:
-//   (a) z-walk — keeps FP64 running sums over the last WZ planes of four anchored moments
+//   (a) z-walk — FP64 sums over the last WZ planes of four anchored moments
 //         a = x - K,  e = y - x,  a*b (b = y - K),  e*e
-//       in registers; the leaving plane's x sits in a per-thread register ring (the paper's
-//       FIFO, moved from window partials to raw samples; a shifting ring, so the plane loop
-//       needs no unrolling), which also gives the z-window min/max of x, and its
-//       y is re-read from L2; the next plane is prefetched into registers one plane ahead;
+//       kept in registers: between resyncs the sums slide (add the entering plane, subtract the
+//       leaving one), and every WZ planes they are re-summed from scratch over the window's own
+//       planes, so no rounding error lives longer than 2 WZ - 1 planes (a large value
+//       passing through a running sum would otherwise pollute every later window of the column).
+//       The x of the last WZ planes sits in a shifting register ring (the paper's FIFO, moved
+//       from window partials to raw samples), which also gives the z-window min/max of x; the
+//       y of the leaving plane (and of the ring planes at a resync) is re-read from L2.  The
+//       walk also tracks V = max(|a|, |e|) over the planes its sums have touched since the last
+//       resync (the error magnitude of the certificate below);
 //   (b) y-pass — after ONE __syncthreads on a double-buffered shared-memory exchange of the
 //       z-sums, each warp forms running sums over WY rows for its G origin rows;
 //   (c) x-pass — power-of-two doubling with warp shuffles across the 32 lanes (the paper's
 //       shfl_down x-reduction, L270), then the per-window mix in the cancellation-free form
 //         ssim = A/(A + mu_e^2) * B/(B + s_e^2),  A = 2 mu_x mu_y + C1,  B = 2 s_xy + C2
 //       (identical to Wang et al.'s formula with C3 = C2/2, reading R14), with L = max - min of
-//       the original window (reading R15) or the global range.
-// K is one anchor per block (the tile-centre sample of its first plane) so the moment sums stay
-// small; every sum is FP64.  Window extents are compile-time (cubic 3-D, square 2-D, 1-D).
+//       the original window (reading R15) or the global range;
+//   (d) certificate — an a-posteriori bound on the window's rounding error from V, |K| and the
+//       two denominators (derivation at ssim_cert below); a window whose bound exceeds
+//       kSsimTau is recomputed exactly (two-pass, anchored at its own first sample) by its warp
+//       and counted in czc_result.n_ssim_exact (local anchors + bound +
+//       exact fallback).
+// K is one anchor per block (tile_anchor: the tile-centre sample of its first plane, or 0 for
+// tiles spanning decades or crossing zero).  Window extents are
+// compile-time (cubic 3-D, square 2-D, 1-D).
 #include "czc_internal.cuh"
 
 namespace czc {
 
 constexpr int kP3Warps = 8;
 constexpr int kP3Threads = 32 * kP3Warps;
+constexpr double kU = 1.1102230246251565e-16;   // unit roundoff of FP64, 2^-53
+// Per-window error budget of the fast path.  The parity tolerance of SSIM is 1e-6 absolute on
+// every window and on the mean (north_star); a window whose certified bound exceeds this is
+// recomputed exactly.
+constexpr double kSsimTau = 2.5e-7;
 
 template <typename T, int WX, int WY, int WZ, int G>
 struct SsimGeom {
@@ -39,13 +55,13 @@ struct SsimGeom {
   static constexpr int FY = TY + WY - 1;                 // footprint rows
   static constexpr int KC = (FY + kP3Warps - 1) / kP3Warps;   // z-walk rows per thread
   static constexpr int ZSTRIDE = FY * 32;                // one component plane of the exchange
-  // exchange buffer: { 4 double comps, 2 min/max comps of the input type } x FY x 32, double-buffered
-  static constexpr size_t buf_bytes = (size_t)ZSTRIDE * (4 * sizeof(double) + 2 * sizeof(T));
+  // exchange buffer: { 4 double comps, 2 min/max comps of the input type, 1 float magnitude }
+  // x FY x 32, double-buffered
+  static constexpr size_t buf_bytes = (size_t)ZSTRIDE * (4 * sizeof(double) + 2 * sizeof(T) + sizeof(float));
   static constexpr size_t smem = 2 * buf_bytes;
 };
 
 __device__ __forceinline__ double shd(double v, int d) { return __shfl_down_sync(0xffffffffu, v, d); }
-__device__ __forceinline__ float shf(float v, int d) { return __shfl_down_sync(0xffffffffu, v, d); }
 
 // Sum over lanes [l, l+W) of v (W compile-time): power-of-two doubling + binary decomposition.
 // Lanes whose window leaves the warp return garbage (their origins are outside the tile).
@@ -88,6 +104,147 @@ __device__ __forceinline__ T lane_window_ext(T v) {
   return q;
 }
 
+// ---- certificate ---------------------------------------------------------------------------
+// Error model of one fast-path window (M samples, anchor K, u = 2^-53).  Every sample i the
+// window's sums have touched (the window itself, the <= WZ - 1 planes before it since the last
+// resync, and the <= G - 1 rows above it that the running y-sums add and subtract) satisfies
+// |a_i|, |e_i| <= V, hence |b_i| <= 2V, |a_i b_i| <= 2V^2, e_i^2 <= V^2.  A sliding sum never
+// holds more than W + 1 terms, so with T the term bound of a moment the rounding errors are
+//   z-walk: per column <= (WZ - 1) (fresh resync sum) + 2 (WZ - 1) (slide steps) roundings of
+//           partials <= (WZ + 1) T, i.e. <= 3 WZ M T over the window's WY WX columns;
+//   y-pass: <= (WY - 1) + 2 (G - 1) roundings of partials <= (WY + 1) WZ T per x-column;
+//   x-pass: <= 5 doubling levels of partials <= M T;  terms (a, b, e roundings) 3;  1/M: 1;
+// so |d Sum| <= cV u M T with cV = 3 WZ + WY + 2 G + 13 (incl. slack 4).  With the computed
+// means (|true - computed| <= s = 2 cV u V each, incl. their own roundings):
+//   |d(S_ab/M)| <= 2 cV u V^2,  |d(S_ee/M)| <= cV u V^2,  |d mu_a|, |d mu_e| <= cV u V,
+//   |d s_xy| <= 2 cV u V^2 + (|mu_a| + |mu_b|) 2 cV u V + 8 u V^2        (mu_b = mu_a + mu_e)
+//   |d s_ee| <= cV u V^2 + 2 |mu_e| cV u V + 3 u V^2
+//   |dB| + |d s_ee| <= (5 cV + 19) u V^2 + cV u V q + u D2,   q = 4 (|mu_a| + |mu_b|) + 2 |mu_e| + 10 s
+//   |dA| <= 6 cV u m V + 10 u m^2,  |d mu_e^2| <= 2 cV u V (|mu_e| + s) + (cV u V)^2,
+//                                                              m = |mu_x| + |mu_y| + 2 s,
+// where D1 = A + mu_e^2 = mu_x^2 + mu_y^2 + C1 and D2 = B + s_ee = s_x^2 + s_y^2 + C2.  Since
+// |A| <= D1, mu_e^2 <= 2 D1, |B| <= D2 and s_ee <= 2 D2, each factor of the two-factor form moves
+// by at most 2 (|dA| + |d mu_e^2|) / D1 resp. 2 (|dB| + |d s_ee|) / D2, and the mix adds ~10 u:
+//   |d ssim| <= n2 / D2 + n1 / D1 + 14 u,
+//   n2 = 2 [(5 cV + 19) u V^2 + cV u V q],
+//   n1 = 2 [6 cV u m V + 10 u m^2 + 2 cV u V (|mu_e| + s) + (cV u V)^2].
+// The window is certified when this is <= kSsimTau (cross-multiplied, no division; NaN / inf /
+// non-positive denominators fail the test and take the exact path).  Using the computed means
+// (not their worst case |K| + 2V) keeps windows near zero (QCLOUD-like fields) certified.
+struct SsimCert {
+  double cvu, ka, kc, tau;
+};
+__host__ __device__ constexpr SsimCert ssim_cert(double cV) {
+  return SsimCert{cV * kU, 2.0 * kU * (5.0 * cV + 19.0), 20.0 * kU, kSsimTau - 14.0 * kU};
+}
+// Vf: float magnitude bound (rounded to nearest from the true value: bumped by 2^-22).
+__device__ __forceinline__ bool ssim_certified(const SsimCert& c, float Vf, double mua, double mue, double mux,
+                                               double muy, double D1, double D2) {
+  const double V = (double)Vf * (1.0 + 0x1p-22);
+  const double cuV = c.cvu * V, s = 2.0 * cuV;
+  const double q = fma(4.0, fabs(mua) + fabs(mua + mue), fma(2.0, fabs(mue), 10.0 * s));
+  const double m = fabs(mux) + fabs(muy) + 2.0 * s;
+  const double n2 = fma(c.ka * V, V, 2.0 * cuV * q);
+  const double n1 = 2.0 * fma(6.0 * cuV, m, fma(2.0 * cuV, fabs(mue) + s, cuV * cuV)) + c.kc * m * m;
+  return D1 > 0.0 && D2 > 0.0 && fma(n2, D1, n1 * D2) <= c.tau * D1 * D2;
+}
+
+// The sample magnitude tracked for the certificate: max(|x - K|, |y - x|), as a float that is
+// within one float rounding of the true value (ssim_certified bumps it).
+__device__ __forceinline__ float sample_mag(float xs, float ys, float K32, double, double) {
+  return fmaxf(fabsf(xs - K32), fabsf(ys - xs));
+}
+__device__ __forceinline__ float sample_mag(double, double, float, double a, double e) {
+  return fmaxf((float)fabs(a), (float)fabs(e));
+}
+
+// Butterfly all-reduce over the 32 lanes (every lane gets the same value: IEEE addition, min
+// and max are commutative).
+__device__ __forceinline__ double warp_allsum(double v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+__device__ __forceinline__ double warp_allmin(double v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fmin(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+__device__ __forceinline__ double warp_allmax(double v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fmax(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
+// Anchor of a tile: the certificate's magnitude V = max |x - K| over the samples a window's sums
+// touch, so K should sit near every window's values.  The tile-centre sample does for fields that
+// vary little across a tile (temperature-like); for fields spanning decades or crossing zero
+// (log-normal densities, QCLOUD-like zeros + clouds) K = 0 keeps |x - K| ~ |x|, which scales with
+// the local range L of such fields.  mn / mx: extrema of the tile's first-plane footprint.
+template <typename T>
+__device__ __forceinline__ T tile_anchor(T centre, T mn, T mx) {
+  const bool decades = (mn >= (T)0 && mn < (T)0.25 * mx) || (mx <= (T)0 && mx > (T)0.25 * mn);
+  const bool crosses = mn < (T)0 && mx > (T)0;
+  return (decades || crosses) ? (T)0 : centre;
+}
+template <typename T>
+__device__ __forceinline__ T warp_min_t(T v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = tmin(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+template <typename T>
+__device__ __forceinline__ T warp_max_t(T v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = tmax(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
+// Exact local SSIM of the window with origin (oz, oy, ox) and extents (wz, wy, wx), computed by
+// the whole warp (all lanes must call it with the same arguments; all return the same value):
+// the plain definition of L139 / reading R14-R15 — two passes, means about the window's own first
+// sample, then centred second moments (no cancellation), FP64 throughout.  The fallback of the
+// certified fast path (called only for windows whose bound failed).
+template <typename T>
+__device__ __forceinline__ double ssim_exact_window(const Field3<T> f, int64_t oz, int64_t oy, int64_t ox, int wz, int wy,
+                                                 int wx, bool range_global, double Lglob) {
+  const int lane = threadIdx.x & 31;
+  const int M = wz * wy * wx;
+  const int64_t nx = f.nx;
+  const double x0 = (double)f.xp(oz)[oy * nx + ox];
+  double sx = 0, sy = 0, mn = x0, mx = x0;
+  for (int i = lane; i < M; i += 32) {
+    const int ix = i % wx, r = i / wx, iy = r % wy, iz = r / wy;
+    const int64_t o = (oy + iy) * nx + ox + ix;
+    const double xv = (double)f.xp(oz + iz)[o], yv = (double)f.yp(oz + iz)[o];
+    sx += xv - x0;
+    sy += yv - x0;
+    mn = fmin(mn, xv);
+    mx = fmax(mx, xv);
+  }
+  sx = warp_allsum(sx);
+  sy = warp_allsum(sy);
+  mn = warp_allmin(mn);
+  mx = warp_allmax(mx);
+  const double mux = x0 + sx / (double)M, muy = x0 + sy / (double)M;
+  double vx = 0, vy = 0, cxy = 0;
+  for (int i = lane; i < M; i += 32) {
+    const int ix = i % wx, r = i / wx, iy = r % wy, iz = r / wy;
+    const int64_t o = (oy + iy) * nx + ox + ix;
+    const double dx = (double)f.xp(oz + iz)[o] - mux, dy = (double)f.yp(oz + iz)[o] - muy;
+    vx = fma(dx, dx, vx);
+    vy = fma(dy, dy, vy);
+    cxy = fma(dx, dy, cxy);
+  }
+  vx = warp_allsum(vx) / (double)M;
+  vy = warp_allsum(vy) / (double)M;
+  cxy = warp_allsum(cxy) / (double)M;
+  double L = range_global ? Lglob : mx - mn;
+  L = (L == 0.0) ? 1.0 : L;
+  const double C1 = (0.01 * L) * (0.01 * L), C2 = (0.03 * L) * (0.03 * L);
+  return ((2.0 * mux * muy + C1) * (2.0 * cxy + C2)) / ((mux * mux + muy * muy + C1) * (vx + vy + C2));
+}
+
 // T = float: the x ring and the exchanged extrema are floats (exact); T = double: doubles, one
 // block per SM for the larger register ring.
 template <typename T, int WX, int WY, int WZ, int G>
@@ -97,6 +254,7 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
   using Gm = SsimGeom<T, WX, WY, WZ, G>;
   constexpr int TX = Gm::TX, FY = Gm::FY, KC = Gm::KC, ZS = Gm::ZSTRIDE;
   constexpr double invM = 1.0 / (double)(WX * WY * WZ);
+  constexpr SsimCert cert = ssim_cert(3.0 * WZ + WY + 2.0 * G + 13.0);
   extern __shared__ __align__(16) unsigned char smem_raw[];
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -110,7 +268,6 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
   int64_t ky = y0 + FY / 2, kx = x0 + 16;
   if (ky > f.ny - 1) ky = f.ny - 1;
   if (kx > f.nx - 1) kx = f.nx - 1;
-  const double K = (zb < zend) ? (double)f.xp(zb)[ky * f.nx + kx] : 0.0;
   const double Lglob = (double)res->p1g.xmax - (double)res->p1g.xmin;
 
   // In-plane offsets (a plane has < 2^31 elements; the launcher checks).  Footprint rows and
@@ -151,17 +308,37 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
 
   double sm[KC][4];
   T ring[KC][WZ];                                        // x of the last WZ planes
+  float vm[KC];                                          // certificate magnitude of the z-sums
 #pragma unroll
   for (int k = 0; k < KC; k++) {
 #pragma unroll
     for (int m = 0; m < 4; m++) sm[k][m] = 0;
 #pragma unroll
     for (int s = 0; s < WZ; s++) ring[k][s] = 0;
+    vm[k] = 0.f;
   }
   load(0, false);
+  // the block's anchor (tile_anchor) from the first plane's footprint: one barrier
+  T Kt = (T)0;
+  {
+    __shared__ T s_ext[2][kP3Warps];
+    T mn = nxt[0].x, mx = nxt[0].x;
+#pragma unroll
+    for (int k = 1; k < KC; k++)
+      if (row_live(k)) { mn = tmin(mn, nxt[k].x); mx = tmax(mx, nxt[k].x); }
+    mn = warp_min_t(mn);
+    mx = warp_max_t(mx);
+    if (lane == 0) { s_ext[0][warp] = mn; s_ext[1][warp] = mx; }
+    __syncthreads();
+#pragma unroll
+    for (int w = 0; w < kP3Warps; w++) { mn = tmin(mn, s_ext[0][w]); mx = tmax(mx, s_ext[1][w]); }
+    if (nsteps > 0) Kt = tile_anchor<T>(f.xp(zb)[ky * f.nx + kx], mn, mx);
+  }
+  const double K = (double)Kt;
+  const float K32 = (float)Kt;
 
   double ssum = 0;
-  unsigned scnt = 0;
+  unsigned scnt = 0, nexact = 0;
   const bool range_global = p.range_mode != 0;
   // origin-grid membership: x and y are fixed per thread, z advances one plane per step
   const int64_t gxl = x0 + lane;
@@ -174,34 +351,59 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
   }
   int zph = (int)(zb % p.sz);                            // phase of origin plane zb
 
+  // moments of one sample into s (sign +1: entering, -1: leaving)
+  auto add_sample = [&](double (&s)[4], const T xs, const T ys, float& v) {
+    const double xd = xs, yd = ys;
+    const double a = xd - K, b = yd - K, e = yd - xd;
+    s[0] += a; s[1] += e; s[2] = fma(a, b, s[2]); s[3] = fma(e, e, s[3]);
+    v = fmaxf(v, sample_mag(xs, ys, K32, a, e));
+  };
+  auto sub_sample = [&](double (&s)[4], const T xs, const T ys) {
+    const double xd = xs, yd = ys;
+    const double a = xd - K, b = yd - K, e = yd - xd;
+    s[0] -= a; s[1] -= e; s[2] = fma(-a, b, s[2]); s[3] = fma(-e, e, s[3]);
+  };
+
   // One plane step; warm = (step >= WZ: a plane leaves the z-window) and, in the warm-up, s =
   // step are compile-time constants at every call site, so the warm-up planes carry no per-step
-  // tests.
-  auto step_body = [&](const int step, const int s, const bool warm) {
+  // tests.  resync (block-uniform): re-sum the z-window from scratch instead of sliding.
+  auto step_body = [&](const int step, const int s, const bool warm, const bool resync) {
     // the prefetched plane is consumed by the z-walk below, then the next one is requested
     // into the same registers (no copies; its latency hides behind the y / x passes)
     const int buf = step & 1;
     double* Zd = reinterpret_cast<double*>(smem_raw + buf * Gm::buf_bytes);
     T* Zm = reinterpret_cast<T*>(Zd + 4 * ZS);
+    float* Zv = reinterpret_cast<float*>(Zm + 2 * ZS);
     const bool full = warm || s == WZ - 1;               // a complete z-window ends here
     // ---- (a) z-walk --------------------------------------------------------------------
+    if (resync) {
+      // window planes zb+step-WZ+1 .. zb+step: ring slots 1..WZ-1 (x) with their y re-read,
+      // plus the entering plane; V restarts from the window's own samples
+#pragma unroll
+      for (int k = 0; k < KC; k++) {
+        if (!row_live(k)) continue;
+#pragma unroll
+        for (int m = 0; m < 4; m++) sm[k][m] = 0;
+        vm[k] = 0.f;
+      }
+#pragma unroll
+      for (int t = 1; t < WZ; t++) {
+        const T* yr = f.yp(zb + step - WZ + t);
+#pragma unroll
+        for (int k = 0; k < KC; k++) {
+          if (!row_live(k)) continue;
+          add_sample(sm[k], ring[k][t], __ldg(yr + off[k]), vm[k]);
+        }
+      }
+    }
 #pragma unroll
     for (int k = 0; k < KC; k++) {
       if (!row_live(k)) continue;
-      {
-        const double xd = nxt[k].x, yd = nxt[k].y;
-        const double a = xd - K, b = yd - K, e = yd - xd;
-        sm[k][0] += a; sm[k][1] += e; sm[k][2] = fma(a, b, sm[k][2]); sm[k][3] = fma(e, e, sm[k][3]);
-      }
-      if (warm) {
-        const double xd = ring[k][0], yd = nyo[k];
-        const double a = xd - K, b = yd - K, e = yd - xd;
-        sm[k][0] -= a; sm[k][1] -= e; sm[k][2] = fma(-a, b, sm[k][2]); sm[k][3] = fma(-e, e, sm[k][3]);
-      }
+      add_sample(sm[k], nxt[k].x, nxt[k].y, vm[k]);
+      if (warm && !resync) sub_sample(sm[k], ring[k][0], nyo[k]);
       // shifting ring (oldest plane first; WZ - 1 register moves per row): the main loop is not
-      // unrolled, so one copy of the step (~4.4 K instructions for the kernel instead of 10.3 K
-      // with a static-slot ring unrolled by WZ) stays in the instruction cache — the
-      // `no_instruction` stalls of the unrolled version cost more than the moves (0.475 -> 0.445 ms)
+      // unrolled, so one copy of the step stays in the instruction cache (the `no_instruction`
+      // stalls of an unrolled static-slot ring cost more than the moves: 0.475 -> 0.445 ms)
 #pragma unroll
       for (int t = 0; t + 1 < WZ; t++) ring[k][t] = ring[k][t + 1];
       ring[k][WZ - 1] = nxt[k].x;
@@ -215,6 +417,7 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
         for (int m = 0; m < 4; m++) Zd[m * ZS + c] = sm[k][m];
         Zm[c] = mn;
         Zm[ZS + c] = mx;
+        Zv[c] = vm[k];
       }
     }
     load(step + 1, warm || s == WZ - 1);
@@ -225,6 +428,7 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
     // ---- (b) y-pass: the G origin rows of this warp (running sums over WY rows) ------------
     double h[G][4];
     T hmn[G], hmx[G];
+    float hv;                                            // V over the union of the G windows' rows
     {
       // y-window min/max: the WY - G + 1 rows shared by all G windows are reduced once
       T cmn = Zm[(warp * G + G - 1) * 32 + lane], cmx = Zm[ZS + (warp * G + G - 1) * 32 + lane];
@@ -233,6 +437,9 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
         cmn = tmin(cmn, Zm[(warp * G + i) * 32 + lane]);
         cmx = tmax(cmx, Zm[ZS + (warp * G + i) * 32 + lane]);
       }
+      hv = Zv[(warp * G) * 32 + lane];
+#pragma unroll
+      for (int i = 1; i < G + WY - 1; i++) hv = fmaxf(hv, Zv[(warp * G + i) * 32 + lane]);
 #pragma unroll
       for (int g = 0; g < G; g++) {
         const int oy = warp * G + g;
@@ -272,6 +479,9 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
       wmn[g] = lane_window_ext<WX, false>(hmn[g]);
       wmx[g] = lane_window_ext<WX, true>(hmx[g]);
     }
+    const float wv = lane_window_ext<WX, true>(hv);
+    double ss[G];
+    unsigned long long fl = 0;                           // bit 32 g + lane: window failed its bound
 #pragma unroll
     for (int g = 0; g < G; g++) {
       const bool ok = zok && gok[g];
@@ -284,13 +494,34 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
       L = (L == 0.0) ? 1.0 : L;
       const double C1 = (0.01 * L) * (0.01 * L), C2 = (0.03 * L) * (0.03 * L);
       const double A = 2.0 * mux * muy + C1, B = 2.0 * sxy + C2;
-      // A, B, A + mu_e^2, B + s_e^2 > 0 (C1, C2 > 0); |rel err of the reciprocal| <= 2u
-      const double ssim = (A * B) * fast_rcp((A + mue * mue) * (B + see));
-      ssum += ok ? ssim : 0.0;
+      const double D1 = A + mue * mue, D2 = B + see;
+      // A, B, D1, D2 > 0 (C1, C2 > 0) up to the certified error; |rel err of the reciprocal| <= 2u
+      ss[g] = (A * B) * fast_rcp(D1 * D2);
+      // ---- (d) certificate ------------------------------------------------------------------
+      const bool flag = ok && !ssim_certified(cert, wv, mua, mue, mux, muy, D1, D2);
+      fl |= (unsigned long long)__ballot_sync(0xffffffffu, flag) << (32 * g);
+    }
+    // failed windows are recomputed exactly by the whole warp (warp-uniform loop, rare)
+    while (fl) {
+      const int bit = __ffsll((long long)fl) - 1, g = bit >> 5, l = bit & 31;
+      fl &= fl - 1;
+      const double v = ssim_exact_window<T>(f, zb + step - WZ + 1, y0 + warp * G + g, x0 + l, WZ, WY, WX,
+                                            range_global, Lglob);
+      if (lane == l) {
+#pragma unroll
+        for (int q = 0; q < G; q++)
+          if (q == g) ss[q] = v;
+        nexact++;
+      }
+    }
+#pragma unroll
+    for (int g = 0; g < G; g++) {
+      const bool ok = zok && gok[g];
+      ssum += ok ? ss[g] : 0.0;
       scnt += ok ? 1u : 0u;
       if (dbg && ok) {
         const int64_t oz = zb + step - WZ + 1, gy = y0 + warp * G + g;
-        dbg[((oz / p.sz) * p.nwy + gy / p.sy) * p.nwx + (x0 + lane) / p.sx] = ssim;
+        dbg[((oz / p.sz) * p.nwy + gy / p.sy) * p.nwx + (x0 + lane) / p.sx] = ss[g];
       }
     }
   };
@@ -299,12 +530,17 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
 #pragma unroll
   for (int s = 0; s < WZ; s++) {
     if (s >= nsteps) break;                              // block-uniform
-    step_body(s, s, false);
+    step_body(s, s, false, false);
   }
+  // steady state: a resync every WZ planes (step = WZ, 2 WZ, ...)
+  int rph = 0;
 #pragma unroll 1
-  for (int step = WZ; step < nsteps; step++) step_body(step, 0, true);
+  for (int step = WZ; step < nsteps; step++) {
+    step_body(step, 0, true, rph == 0);
+    rph = rph + 1 == WZ ? 0 : rph + 1;
+  }
 
-  double rec[kSsimSlots] = {ssum, (double)scnt, 0.0};
+  double rec[kSsimSlots] = {ssum, (double)scnt, (double)nexact};
   const unsigned bid = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
   struct Sum { __device__ int operator()(int) const { return OP_SUM; } };
   __syncthreads();
@@ -359,12 +595,13 @@ static cudaError_t launch_t(const Field3<T>& f, const SsimParams& p, double* par
 
 // ------------------------------------------------------------------------------------------------
 // 2-D fields (square W x W windows): the rows stream like the planes of the 3-D kernel, and the
-// y-window is the running sum of that stream, so no shared-memory exchange and no barrier are
-// needed: warp w of a block owns its own tile of 32 - W + 1 x-origins (lane = footprint column),
-// keeps FP64 running sums of the four anchored moments over the last W rows plus the rows' x in
-// a shifting register ring (warm-up peeled), re-reads the leaving row's y from L2, and
-// per row does the x-pass by shuffles and the mix.  (The 3-D kernel on a one-plane field ran one
-// plane per block: 0.29 ms for the 1800 x 3600 CESM-shaped pair.)
+// y-window is the running sum of that stream (re-summed from scratch every W rows, as the 3-D
+// z-walk), so no shared-memory exchange and no barrier are needed: warp w of a block owns its own
+// tile of 32 - W + 1 x-origins (lane = footprint column), keeps FP64 sums of the four anchored
+// moments over the last W rows plus the rows' x in a shifting register ring (warm-up peeled),
+// re-reads the leaving row's y from L2, and per row does the x-pass by shuffles, the mix and the
+// certificate (exact recompute of failed windows by the warp).  (The 3-D kernel on a one-plane
+// field ran one plane per block: 0.29 ms for the 1800 x 3600 CESM-shaped pair.)
 constexpr int kRowWarps = 8;
 template <typename T, int W>
 __global__ void __launch_bounds__(kRowWarps * 32)
@@ -372,6 +609,7 @@ p3_rows_kernel(Field3<T> f, SsimParams p, int rchunk, double* __restrict__ parts
                unsigned int* __restrict__ ticket, double* __restrict__ dbg) {
   constexpr int TX = 32 - W + 1;
   constexpr double invM = 1.0 / (double)(W * W);
+  constexpr SsimCert cert = ssim_cert(3.0 * W + 1.0 + 2.0 + 13.0);
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int64_t ny = f.ny, nx = f.nx;
   const T* __restrict__ X = f.xp(0);
@@ -383,7 +621,11 @@ p3_rows_kernel(Field3<T> f, SsimParams p, int rchunk, double* __restrict__ parts
   if (ro_end > ny - W + 1) ro_end = ny - W + 1;
   const int nsteps = ro_end > rb ? (int)(ro_end + W - 1 - rb) : 0;
   const int64_t kx = x0 + 16 < nx ? x0 + 16 : nx - 1, ky = rb + W / 2 < ny ? rb + W / 2 : ny - 1;
-  const double K = (double)X[ky * nx + kx];                     // anchor of this warp's tile
+  // anchor of this warp's tile (tile_anchor) from its first row
+  const T fr = X[rb * nx + gxc];
+  const T Kt = tile_anchor<T>(X[ky * nx + kx], warp_min_t(fr), warp_max_t(fr));
+  const double K = (double)Kt;
+  const float K32 = (float)Kt;
   const double Lglob = res->p1g.xmax - res->p1g.xmin;
   const bool range_global = p.range_mode != 0;
   const bool xok = lane < TX && gx <= nx - W && (gx % p.sx) == 0;
@@ -397,25 +639,35 @@ p3_rows_kernel(Field3<T> f, SsimParams p, int rchunk, double* __restrict__ parts
       if (has_old) { nyo = __ldg(pyo); pyo += nx; }
     }
   };
-  double sm0 = 0, sm1 = 0, sm2 = 0, sm3 = 0;
+  double sm[4] = {0, 0, 0, 0};
+  float vm = 0.f;
   T ring[W];
 #pragma unroll
   for (int t = 0; t < W; t++) ring[t] = 0;
   double ssum = 0;
-  unsigned scnt = 0;
+  unsigned scnt = 0, nexact = 0;
   int rph = (int)(rb % p.sy);
+  auto add_sample = [&](const T xs, const T ys) {
+    const double xd = xs, yd = ys;
+    const double a = xd - K, b = yd - K, e = yd - xd;
+    sm[0] += a; sm[1] += e; sm[2] = fma(a, b, sm[2]); sm[3] = fma(e, e, sm[3]);
+    vm = fmaxf(vm, sample_mag(xs, ys, K32, a, e));
+  };
   load(0, false);
-  auto step_body = [&](const int step, const int s, const bool warm) {
+  auto step_body = [&](const int step, const int s, const bool warm, const bool resync) {
     const bool full = warm || s == W - 1;
-    {
-      const double xd = nx_, yd = ny_;
-      const double a = xd - K, b = yd - K, e = yd - xd;
-      sm0 += a; sm1 += e; sm2 = fma(a, b, sm2); sm3 = fma(e, e, sm3);
+    if (resync) {                                               // rows rb+step-W+1 .. rb+step
+      sm[0] = sm[1] = sm[2] = sm[3] = 0;
+      vm = 0.f;
+      const T* yr = Y + (rb + step - W + 1) * nx + gxc;
+#pragma unroll
+      for (int t = 1; t < W; t++, yr += nx) add_sample(ring[t], __ldg(yr));
     }
-    if (warm) {
+    add_sample(nx_, ny_);
+    if (warm && !resync) {
       const double xd = ring[0], yd = nyo;
       const double a = xd - K, b = yd - K, e = yd - xd;
-      sm0 -= a; sm1 -= e; sm2 = fma(-a, b, sm2); sm3 = fma(-e, e, sm3);
+      sm[0] -= a; sm[1] -= e; sm[2] = fma(-a, b, sm[2]); sm[3] = fma(-e, e, sm[3]);
     }
 #pragma unroll
     for (int t = 0; t + 1 < W; t++) ring[t] = ring[t + 1];     // shifting ring, oldest first
@@ -425,9 +677,10 @@ p3_rows_kernel(Field3<T> f, SsimParams p, int rchunk, double* __restrict__ parts
     T mn = ring[0], mx = ring[0];
 #pragma unroll
     for (int t = 1; t < W; t++) { mn = tmin(mn, ring[t]); mx = tmax(mx, ring[t]); }
-    const double S0 = lane_window_sum<W>(sm0), S1 = lane_window_sum<W>(sm1);
-    const double S2 = lane_window_sum<W>(sm2), S3 = lane_window_sum<W>(sm3);
+    const double S0 = lane_window_sum<W>(sm[0]), S1 = lane_window_sum<W>(sm[1]);
+    const double S2 = lane_window_sum<W>(sm[2]), S3 = lane_window_sum<W>(sm[3]);
     const T wmn = lane_window_ext<W, false>(mn), wmx = lane_window_ext<W, true>(mx);
+    const float wv = lane_window_ext<W, true>(vm);
     const bool ok = xok && rph == 0;                            // origin row rb + step - W + 1
     rph = rph + 1 == p.sy ? 0 : rph + 1;
     const double mua = S0 * invM, mue = S1 * invM;
@@ -438,7 +691,16 @@ p3_rows_kernel(Field3<T> f, SsimParams p, int rchunk, double* __restrict__ parts
     L = (L == 0.0) ? 1.0 : L;
     const double C1 = (0.01 * L) * (0.01 * L), C2 = (0.03 * L) * (0.03 * L);
     const double A = 2.0 * mux * muy + C1, B = 2.0 * sxy + C2;
-    const double ssim = (A * B) * fast_rcp((A + mue * mue) * (B + see));
+    const double D1 = A + mue * mue, D2 = B + see;
+    double ssim = (A * B) * fast_rcp(D1 * D2);
+    const bool flag = ok && !ssim_certified(cert, wv, mua, mue, mux, muy, D1, D2);
+    unsigned fl = __ballot_sync(0xffffffffu, flag);
+    while (fl) {
+      const int l = __ffs(fl) - 1;
+      fl &= fl - 1;
+      const double v = ssim_exact_window<T>(f, 0, rb + step - W + 1, x0 + l, 1, W, W, range_global, Lglob);
+      if (lane == l) { ssim = v; nexact++; }
+    }
     ssum += ok ? ssim : 0.0;
     scnt += ok ? 1u : 0u;
     if (dbg && ok) dbg[((rb + step - W + 1) / p.sy) * p.nwx + gx / p.sx] = ssim;
@@ -446,11 +708,15 @@ p3_rows_kernel(Field3<T> f, SsimParams p, int rchunk, double* __restrict__ parts
 #pragma unroll
   for (int s = 0; s < W; s++) {
     if (s >= nsteps) break;                                     // block-uniform
-    step_body(s, s, false);
+    step_body(s, s, false, false);
   }
+  int qph = 0;
 #pragma unroll 1
-  for (int step = W; step < nsteps; step++) step_body(step, 0, true);
-  double rec[kSsimSlots] = {ssum, (double)scnt, 0.0};
+  for (int step = W; step < nsteps; step++) {
+    step_body(step, 0, true, qph == 0);
+    qph = qph + 1 == W ? 0 : qph + 1;
+  }
+  double rec[kSsimSlots] = {ssum, (double)scnt, (double)nexact};
   struct Sum { __device__ int operator()(int) const { return OP_SUM; } };
   const unsigned bid = blockIdx.x + gridDim.x * blockIdx.y;
   block_reduce_slots<kSsimSlots>(rec, Sum{}, parts + (size_t)bid * kSsimSlots);

@@ -137,10 +137,11 @@ struct Ssim4Params {
   int range_mode;
 };
 
-// Local SSIM of every window of the grid, one window per thread step: FP64 sums of the moments
-// a = x - K, e = y - x, a (y - K), e^2 anchored at the window's first original sample K (the
-// cancellation is bounded by the window's own range), exact min / max of x, then the mix of the
-// 3-D engine (cancellation-free two-factor form, reading R14 / R15).
+// Local SSIM of every window of the grid, one window per thread step, by the plain definition
+// (L139, readings R14-R15): two passes over the window's w0 w1 w2 w3 samples — FP64 means about
+// the window's own first sample, exact min / max of x, then centred second moments — and the
+// textbook mix.  No running sums, so no rounding error outlives its window (the 3-D engines'
+// certificate is not needed here).
 template <typename T>
 __global__ void __launch_bounds__(kG4Threads)
 ssim4_kernel(Field4<T> s, Ssim4Params p, double* __restrict__ parts, DevResults* __restrict__ res,
@@ -154,7 +155,7 @@ ssim4_kernel(Field4<T> s, Ssim4Params p, double* __restrict__ parts, DevResults*
     decode4(i, p.nw, c4);
     const int64_t o = c4[0] * p.s[0] * s.st[0] + c4[1] * p.s[1] * s.st[1] + c4[2] * p.s[2] * s.st[2] + c4[3] * p.s[3];
     const double K = s.x[o];
-    double sa = 0, se = 0, sab = 0, see = 0;
+    double sx = 0, sy = 0;
     T mn = s.x[o], mx = mn;
     for (int l = 0; l < p.w[0]; l++)
       for (int k = 0; k < p.w[1]; k++)
@@ -162,120 +163,35 @@ ssim4_kernel(Field4<T> s, Ssim4Params p, double* __restrict__ parts, DevResults*
           const int64_t r = o + l * s.st[0] + k * s.st[1] + j * s.st[2];
           for (int q = 0; q < p.w[3]; q++) {
             const T xv = __ldg(s.x + r + q), yv = __ldg(s.y + r + q);
-            const double xd = xv, yd = yv;
-            const double a = xd - K, b = yd - K, e = yd - xd;
-            sa += a; se += e; sab = fma(a, b, sab); see = fma(e, e, see);
+            sx += (double)xv - K;
+            sy += (double)yv - K;
             mn = tmin(mn, xv);
             mx = tmax(mx, xv);
           }
         }
-    const double mua = sa * invM, mue = se * invM;
-    const double mux = K + mua, muy = mux + mue;
-    const double sxy = sab * invM - mua * (mua + mue);
-    const double sv = see * invM - mue * mue;
+    const double mux = K + sx * invM, muy = K + sy * invM;
+    double vx = 0, vy = 0, cxy = 0;
+    for (int l = 0; l < p.w[0]; l++)
+      for (int k = 0; k < p.w[1]; k++)
+        for (int j = 0; j < p.w[2]; j++) {
+          const int64_t r = o + l * s.st[0] + k * s.st[1] + j * s.st[2];
+          for (int q = 0; q < p.w[3]; q++) {
+            const double dx = (double)__ldg(s.x + r + q) - mux, dy = (double)__ldg(s.y + r + q) - muy;
+            vx = fma(dx, dx, vx);
+            vy = fma(dy, dy, vy);
+            cxy = fma(dx, dy, cxy);
+          }
+        }
+    vx *= invM;
+    vy *= invM;
+    cxy *= invM;
     double L = p.range_mode ? Lglob : (double)mx - (double)mn;
     L = (L == 0.0) ? 1.0 : L;
     const double C1 = (0.01 * L) * (0.01 * L), C2 = (0.03 * L) * (0.03 * L);
-    const double A = 2.0 * mux * muy + C1, B = 2.0 * sxy + C2;
-    const double ssim = (A * B) / ((A + mue * mue) * (B + sv));
+    const double ssim = ((2.0 * mux * muy + C1) * (2.0 * cxy + C2)) / ((mux * mux + muy * muy + C1) * (vx + vy + C2));
     ssum += ssim;
     scnt += 1.0;
     if (dbg) dbg[i] = ssim;
-  }
-  double rec[kSsimSlots] = {ssum, scnt, 0.0};
-  block_reduce_slots<kSsimSlots>(rec, Sum4Op{}, parts + (size_t)blockIdx.x * kSsimSlots);
-  if (!last_block_arrive(ticket)) return;
-  finish_slots<kSsimSlots>(parts, gridDim.x, Sum4Op{}, res->rec.ssim);
-  if (threadIdx.x == 0) *ticket = 0;
-}
-
-// Step 1 along axis 2 (the common case): a thread takes a run of kRun4 consecutive axis-2
-// origins and slides along that axis — per window one new slab of w0 w1 w3 samples enters and
-// one leaves (recomputed: no per-thread sums ring), instead of w0 w1 w2 w3 samples per window.
-// Adjacent threads take adjacent x-origins (x stays the fastest index), so every load of a warp
-// is coalesced and neighbouring windows share L1 lines.  The slab extrema of the last w2 slabs
-// sit in a per-thread shared-memory ring; the moments are anchored at the run's first sample.
-constexpr int kRun4 = 16;
-constexpr int kRunThreads = 128;                   // the extrema ring: 16 x 128 x 2 x sizeof(T)
-template <typename T>
-__device__ __forceinline__ void slab4(const Field4<T>& s, int64_t base, const int w[4], double K, double& sa,
-                                      double& se, double& sab, double& see, T& mn, T& mx) {
-  sa = se = sab = see = 0;
-  mn = s.x[base];
-  mx = mn;
-  for (int l = 0; l < w[0]; l++)
-    for (int k = 0; k < w[1]; k++) {
-      const int64_t r = base + l * s.st[0] + k * s.st[1];
-      for (int q = 0; q < w[3]; q++) {
-        const T xv = __ldg(s.x + r + q), yv = __ldg(s.y + r + q);
-        const double xd = xv, yd = yv;
-        const double a = xd - K, b = yd - K, e = yd - xd;
-        sa += a; se += e; sab = fma(a, b, sab); see = fma(e, e, see);
-        mn = tmin(mn, xv);
-        mx = tmax(mx, xv);
-      }
-    }
-}
-
-template <typename T>
-__global__ void __launch_bounds__(kRunThreads)
-ssim4_run_kernel(Field4<T> s, Ssim4Params p, double* __restrict__ parts, DevResults* __restrict__ res,
-                 unsigned int* __restrict__ ticket, double* __restrict__ dbg) {
-  __shared__ T ring_mn[16][kRunThreads], ring_mx[16][kRunThreads];   // w2 <= 16 (kMaxWin)
-  const double Lglob = res->p1g.xmax - res->p1g.xmin;
-  const double invM = 1.0 / (double)(p.w[0] * p.w[1] * p.w[2] * p.w[3]);
-  const int w2 = p.w[2];
-  const int64_t nr = (p.nw[2] + kRun4 - 1) / kRun4;             // runs along axis 2
-  const int64_t lenr[4] = {p.nw[0], p.nw[1], nr, p.nw[3]};
-  const int64_t total = lenr[0] * lenr[1] * lenr[2] * lenr[3];
-  const int t = threadIdx.x;
-  double ssum = 0, scnt = 0;
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + t; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    int64_t c4[4];
-    decode4(i, lenr, c4);
-    const int64_t r0 = c4[2] * kRun4;
-    const int64_t r1 = min(r0 + kRun4, p.nw[2]);                // axis-2 origins [r0, r1)
-    const int64_t base = c4[0] * p.s[0] * s.st[0] + c4[1] * p.s[1] * s.st[1] + c4[3] * p.s[3];
-    const double K = s.x[base + r0 * s.st[2]];
-    double Sa = 0, Se = 0, Sab = 0, See = 0;
-    for (int q = 0; q < w2; q++) {                               // the first window's slabs
-      double a, e, ab, ee;
-      T mn, mx;
-      slab4(s, base + (r0 + q) * s.st[2], p.w, K, a, e, ab, ee, mn, mx);
-      Sa += a; Se += e; Sab += ab; See += ee;
-      ring_mn[q][t] = mn;
-      ring_mx[q][t] = mx;
-    }
-    for (int64_t o = r0; o < r1; o++) {
-      if (o > r0) {                                              // slide: slab o+w2-1 in, o-1 out
-        double a, e, ab, ee, ao, eo, abo, eeo;
-        T mn, mx, mno, mxo;
-        slab4(s, base + (o + w2 - 1) * s.st[2], p.w, K, a, e, ab, ee, mn, mx);
-        slab4(s, base + (o - 1) * s.st[2], p.w, K, ao, eo, abo, eeo, mno, mxo);
-        Sa += a - ao; Se += e - eo; Sab += ab - abo; See += ee - eeo;
-        const int slot = (int)((o - r0 + w2 - 1) % 16);
-        ring_mn[slot][t] = mn;
-        ring_mx[slot][t] = mx;
-      }
-      T wmn = ring_mn[(o - r0) % 16][t], wmx = ring_mx[(o - r0) % 16][t];
-      for (int q = 1; q < w2; q++) {
-        const int slot = (int)((o - r0 + q) % 16);
-        wmn = tmin(wmn, ring_mn[slot][t]);
-        wmx = tmax(wmx, ring_mx[slot][t]);
-      }
-      const double mua = Sa * invM, mue = Se * invM;
-      const double mux = K + mua, muy = mux + mue;
-      const double sxy = Sab * invM - mua * (mua + mue);
-      const double sv = See * invM - mue * mue;
-      double L = p.range_mode ? Lglob : (double)wmx - (double)wmn;
-      L = (L == 0.0) ? 1.0 : L;
-      const double C1 = (0.01 * L) * (0.01 * L), C2 = (0.03 * L) * (0.03 * L);
-      const double A = 2.0 * mux * muy + C1, B = 2.0 * sxy + C2;
-      const double ssim = (A * B) / ((A + mue * mue) * (B + sv));
-      ssum += ssim;
-      scnt += 1.0;
-      if (dbg) dbg[((c4[0] * p.nw[1] + c4[1]) * p.nw[2] + o) * p.nw[3] + c4[3]] = ssim;
-    }
   }
   double rec[kSsimSlots] = {ssum, scnt, 0.0};
   block_reduce_slots<kSsimSlots>(rec, Sum4Op{}, parts + (size_t)blockIdx.x * kSsimSlots);
@@ -339,14 +255,7 @@ cudaError_t launch_ssim4(const T* x, const T* y, const int64_t n[4], const int w
     total *= p.nw[a];
   }
   p.range_mode = range_mode;
-  if (p.s[2] == 1 && p.w[2] <= 16) {
-    const int64_t runs = total / p.nw[2] * ((p.nw[2] + kRun4 - 1) / kRun4);
-    int64_t b = (runs + kRunThreads - 1) / kRunThreads;
-    if (b > g4_max_blocks(sms)) b = g4_max_blocks(sms);
-    ssim4_run_kernel<T><<<(unsigned)(b < 1 ? 1 : b), kRunThreads, 0, st>>>(f, p, parts, res, ticket, dbg);
-  }
-  else
-    ssim4_kernel<T><<<g4_grid(total, sms), kG4Threads, 0, st>>>(f, p, parts, res, ticket, dbg);
+  ssim4_kernel<T><<<g4_grid(total, sms), kG4Threads, 0, st>>>(f, p, parts, res, ticket, dbg);
   return cudaGetLastError();
 }
 

@@ -167,6 +167,45 @@ class TestDeriv:
         assert r["der2_f_min"] == r["der2_f_max"] == 2 * np.abs(q).sum()
         assert r["lap_mse"] == 0 and r["der1_maxabs"] == 0
 
+    def test_finite_psnr_rmse_closed_form(self, orc):
+        """Finite per-field PSNR / RMSE.  x = alpha z^2 + beta p_x, y = x +
+        gamma p_y (dyadic, exact in float32): on the interior (z = 1..nz-2)
+          Div(x) = 2 alpha z + beta  (range 2 alpha (nz - 3)),
+        with D_a = (f(+1) - f(-1)) / 2: D_z x = 2 alpha z, D_x x = beta, D_y y - D_y x = gamma, so
+          dDiv = gamma, dDer1 = |2 gamma| (Eq. 1 has no 1/2), dLap = 0, dDer2 = 0,
+          Der1(x) = 4 alpha z + 2 beta (range 4 alpha (nz - 3)),
+          Grad(x) = sqrt((2 alpha z)^2 + beta^2),  Grad(y) = sqrt((2 alpha z)^2 + beta^2 + gamma^2).
+        PSNR_F = 20 log10(max F(x) - min F(x)) - 10 log10(mse_F): the range of the ORIGINAL's field
+        and 20 vs 10 are both pinned (a range of F(y), or 10 log10 of the range, fails)."""
+        nz, ny, nx = 11, 6, 7
+        a, b, g = 2.0 ** -4, 2.0 ** -3, 2.0 ** -5
+        z, yy, xx = np.indices((nz, ny, nx)).astype(np.float64)
+        x = (a * z * z + b * xx).astype(np.float32)
+        y = (a * z * z + b * xx + g * yy).astype(np.float32)
+        assert np.all(y.astype(np.float64) - x.astype(np.float64) == g * yy)
+        r = orc.deriv(x, y)
+        nI = (nz - 2) * (ny - 2) * (nx - 2)
+        assert r["n_interior"] == nI
+        zi = np.arange(1, nz - 1, dtype=np.float64)
+        # Div: constant error gamma, range 2 alpha (nz - 3)
+        assert r["div_maxabs"] == g and r["div_mae"] == g and r["div_mse"] == g * g and r["div_rmse"] == g
+        assert r["div_f_min"] == 2 * a * 1 + b and r["div_f_max"] == 2 * a * (nz - 2) + b
+        assert r["div_psnr"] == pytest.approx(20 * math.log10(2 * a * (nz - 3)) - 10 * math.log10(g * g), abs=1e-12)
+        # Der1: constant error 2 gamma, range 4 alpha (nz - 3)
+        assert r["der1_mse"] == 4 * g * g and r["der1_rmse"] == 2 * g
+        assert r["der1_psnr"] == pytest.approx(20 * math.log10(4 * a * (nz - 3)) - 10 * math.log10(4 * g * g), abs=1e-12)
+        # Lap / Der2: zero error -> +inf
+        assert r["lap_mse"] == 0 and r["lap_psnr"] == math.inf and r["der2_psnr"] == math.inf
+        # Grad: per-plane closed form, mean over the interior
+        gx = np.sqrt((2 * a * zi) ** 2 + b * b)
+        gy = np.sqrt((2 * a * zi) ** 2 + b * b + g * g)
+        mse = float(np.mean((gy - gx) ** 2))
+        assert r["grad_mse"] == pytest.approx(mse, rel=1e-13)
+        assert r["grad_rmse"] == pytest.approx(math.sqrt(mse), rel=1e-13)
+        assert r["grad_maxabs"] == pytest.approx(float(np.max(gy - gx)), rel=1e-13)
+        rng = gx.max() - gx.min()
+        assert r["grad_psnr"] == pytest.approx(20 * math.log10(rng) - 10 * math.log10(mse), abs=1e-10)
+
     @pytest.mark.parametrize("shape", [(12, 14, 16), (30, 40), (9, 1, 33)])
     def test_against_numpy_scipy(self, orc, shape):
         spec = synth.config("C1", dims=shape)
@@ -314,6 +353,21 @@ class TestSSIM:
         for i in rng.choice(len(origins), size=min(20, len(origins)), replace=False):
             v = orc.ssim_window(x, y, origins[i], [w] * len(shape))
             assert abs(v - ref[i]) < 1e-13
+
+    @pytest.mark.parametrize("cfg,shape,w,s,kw", [("C1", (8, 9, 10), 4, 1, {}),
+                                                  ("C2q", (9, 10, 12), 3, 2, {}),
+                                                  ("C4", (24, 30), 8, 3, {}),
+                                                  ("C1", (10, 9, 14), 5, 1, {"kind": "step", "eb": 0.1})])
+    def test_window_map_brute_force(self, orc, cfg, shape, w, s, kw):
+        """czco_ssim_windows (every window's local SSIM, the per-window reference of the GPU
+        parity tests) against the numpy brute force, element by element, incl. a step field."""
+        x, y = synth.make_pair(synth.config(cfg, dims=shape, **kw))
+        x, y = x.numpy(), y.numpy()
+        ref = ssim_brute_numpy(x, y, w, s)
+        got = orc.ssim_windows(x, y, [w] * len(shape), [s] * len(shape))
+        assert got.shape == tuple((n - w) // s + 1 for n in shape)
+        np.testing.assert_allclose(got.ravel(), ref, rtol=0, atol=1e-12)
+        assert abs(got.mean() - orc.ssim(x, y, [w] * len(shape), [s] * len(shape))[0]) < 1e-14
 
     def test_no_window(self, orc):
         x = dyadic_field((5, 5, 5))
