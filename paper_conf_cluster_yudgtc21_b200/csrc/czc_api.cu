@@ -91,6 +91,12 @@ struct czc_ctx {
   // pipelined host path
   cudaStream_t copy_stream[2] = {nullptr, nullptr};   // [0]: H2D chunks (x then y); [1] unused
   cudaEvent_t copy_ev[2][kMaxHostChunks] = {};
+  // NCCL slab mode: halo exchange on its own stream (overlapping P1), and the validated slab
+  // table of the last call signature (re-validated collectively only when the signature changes)
+  cudaStream_t halo_stream = nullptr;
+  cudaEvent_t halo_ev[2] = {};        // [0]: inputs ready on the compute stream, [1]: halos received
+  std::vector<int64_t> slab_key;
+  std::vector<int64_t> slab_tab;      // 2 per rank: z0, nz_local
 };
 
 static const char* kStatusStr[] = {"ok", "invalid argument", "invalid shape", "unsupported dtype",
@@ -173,6 +179,8 @@ extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
     }
     const size_t rb = (size_t)ctx->max_records * sizeof(Record);
     if ((e = cudaMalloc(&ctx->dres, sizeof(DevResults))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(res)"); break; }
+    // every record byte is defined (the D2H copy of a call carries slots of groups it did not run)
+    if ((e = cudaMemsetAsync(ctx->dres, 0, sizeof(DevResults), ctx->stream)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMemset(res)"); break; }
     if ((e = cudaMallocHost(&ctx->hrec, rb)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMallocHost"); break; }
     if ((e = cudaMalloc(&ctx->tickets, TICKET_N * sizeof(unsigned int))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(tickets)"); break; }
     if ((e = cudaMemsetAsync(ctx->tickets, 0, TICKET_N * sizeof(unsigned int), ctx->stream)) != cudaSuccess ||
@@ -186,6 +194,12 @@ extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
       if ((e = cudaMalloc(&ctx->dstates, (size_t)ctx->max_records * sizeof(P1State))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(states)"); break; }
     }
     if (slab_mode) {
+      if ((e = cudaStreamCreateWithFlags(&ctx->halo_stream, cudaStreamNonBlocking)) != cudaSuccess ||
+          (e = cudaEventCreateWithFlags(&ctx->halo_ev[0], cudaEventDisableTiming)) != cudaSuccess ||
+          (e = cudaEventCreateWithFlags(&ctx->halo_ev[1], cudaEventDisableTiming)) != cudaSuccess) {
+        st = cuda_fail(ctx, e, "halo stream");
+        break;
+      }
       ctx->comm = comm_create(c.nccl_uid, c.rank, std::max(1, c.nranks), &ctx->last_error);
       if (!ctx->comm) { st = CZC_ERR_COMM; break; }
     }
@@ -221,6 +235,9 @@ extern "C" void czc_free(czc_ctx* ctx) {
     if (ctx->copy_stream[c]) cudaStreamDestroy(ctx->copy_stream[c]);
   }
   if (ctx->gexec) cudaGraphExecDestroy(ctx->gexec);
+  for (int i = 0; i < 2; i++)
+    if (ctx->halo_ev[i]) cudaEventDestroy(ctx->halo_ev[i]);
+  if (ctx->halo_stream) cudaStreamDestroy(ctx->halo_stream);
   if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
   delete ctx;
 }
@@ -696,73 +713,136 @@ static czc_status assess_loopback(czc_ctx* ctx, const Plan& P, const E* x, const
   return CZC_OK;
 }
 
-// NCCL slab mode: this rank holds planes [z0, z0 + nzl) of the global field.
+// NCCL slab mode: this rank holds planes [z0, z0 + nzl) of the global field (SURVEY.md §8(e)).
+//  * Slab table: when this rank's call signature (its slab, the global shape, the halo depth, the
+//    element type) differs from the last call's, every buffer the signature needs is allocated
+//    FIRST and the slab table is all-gathered together with each rank's allocation status, so a
+//    local failure is a collective decision (no rank leaves a peer waiting in a
+//    collective) and a bad decomposition fails on every rank.  A repeated signature skips that
+//    allgather and its host synchronisation; a 16-byte allgather at the end of the call still
+//    checks that every rank kept its slab (a changed decomposition returns CZC_ERR_SHAPE on all
+//    ranks and is re-validated on the next call).
+//  * Halo exchange: grouped send / recv on the halo communicator and stream, ordered after the
+//    caller's inputs, overlapping P1 and the P1-state allgather on the compute stream; P2 / P3
+//    wait for it (an event).
+//  * Collectives on the compute stream: the P1 states (merged in rank order on the device: every
+//    rank needs the global mu_e, sigma_e^2), then the per-rank records (combined in rank order on
+//    the host by combine_and_finish, the code exported as czc_combine).
+//  * A CUDA / NCCL failure after the first collective of a call aborts this rank's communicators
+//    (its queued operations are dropped) and the context returns CZC_ERR_COMM from then on.
 template <typename E>
 static czc_status assess_ranks(czc_ctx* ctx, const Plan& P, const E* x, const E* y, const czc_shape* shape,
                                czc_result* out, uint64_t mask) {
-  const cudaStream_t s = ctx->stream;
+  const cudaStream_t s = ctx->stream, hs = ctx->halo_stream;
   const bool timing = ctx->cfg.timing != 0;
+  if (!comm_usable(ctx->comm)) { ctx->last_error = "communicator aborted by an earlier failure"; return CZC_ERR_COMM; }
   const int nranks = comm_size(ctx->comm), rank = comm_rank(ctx->comm);
   const int64_t nz = P.g3[0], plane = P.g3[1] * P.g3[2];
   if (P.D != 3 || shape->dims[0] != nz) { ctx->last_error = "slab mode needs a 3-D field split along dims[0]"; return CZC_ERR_SHAPE; }
   const int64_t z0 = shape->z0, nzl = shape->nz_local > 0 ? shape->nz_local : nz;
-  // slab table: every rank validates every slab identically (a collective decision, no hang)
-  int64_t mine[2] = {z0, nzl};
-  CZC_CUDA(ctx, cudaMemcpyAsync(ctx->dgather_in, mine, sizeof(mine), cudaMemcpyHostToDevice, s));
-  if (!comm_allgather(ctx->comm, ctx->dgather_in, ctx->dgather, sizeof(mine), s, &ctx->last_error)) return CZC_ERR_COMM;
-  std::vector<int64_t> flat(2 * nranks);
-  CZC_CUDA(ctx, cudaMemcpyAsync(flat.data(), ctx->dgather, flat.size() * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-  CZC_CUDA(ctx, cudaStreamSynchronize(s));
-  std::vector<std::pair<int64_t, int64_t>> tab(nranks);
-  for (int r = 0; r < nranks; r++) tab[r] = {flat[2 * r], flat[2 * r + 1]};
   const int64_t H = halo_depth(P);
-  if (!slabs_ok(tab, nz, H)) { ctx->last_error = "slabs must tile dims[0] in rank order, each >= the halo depth"; return CZC_ERR_SHAPE; }
-  const SsimParams sp = ssim_params(P, ctx->cfg);
-  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
-  // halo exchange: H planes up from rank+1, one plane (derivatives) down from rank-1
+  // halo: H planes up from rank+1, one plane (derivatives) down from rank-1
   const int64_t hlo = (P.run_deriv && z0 > 0) ? 1 : 0;
   const int64_t hhi = std::min(H, nz - (z0 + nzl));
   const int64_t prev_hhi = rank > 0 ? std::min(H, nz - z0) : 0;
   const bool next_lo = P.run_deriv && rank + 1 < nranks;
   const size_t pb = (size_t)plane * sizeof(E);
-  czc_status st = ensure_buf(ctx, &ctx->halo, &ctx->halo_cap, 2 * (size_t)(hlo + hhi) * pb + 16);
-  if (st != CZC_OK) return st;
+  const SsimParams sp = ssim_params(P, ctx->cfg);
   E *xlo, *ylo, *xhi, *yhi;
+  const std::vector<int64_t> key = {z0, nzl, nz, P.g3[1], P.g3[2], H, P.run_deriv, (int64_t)sizeof(E)};
+  if (key != ctx->slab_key) {
+    ctx->slab_key.clear();
+    // allocate first (halo planes, kernel scratch), then one collective decision
+    czc_status local = ensure_buf(ctx, &ctx->halo, &ctx->halo_cap, 2 * (size_t)(hlo + hhi) * pb + 16);
+    if (local == CZC_OK) {
+      const Field3<E> F0 = slab_field(ctx, P, x, y, z0, nzl, hlo, hhi, &xlo, &ylo, &xhi, &yhi);
+      local = ensure_scratch(ctx, P, F0, sp);
+    }
+    if (local == CZC_OK) local = ensure_buf(ctx, &ctx->parts, &ctx->parts_cap, (size_t)ctx->p1_grid_cap * sizeof(P1State));
+    const int64_t mine[3] = {z0, nzl, (int64_t)local};
+    CZC_CUDA(ctx, cudaMemcpyAsync(ctx->dgather_in, mine, sizeof(mine), cudaMemcpyHostToDevice, s));
+    if (!comm_allgather(ctx->comm, ctx->dgather_in, ctx->dgather, sizeof(mine), s, &ctx->last_error)) return CZC_ERR_COMM;
+    std::vector<int64_t> flat(3 * nranks);
+    CZC_CUDA(ctx, cudaMemcpyAsync(flat.data(), ctx->dgather, flat.size() * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CZC_CUDA(ctx, cudaStreamSynchronize(s));
+    for (int r = 0; r < nranks; r++)
+      if (flat[3 * r + 2] != CZC_OK) {
+        ctx->last_error = "rank " + std::to_string(r) + " could not set up its slab: " + czc_strerror((czc_status)flat[3 * r + 2]);
+        return (czc_status)flat[3 * r + 2];
+      }
+    std::vector<std::pair<int64_t, int64_t>> tab(nranks);
+    for (int r = 0; r < nranks; r++) tab[r] = {flat[3 * r], flat[3 * r + 1]};
+    if (!slabs_ok(tab, nz, H)) { ctx->last_error = "slabs must tile dims[0] in rank order, each >= the halo depth"; return CZC_ERR_SHAPE; }
+    ctx->slab_tab.assign(2 * nranks, 0);
+    for (int r = 0; r < nranks; r++) { ctx->slab_tab[2 * r] = tab[r].first; ctx->slab_tab[2 * r + 1] = tab[r].second; }
+    ctx->slab_key = key;
+  }
+  // from here on every buffer exists; a failure aborts the communicators (see above)
+  auto fail = [&](czc_status st) {
+    comm_abort(ctx->comm);
+    ctx->slab_key.clear();
+    return st;
+  };
+#define CZC_SLAB(call)                                                              \
+  do {                                                                              \
+    cudaError_t _e = (call);                                                        \
+    if (_e != cudaSuccess) return fail(cuda_fail(ctx, _e, #call));                  \
+  } while (0)
   const Field3<E> F = slab_field(ctx, P, x, y, z0, nzl, hlo, hhi, &xlo, &ylo, &xhi, &yhi);
-  if (!comm_group_begin(&ctx->last_error)) return CZC_ERR_COMM;
+  if (timing) CZC_SLAB(cudaEventRecord(ctx->ev[0], s));
+  // halo exchange on the halo stream, after the caller's writes of x / y (and this context's
+  // previous kernels, which read the halo buffers) on the compute stream
+  CZC_SLAB(cudaEventRecord(ctx->halo_ev[0], s));
+  CZC_SLAB(cudaStreamWaitEvent(hs, ctx->halo_ev[0], 0));
+  if (!comm_group_begin(&ctx->last_error)) return fail(CZC_ERR_COMM);
   bool ok = true;
   if (rank > 0 && prev_hhi > 0) {
-    ok &= comm_send(ctx->comm, x, prev_hhi * pb, rank - 1, s, &ctx->last_error);
-    ok &= comm_send(ctx->comm, y, prev_hhi * pb, rank - 1, s, &ctx->last_error);
+    ok &= comm_send(ctx->comm, x, prev_hhi * pb, rank - 1, hs, &ctx->last_error);
+    ok &= comm_send(ctx->comm, y, prev_hhi * pb, rank - 1, hs, &ctx->last_error);
   }
   if (next_lo) {
-    ok &= comm_send(ctx->comm, x + (nzl - 1) * plane, pb, rank + 1, s, &ctx->last_error);
-    ok &= comm_send(ctx->comm, y + (nzl - 1) * plane, pb, rank + 1, s, &ctx->last_error);
+    ok &= comm_send(ctx->comm, x + (nzl - 1) * plane, pb, rank + 1, hs, &ctx->last_error);
+    ok &= comm_send(ctx->comm, y + (nzl - 1) * plane, pb, rank + 1, hs, &ctx->last_error);
   }
   if (hhi > 0) {
-    ok &= comm_recv(ctx->comm, xhi, hhi * pb, rank + 1, s, &ctx->last_error);
-    ok &= comm_recv(ctx->comm, yhi, hhi * pb, rank + 1, s, &ctx->last_error);
+    ok &= comm_recv(ctx->comm, xhi, hhi * pb, rank + 1, hs, &ctx->last_error);
+    ok &= comm_recv(ctx->comm, yhi, hhi * pb, rank + 1, hs, &ctx->last_error);
   }
   if (hlo > 0) {
-    ok &= comm_recv(ctx->comm, xlo, pb, rank - 1, s, &ctx->last_error);
-    ok &= comm_recv(ctx->comm, ylo, pb, rank - 1, s, &ctx->last_error);
+    ok &= comm_recv(ctx->comm, xlo, pb, rank - 1, hs, &ctx->last_error);
+    ok &= comm_recv(ctx->comm, ylo, pb, rank - 1, hs, &ctx->last_error);
   }
-  if (!comm_group_end(&ctx->last_error) || !ok) return CZC_ERR_COMM;
-  // P1 on the local slab, then one small allgather of the states, merged in rank order on device
-  if ((st = p1_local(ctx, P, x, y, nzl * plane)) != CZC_OK) return st;
+  if (!comm_group_end(&ctx->last_error) || !ok) return fail(CZC_ERR_COMM);
+  CZC_SLAB(cudaEventRecord(ctx->halo_ev[1], hs));
+  // P1 on the local slab (overlaps the halo transfer), one small allgather of the states, merged
+  // in rank order on the device
   if (P.run_p1) {
-    if (!comm_allgather(ctx->comm, &ctx->dres->rec.p1, ctx->dstates, sizeof(P1State), s, &ctx->last_error)) return CZC_ERR_COMM;
-    CZC_CUDA(ctx, launch_p1_combine((const P1State*)ctx->dstates, nranks, ctx->dres, s));
+    CZC_SLAB(launch_p1(x, y, nzl * plane, ctx->p1_grid_cap, (P1State*)ctx->parts, ctx->dres, ctx->tickets + TICKET_P1, s));
+    if (!comm_allgather(ctx->comm, &ctx->dres->rec.p1, ctx->dstates, sizeof(P1State), s, &ctx->last_error)) return fail(CZC_ERR_COMM);
+    CZC_SLAB(launch_p1_combine((const P1State*)ctx->dstates, nranks, ctx->dres, s));
   }
-  if (P.run_pdf) CZC_CUDA(ctx, launch_pdf(x, y, nzl * plane, P.nb, ctx->p1_grid_cap, ctx->dres, s));
-  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
-  if ((st = run_p23(ctx, P, F, sp)) != CZC_OK) return st;
-  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[4], s));
-  // second small allgather: every rank's record, combined in rank order on the host
-  if (!comm_allgather(ctx->comm, &ctx->dres->rec, ctx->dgather, sizeof(Record), s, &ctx->last_error)) return CZC_ERR_COMM;
-  CZC_CUDA(ctx, copy_records(ctx->hrec, (const Record*)ctx->dgather, nranks, P.run_pdf, s));
-  if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[5], s));
-  CZC_CUDA(ctx, cudaStreamSynchronize(s));
+  if (P.run_pdf) CZC_SLAB(launch_pdf(x, y, nzl * plane, P.nb, ctx->p1_grid_cap, ctx->dres, s));
+  if (timing) CZC_SLAB(cudaEventRecord(ctx->ev[1], s));
+  CZC_SLAB(cudaStreamWaitEvent(s, ctx->halo_ev[1], 0));
+  czc_status st = run_p23(ctx, P, F, sp);               // scratch sized above: no allocation
+  if (st != CZC_OK) return fail(st);
+  if (timing) CZC_SLAB(cudaEventRecord(ctx->ev[4], s));
+  // every rank's record, combined in rank order on the host; plus the slab check of this call
+  if (!comm_allgather(ctx->comm, &ctx->dres->rec, ctx->dgather, sizeof(Record), s, &ctx->last_error)) return fail(CZC_ERR_COMM);
+  CZC_SLAB(copy_records(ctx->hrec, (const Record*)ctx->dgather, nranks, P.run_pdf, s));
+  const int64_t mine2[2] = {z0, nzl};
+  CZC_SLAB(cudaMemcpyAsync(ctx->dgather_in, mine2, sizeof(mine2), cudaMemcpyHostToDevice, s));
+  if (!comm_allgather(ctx->comm, ctx->dgather_in, ctx->dstates, sizeof(mine2), s, &ctx->last_error)) return fail(CZC_ERR_COMM);
+  std::vector<int64_t> now(2 * nranks);
+  CZC_SLAB(cudaMemcpyAsync(now.data(), ctx->dstates, now.size() * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  if (timing) CZC_SLAB(cudaEventRecord(ctx->ev[5], s));
+  CZC_SLAB(cudaStreamSynchronize(s));
+#undef CZC_SLAB
+  if (now != ctx->slab_tab) {          // some rank changed its slab without the others
+    ctx->slab_key.clear();
+    ctx->last_error = "the slab decomposition changed on some ranks but not on others";
+    return CZC_ERR_SHAPE;
+  }
   combine_and_finish(P, ctx->hrec, nranks, mask, out);
   finish_timing(ctx, out);
   return CZC_OK;

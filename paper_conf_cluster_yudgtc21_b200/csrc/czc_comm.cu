@@ -7,8 +7,10 @@
 
 namespace czc {
 struct CommState {
-  ncclComm_t comm;
+  ncclComm_t comm;      // collectives (slab table, P1 states, records)
+  ncclComm_t halo;      // halo send / recv (split from comm: its own stream, overlapping P1)
   int rank, size;
+  bool aborted;
 };
 int comm_available() { return 1; }
 static bool ok(ncclResult_t r, const char* what, std::string* err) {
@@ -23,7 +25,13 @@ CommState* comm_create(const void* uid128, int rank, int nranks, std::string* er
   CommState* c = new CommState();
   c->rank = rank;
   c->size = nranks;
+  c->aborted = false;
   if (!ok(ncclCommInitRank(&c->comm, nranks, id, rank), "ncclCommInitRank", err)) {
+    delete c;
+    return nullptr;
+  }
+  if (!ok(ncclCommSplit(c->comm, 0, rank, &c->halo, nullptr), "ncclCommSplit", err)) {
+    ncclCommDestroy(c->comm);
     delete c;
     return nullptr;
   }
@@ -31,9 +39,19 @@ CommState* comm_create(const void* uid128, int rank, int nranks, std::string* er
 }
 void comm_destroy(CommState* c) {
   if (!c) return;
-  ncclCommDestroy(c->comm);
+  if (!c->aborted) {
+    ncclCommDestroy(c->halo);
+    ncclCommDestroy(c->comm);
+  }
   delete c;
 }
+void comm_abort(CommState* c) {
+  if (!c || c->aborted) return;
+  c->aborted = true;
+  ncclCommAbort(c->halo);                  // this rank's queued operations are dropped
+  ncclCommAbort(c->comm);
+}
+bool comm_usable(const CommState* c) { return c && !c->aborted; }
 int comm_rank(const CommState* c) { return c->rank; }
 int comm_size(const CommState* c) { return c->size; }
 bool comm_allgather(CommState* c, const void* send, void* recv, size_t bytes, cudaStream_t st, std::string* err) {
@@ -42,10 +60,10 @@ bool comm_allgather(CommState* c, const void* send, void* recv, size_t bytes, cu
 bool comm_group_begin(std::string* err) { return ok(ncclGroupStart(), "ncclGroupStart", err); }
 bool comm_group_end(std::string* err) { return ok(ncclGroupEnd(), "ncclGroupEnd", err); }
 bool comm_send(CommState* c, const void* buf, size_t bytes, int peer, cudaStream_t st, std::string* err) {
-  return ok(ncclSend(buf, bytes, ncclUint8, peer, c->comm, st), "ncclSend", err);
+  return ok(ncclSend(buf, bytes, ncclUint8, peer, c->halo, st), "ncclSend", err);
 }
 bool comm_recv(CommState* c, void* buf, size_t bytes, int peer, cudaStream_t st, std::string* err) {
-  return ok(ncclRecv(buf, bytes, ncclUint8, peer, c->comm, st), "ncclRecv", err);
+  return ok(ncclRecv(buf, bytes, ncclUint8, peer, c->halo, st), "ncclRecv", err);
 }
 }  // namespace czc
 #else
@@ -57,6 +75,8 @@ CommState* comm_create(const void*, int, int, std::string* err) {
   return nullptr;
 }
 void comm_destroy(CommState*) {}
+void comm_abort(CommState*) {}
+bool comm_usable(const CommState*) { return false; }
 int comm_rank(const CommState* c) { return c ? c->rank : 0; }
 int comm_size(const CommState* c) { return c ? c->size : 1; }
 bool comm_allgather(CommState*, const void*, void*, size_t, cudaStream_t, std::string* err) { if (err) *err = "no NCCL"; return false; }
