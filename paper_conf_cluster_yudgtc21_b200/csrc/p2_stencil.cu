@@ -1049,7 +1049,7 @@ static dim3 deriv_grid(const Field3<T>& s, int zchunk, int* zc) {
     return dim3((unsigned)(U < G ? (U > 0 ? U : 1) : G), 1, 1);
   }
   int64_t c = zchunk;
-  const int64_t fill = cdiv(planes * tiles, 148 * 4);
+  const int64_t fill = cdiv(planes * tiles, (int64_t)sm_count() * 4);
   if (fill < c) c = fill < 8 ? 8 : fill;
   c = cdiv(planes, cdiv(planes, c));          // equal chunks
   *zc = (int)c;
