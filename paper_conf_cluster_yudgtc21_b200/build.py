@@ -95,7 +95,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         list(ex.map(run, jobs))
     objs = [os.path.join(OBJ, s.replace(".cu", ".o")) for s in SOURCES]
     if force or jobs or _stale(SO, objs):
-        cmd = [nvcc] + ARCH + ["-shared", "-o", SO + ".tmp"] + objs + ["-lcudart_static"]
+        cmd = [nvcc] + ARCH + ["-shared", "-o", SO + ".tmp"] + objs + ["-lcudart_static", "-ldl"]
         tn = _torch_nccl()
         if tn:
             cmd += ["-L" + tn[1], "-l:libnccl.so.2", "-Xlinker", "-rpath=" + tn[1]]

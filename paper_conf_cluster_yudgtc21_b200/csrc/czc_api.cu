@@ -15,8 +15,16 @@
 #include <utility>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>   // header-only NVTX 3: host ranges for nsys / ncu --nvtx (no-ops without a tool)
+
 #include "czc_comm.h"
 #include "czc_internal.cuh"
+
+// Host-side NVTX range for the duration of a scope (tracing: `ncu --nvtx --nvtx-include czc/`).
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
 
 namespace czc {
 // Launchers, instantiated for E = float and E = double in their .cu files.
@@ -97,6 +105,7 @@ struct czc_ctx {
   cudaEvent_t halo_ev[2] = {};        // [0]: inputs ready on the compute stream, [1]: halos received
   std::vector<int64_t> slab_key;
   std::vector<int64_t> slab_tab;      // 2 per rank: z0, nz_local
+  int64_t* hpin = nullptr;            // pinned host staging for the small slab-table copies
 };
 
 static const char* kStatusStr[] = {"ok", "invalid argument", "invalid shape", "unsupported dtype",
@@ -182,6 +191,10 @@ extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
     // every record byte is defined (the D2H copy of a call carries slots of groups it did not run)
     if ((e = cudaMemsetAsync(ctx->dres, 0, sizeof(DevResults), ctx->stream)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMemset(res)"); break; }
     if ((e = cudaMallocHost(&ctx->hrec, rb)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMallocHost"); break; }
+    if ((e = cudaMallocHost(&ctx->hpin, (size_t)(4 + 3 * ctx->max_records) * sizeof(int64_t))) != cudaSuccess) {
+      st = cuda_fail(ctx, e, "cudaMallocHost");
+      break;
+    }
     if ((e = cudaMalloc(&ctx->tickets, TICKET_N * sizeof(unsigned int))) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(tickets)"); break; }
     if ((e = cudaMemsetAsync(ctx->tickets, 0, TICKET_N * sizeof(unsigned int), ctx->stream)) != cudaSuccess ||
         (e = cudaStreamSynchronize(ctx->stream)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMemset"); break; }
@@ -219,6 +232,7 @@ extern "C" void czc_free(czc_ctx* ctx) {
   if (ctx->comm) comm_destroy(ctx->comm);
   cudaFree(ctx->dres);
   cudaFreeHost(ctx->hrec);
+  cudaFreeHost(ctx->hpin);
   cudaFree(ctx->tickets);
   cudaFree(ctx->parts);
   cudaFree(ctx->din[0]);
@@ -509,15 +523,21 @@ static czc_status run_p23(czc_ctx* ctx, const Plan& P, const Field3<E>& F, const
   const cudaStream_t s = ctx->stream;
   czc_status st = ensure_scratch(ctx, P, F, sp);
   if (st != CZC_OK) return st;
-  if (P.run_deriv)
+  if (P.run_deriv) {
+    NvtxRange r_("czc/P2 derivatives");
     CZC_CUDA(ctx, launch_deriv(F, kZchunkDeriv, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_DERIV, s));
+  }
   if (ctx->cfg.timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
-  if (P.run_ac)
+  if (P.run_ac) {
+    NvtxRange r_("czc/P2 autocorrelation");
     CZC_CUDA(ctx, launch_ac(F, P.T, 0, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_ACZ, s));
+  }
   if (ctx->cfg.timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));
-  if (P.run_ssim)
+  if (P.run_ssim) {
+    NvtxRange r_("czc/P3 SSIM");
     CZC_CUDA(ctx, launch_ssim(P.kind, P.W, F, sp, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_SSIM,
                               ctx->cfg.debug_wssim, s, nullptr));
+  }
   return CZC_OK;
 }
 
@@ -552,6 +572,7 @@ static czc_status enqueue_single(czc_ctx* ctx, const Plan& P, const E* x, const 
   const cudaStream_t s = ctx->stream;
   const bool timing = ctx->cfg.timing != 0;
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
+  NvtxRange r_("czc/enqueue");
   czc_status st = p1_local(ctx, P, x, y, F.nz * F.ny * F.nx);
   if (st != CZC_OK) return st;
   if (P.run_pdf) CZC_CUDA(ctx, launch_pdf(x, y, F.nz * F.ny * F.nx, P.nb, ctx->p1_grid_cap, ctx->dres, s));
@@ -759,12 +780,15 @@ static czc_status assess_ranks(czc_ctx* ctx, const Plan& P, const E* x, const E*
       local = ensure_scratch(ctx, P, F0, sp);
     }
     if (local == CZC_OK) local = ensure_buf(ctx, &ctx->parts, &ctx->parts_cap, (size_t)ctx->p1_grid_cap * sizeof(P1State));
-    const int64_t mine[3] = {z0, nzl, (int64_t)local};
-    CZC_CUDA(ctx, cudaMemcpyAsync(ctx->dgather_in, mine, sizeof(mine), cudaMemcpyHostToDevice, s));
-    if (!comm_allgather(ctx->comm, ctx->dgather_in, ctx->dgather, sizeof(mine), s, &ctx->last_error)) return CZC_ERR_COMM;
-    std::vector<int64_t> flat(3 * nranks);
-    CZC_CUDA(ctx, cudaMemcpyAsync(flat.data(), ctx->dgather, flat.size() * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    int64_t* pin = ctx->hpin;
+    pin[0] = z0;
+    pin[1] = nzl;
+    pin[2] = (int64_t)local;
+    CZC_CUDA(ctx, cudaMemcpyAsync(ctx->dgather_in, pin, 3 * sizeof(int64_t), cudaMemcpyHostToDevice, s));
+    if (!comm_allgather(ctx->comm, ctx->dgather_in, ctx->dgather, 3 * sizeof(int64_t), s, &ctx->last_error)) return CZC_ERR_COMM;
+    CZC_CUDA(ctx, cudaMemcpyAsync(pin + 3, ctx->dgather, 3 * (size_t)nranks * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     CZC_CUDA(ctx, cudaStreamSynchronize(s));
+    const std::vector<int64_t> flat(pin + 3, pin + 3 + 3 * nranks);
     for (int r = 0; r < nranks; r++)
       if (flat[3 * r + 2] != CZC_OK) {
         ctx->last_error = "rank " + std::to_string(r) + " could not set up its slab: " + czc_strerror((czc_status)flat[3 * r + 2]);
@@ -830,14 +854,17 @@ static czc_status assess_ranks(czc_ctx* ctx, const Plan& P, const E* x, const E*
   // every rank's record, combined in rank order on the host; plus the slab check of this call
   if (!comm_allgather(ctx->comm, &ctx->dres->rec, ctx->dgather, sizeof(Record), s, &ctx->last_error)) return fail(CZC_ERR_COMM);
   CZC_SLAB(copy_records(ctx->hrec, (const Record*)ctx->dgather, nranks, P.run_pdf, s));
-  const int64_t mine2[2] = {z0, nzl};
-  CZC_SLAB(cudaMemcpyAsync(ctx->dgather_in, mine2, sizeof(mine2), cudaMemcpyHostToDevice, s));
-  if (!comm_allgather(ctx->comm, ctx->dgather_in, ctx->dstates, sizeof(mine2), s, &ctx->last_error)) return fail(CZC_ERR_COMM);
-  std::vector<int64_t> now(2 * nranks);
-  CZC_SLAB(cudaMemcpyAsync(now.data(), ctx->dstates, now.size() * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  // (pinned staging: a pageable copy would block the host until the kernels above finish)
+  int64_t* pin = ctx->hpin;            // [0, 2): this rank's slab, [2, 2 + 2 nranks): the gathered table
+  pin[0] = z0;
+  pin[1] = nzl;
+  CZC_SLAB(cudaMemcpyAsync(ctx->dgather_in, pin, 2 * sizeof(int64_t), cudaMemcpyHostToDevice, s));
+  if (!comm_allgather(ctx->comm, ctx->dgather_in, ctx->dstates, 2 * sizeof(int64_t), s, &ctx->last_error)) return fail(CZC_ERR_COMM);
+  CZC_SLAB(cudaMemcpyAsync(pin + 2, ctx->dstates, 2 * (size_t)nranks * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
   if (timing) CZC_SLAB(cudaEventRecord(ctx->ev[5], s));
   CZC_SLAB(cudaStreamSynchronize(s));
 #undef CZC_SLAB
+  const std::vector<int64_t> now(pin + 2, pin + 2 + 2 * nranks);
   if (now != ctx->slab_tab) {          // some rank changed its slab without the others
     ctx->slab_key.clear();
     ctx->last_error = "the slab decomposition changed on some ranks but not on others";
@@ -934,6 +961,7 @@ extern "C" czc_status czc_assess(czc_ctx* ctx, const void* orig, const void* rec
                                  czc_dtype dtype, uint64_t metric_mask, czc_result* out) {
   czc_status st = check_common(ctx, orig, recon, shape, dtype, out);
   if (st != CZC_OK) return st;
+  NvtxRange r_("czc/assess");
   if (cudaSetDevice(ctx->device) != cudaSuccess) return cuda_fail(ctx, cudaGetLastError(), "cudaSetDevice");
   if ((st = check_device_ptr(ctx, orig, "orig")) != CZC_OK || (st = check_device_ptr(ctx, recon, "recon")) != CZC_OK)
     return st;
@@ -1063,6 +1091,7 @@ extern "C" czc_status czc_assess_host(czc_ctx* ctx, const void* orig, const void
                                       czc_dtype dtype, uint64_t metric_mask, czc_result* out) {
   czc_status st = check_common(ctx, orig, recon, shape, dtype, out);
   if (st != CZC_OK) return st;
+  NvtxRange r_("czc/assess_host");
   if (shape->ndim < 1 || shape->ndim > CZC_MAX_DIMS) return CZC_ERR_SHAPE;
   int64_t n = 1;
   for (int i = 0; i < shape->ndim; i++) {
