@@ -39,7 +39,7 @@
 extern "C" {
 #endif
 
-#define CZC_ABI_VERSION 4
+#define CZC_ABI_VERSION 5
 #define CZC_MAX_DIMS 4           /* ndim 1..3 on the streamed engines; 4-D fields (NEXT row f3)    */
 #define CZC_MAX_LAG 16           /* largest supported autocorrelation lag (paper uses <= 10, L345) */
 #define CZC_PDF_MAX_BINS 256     /* largest number of error-PDF bins                              */
@@ -98,6 +98,11 @@ typedef struct czc_config {
                                  /* buffers, owned ranges, rank-ordered combine) with device     */
                                  /* copies in place of NCCL; 0/1 = off.  Requires nranks <= 1.   */
   int pdf_bins;                  /* CZC_M_PDF: bins per PDF, 1..CZC_PDF_MAX_BINS; 0 -> 100       */
+  double* debug_der;             /* optional DEVICE buffer of 5 x n_interior doubles: the error   */
+                                 /* dF = F(recon) - F(orig) of every interior point (Alg. 2 */
+                                 /* "Der"), field-major (DER1, DER2, GRAD, DIV, LAP), points in C  */
+                                 /* order of the interior grid (extent n_a - 2 per active axis);  */
+                                 /* NULL = not written (not on the timed path)                    */
 } czc_config;
 
 /* Field shape.  Single GPU: z0 = 0 and nz_local = dims[0] (or 0 meaning dims[0]).

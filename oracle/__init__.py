@@ -79,9 +79,10 @@ def _load():
         UP = ctypes.POINTER(ctypes.c_uint64)
         lib.czco_pdf.argtypes = [P, P, ctypes.c_uint64, ctypes.c_int, DP, DP, UP, DP, DP, UP, UP]
         lib.czco_ssim_windows.argtypes = [P, P, ctypes.c_int, I64P, I64P, I64P, ctypes.c_int, P]
+        lib.czco_deriv_points.argtypes = [P, P, ctypes.c_int, I64P, P]
         lib.czco_threads.restype = ctypes.c_int
         for name in ("czco_p1", "czco_deriv", "czco_autocorr", "czco_ssim_window", "czco_ssim", "czco_pdf",
-                     "czco_ssim_windows"):
+                     "czco_ssim_windows", "czco_deriv_points"):
             f32, f64 = getattr(lib, name), getattr(lib, name + "_f64")
             f64.argtypes = f32.argtypes
             f64.restype = f32.restype
@@ -141,6 +142,24 @@ def deriv(x, y, dims=None) -> Dict[str, float]:
         for s in DERIV_STATS:
             out[f"{f}_{s}"] = getattr(r.f[i], s)
     return out
+
+
+def deriv_points(x, y, dims=None) -> np.ndarray:
+    """Per-point dF = F(y) - F(x) of the five derived fields (czco_deriv_points): shape
+    (5, n_interior), fields DER1, DER2, GRAD, DIV, LAP, points in C order of the interior grid."""
+    x, y = _pair(x, y)
+    nd, d = _dims(x, dims)
+    shp = tuple(x.shape) if dims is None else tuple(int(v) for v in dims)
+    nI = 1
+    for n in shp:
+        nI *= (n - 2 if n > 2 else 0) if n > 1 else 1
+    out = np.empty(5 * max(nI, 1), dtype=np.float64)
+    rc = _fn("czco_deriv_points", x)(x.ctypes.data, y.ctypes.data, nd, d, out.ctypes.data)
+    if rc == 3:
+        return np.empty((5, 0))
+    if rc:
+        raise ValueError(f"czco_deriv_points failed ({rc})")
+    return out.reshape(5, nI)
 
 
 def autocorr(x, y, max_lag: int = 10, dims=None):

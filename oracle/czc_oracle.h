@@ -49,6 +49,11 @@ int czco_p1(const float* x, const float* y, uint64_t n, czco_p1_t* out);
 
 int czco_deriv(const float* x, const float* y, int ndim, const int64_t* dims, czco_deriv_t* out);
 
+/* Per-point errors dF = F(y) - F(x) of the five derived fields (Alg. 2 "Der"), out =
+ * 5 x n_interior doubles, field-major, interior points in C order; returns 3 if no interior. */
+int czco_deriv_points(const float* x, const float* y, int ndim, const int64_t* dims, double* out);
+int czco_deriv_points_f64(const double* x, const double* y, int ndim, const int64_t* dims, double* out);
+
 /* Eq. 2 (L133): ac[0..max_lag], count[0..max_lag] (= ne_tau).  mu, sigma^2 over all N elements. */
 int czco_autocorr(const float* x, const float* y, int ndim, const int64_t* dims, int max_lag,
                   double* ac, uint64_t* count);

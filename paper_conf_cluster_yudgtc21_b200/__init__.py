@@ -46,7 +46,8 @@ class Config(ctypes.Structure):
                 ("ssim_window", ctypes.c_int * MAX_DIMS), ("ssim_step", ctypes.c_int * MAX_DIMS),
                 ("ssim_range_mode", ctypes.c_int), ("ac_max_lag", ctypes.c_int), ("timing", ctypes.c_int),
                 ("rank", ctypes.c_int), ("nranks", ctypes.c_int), ("nccl_uid", ctypes.c_void_p),
-                ("debug_wssim", ctypes.c_void_p), ("loopback_slabs", ctypes.c_int), ("pdf_bins", ctypes.c_int)]
+                ("debug_wssim", ctypes.c_void_p), ("loopback_slabs", ctypes.c_int), ("pdf_bins", ctypes.c_int),
+                ("debug_der", ctypes.c_void_p)]
 
 
 class Shape(ctypes.Structure):
@@ -142,7 +143,7 @@ def _per_axis(v, ndim) -> Sequence[int]:
 def make_config(ndim: int = 3, device: int = -1, stream: Optional[int] = None, ssim_window=8, ssim_step=1,
                 ssim_range_mode: int = 0, ac_max_lag: int = 10, timing: bool = False, rank: int = 0,
                 nranks: int = 1, nccl_uid: Optional[bytes] = None, debug_wssim: Optional[int] = None,
-                loopback_slabs: int = 0, pdf_bins: int = 0) -> Config:
+                loopback_slabs: int = 0, pdf_bins: int = 0, debug_der: Optional[int] = None) -> Config:
     c = Config()
     c.device = device
     c.stream = stream
@@ -161,6 +162,7 @@ def make_config(ndim: int = 3, device: int = -1, stream: Optional[int] = None, s
     c.debug_wssim = debug_wssim
     c.loopback_slabs = loopback_slabs
     c.pdf_bins = pdf_bins
+    c.debug_der = debug_der
     return c
 
 

@@ -42,7 +42,7 @@ template <typename E>
 int64_t ac_blocks(const Field3<E>& s, int T);
 template <typename E>
 cudaError_t launch_deriv(const Field3<E>& s, int zchunk, double* parts, DevResults* res,
-                         unsigned int* ticket, cudaStream_t st);
+                         unsigned int* ticket, double* dbg, cudaStream_t st);
 template <typename E>
 cudaError_t launch_ac(const Field3<E>& s, int T, int zchunk, double* parts, DevResults* res,
                       unsigned int* ticket, cudaStream_t st);
@@ -54,7 +54,7 @@ cudaError_t launch_ssim(int kind, int W, const Field3<E>& f, const SsimParams& p
 int64_t g4_max_blocks(int sms);
 template <typename E>
 cudaError_t launch_deriv4(const E* x, const E* y, const int64_t n[4], int sms, double* parts, DevResults* res,
-                          unsigned int* ticket, cudaStream_t st);
+                          unsigned int* ticket, double* dbg, cudaStream_t st);
 template <typename E>
 cudaError_t launch_ac4(const E* x, const E* y, const int64_t n[4], int T, int sms, double* parts, DevResults* res,
                        unsigned int* ticket, cudaStream_t st);
@@ -525,7 +525,8 @@ static czc_status run_p23(czc_ctx* ctx, const Plan& P, const Field3<E>& F, const
   if (st != CZC_OK) return st;
   if (P.run_deriv) {
     NvtxRange r_("czc/P2 derivatives");
-    CZC_CUDA(ctx, launch_deriv(F, kZchunkDeriv, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_DERIV, s));
+    CZC_CUDA(ctx, launch_deriv(F, kZchunkDeriv, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_DERIV,
+                               ctx->cfg.debug_der, s));
   }
   if (ctx->cfg.timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
   if (P.run_ac) {
@@ -606,7 +607,8 @@ static czc_status assess_single(czc_ctx* ctx, const Plan& P, const E* x, const E
         (int64_t)(uintptr_t)x, (int64_t)(uintptr_t)y, (int64_t)sizeof(E), P.g3[0], P.g3[1], P.g3[2],
         P.run_p1, P.run_deriv, P.run_ac, P.run_ssim, P.run_pdf, P.W, P.kind, P.T, P.nb,
         P.step[0], P.step[1], P.step[2], ctx->cfg.ssim_range_mode,
-        (int64_t)(uintptr_t)ctx->cfg.debug_wssim, (int64_t)(uintptr_t)ctx->parts, (int64_t)ctx->parts_cap};
+        (int64_t)(uintptr_t)ctx->cfg.debug_wssim, (int64_t)(uintptr_t)ctx->cfg.debug_der,
+        (int64_t)(uintptr_t)ctx->parts, (int64_t)ctx->parts_cap};
     if (!ctx->gexec || key != ctx->gkey) {
       if (ctx->gexec) { cudaGraphExecDestroy(ctx->gexec); ctx->gexec = nullptr; }
       cudaGraph_t g = nullptr;
@@ -903,7 +905,8 @@ static czc_status assess_4d(czc_ctx* ctx, const Plan& P, const E* x, const E* y,
   if ((st = p1_local(ctx, P, x, y, N)) != CZC_OK) return st;
   if (P.run_pdf) CZC_CUDA(ctx, launch_pdf(x, y, N, P.nb, ctx->p1_grid_cap, ctx->dres, s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
-  if (P.run_deriv) CZC_CUDA(ctx, launch_deriv4(x, y, P.g4, ctx->sm_count, parts, ctx->dres, ctx->tickets + TICKET_DERIV, s));
+  if (P.run_deriv)
+    CZC_CUDA(ctx, launch_deriv4(x, y, P.g4, ctx->sm_count, parts, ctx->dres, ctx->tickets + TICKET_DERIV, ctx->cfg.debug_der, s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
   if (P.run_ac) CZC_CUDA(ctx, launch_ac4(x, y, P.g4, P.T, ctx->sm_count, parts, ctx->dres, ctx->tickets + TICKET_ACZ, s));
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));

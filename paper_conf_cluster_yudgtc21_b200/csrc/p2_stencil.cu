@@ -89,6 +89,18 @@ __device__ __forceinline__ void scale_halved(double (&acc)[kDerivSlots]) {
   }
 }
 
+// Per-point debug output (czc_config.debug_der): dF = F(y) - F(x) of interior point `idx` (C
+// order of the interior grid) for the five fields, field-major with stride nI.  F[GRAD] / F[DIV]
+// hold 2 Grad / 2 Div (deriv_fields): their difference is halved, exactly.
+__device__ __forceinline__ void deriv_debug(double* dbg, int64_t nI, int64_t idx, const double (&Fx)[CZC_NDERIV],
+                                            const double (&Fy)[CZC_NDERIV]) {
+#pragma unroll
+  for (int f = 0; f < CZC_NDERIV; f++) {
+    const double d = Fy[f] - Fx[f];
+    dbg[f * nI + idx] = (f == CZC_GRAD || f == CZC_DIV) ? 0.5 * d : d;
+  }
+}
+
 struct DerivOp {
   __device__ int operator()(int k) const { return deriv_op(k); }
 };
@@ -102,7 +114,7 @@ struct SumOp {
 template <typename T, bool ZA, bool YA, int BX, int BY>
 __global__ void __launch_bounds__(BX * BY, 2)
 deriv_kernel(Field3<T> s, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
-             unsigned int* __restrict__ ticket) {
+             unsigned int* __restrict__ ticket, double* __restrict__ dbg) {
   constexpr int kTX = BX, kTY = BY;
   // halo cells of one plane tile: the full ring with a y axis, the two x ends without
   constexpr int kHalo = YA ? 2 * (kTX + 2) + 2 * kTY : 2;
@@ -167,6 +179,10 @@ deriv_kernel(Field3<T> s, int zchunk, double* __restrict__ parts, DevResults* __
       double Fx[CZC_NDERIV], Fy[CZC_NDERIV];
       deriv_fields<ZA, YA>(x0, xp, xm, yn.x, ys.x, xe.x, xw.x, Fx);
       deriv_fields<ZA, YA>(y0, yp, ym, yn.y, ys.y, xe.y, xw.y, Fy);
+      if (dbg) {
+        const int64_t ix = s.nx - 2, iy = YA ? s.ny - 2 : 1, iz = ZA ? s.nz - 2 : 1;
+        deriv_debug(dbg, iz * iy * ix, ((ZA ? z - 1 : 0) * iy + (YA ? gy - 1 : 0)) * ix + gx - 1, Fx, Fy);
+      }
 #pragma unroll
       for (int fi = 0; fi < CZC_NDERIV; fi++) {
         const double d = Fy[fi] - Fx[fi];
@@ -195,7 +211,7 @@ deriv_kernel(Field3<T> s, int zchunk, double* __restrict__ parts, DevResults* __
 template <typename T>
 __global__ void __launch_bounds__(256)
 deriv2_kernel(Field3<T> s, int zchunk, double* __restrict__ parts, DevResults* __restrict__ res,
-              unsigned int* __restrict__ ticket) {
+              unsigned int* __restrict__ ticket, double* __restrict__ dbg) {
   const int lane = threadIdx.x & 31;
   const int64_t gx = (int64_t)blockIdx.x * 256 + threadIdx.x;
   const int64_t nx = s.nx, nrow = s.nz;
@@ -238,6 +254,7 @@ deriv2_kernel(Field3<T> s, int zchunk, double* __restrict__ parts, DevResults* _
         double Fx[CZC_NDERIV], Fy[CZC_NDERIV];
         deriv_fields<true, false>(x0, xp, xm, 0.0, 0.0, xe, xw, Fx);
         deriv_fields<true, false>(y0, yp, ym, 0.0, 0.0, ye, yw, Fy);
+        if (dbg) deriv_debug(dbg, (nrow - 2) * (nx - 2), (zb + i - 1) * (nx - 2) + gx - 1, Fx, Fy);
 #pragma unroll
         for (int fi = 0; fi < CZC_NDERIV; fi++) {
           const double d = Fy[fi] - Fx[fi];
@@ -262,10 +279,10 @@ deriv2_kernel(Field3<T> s, int zchunk, double* __restrict__ parts, DevResults* _
 // 3-D variant with two points per thread: threads (32, 4) cover a 32 x 8 tile, thread (tx, ty)
 // owns rows ty and ty + 4.  The 25 accumulators are shared by both points (half the registers
 // per point) and the two independent stencils double each warp's instruction-level parallelism.
-template <typename T, int PTS>
+template <typename T, int PTS, bool DBG>
 __global__ void __launch_bounds__(kTX * kTY / PTS, sizeof(T) == 4 ? 4 : 3)
 deriv3_kernel(Field3<T> s, int zc, double* __restrict__ parts, DevResults* __restrict__ res,
-              unsigned int* __restrict__ ticket) {
+              unsigned int* __restrict__ ticket, double* __restrict__ dbg) {
   constexpr int RY = kTY / PTS;                    // thread rows
   constexpr int kHalo = 2 * (kTX + 2) + 2 * kTY;
   static_assert(kHalo <= kTX * RY, "halo larger than the block");
@@ -371,6 +388,9 @@ deriv3_kernel(Field3<T> s, int zc, double* __restrict__ parts, DevResults* __res
         double Fx[CZC_NDERIV], Fy[CZC_NDERIV];
         deriv_fields<true, true>(x0[p], xp[p], xm[p], yn.x, ys.x, xe.x, xw.x, Fx);
         deriv_fields<true, true>(y0[p], yp[p], ym[p], yn.y, ys.y, xe.y, xw.y, Fy);
+        if (DBG)                                   // compile-time: no branch on the timed path
+          deriv_debug(dbg, (s.nz - 2) * (s.ny - 2) * (s.nx - 2),
+                      ((zb + i - 1) * (s.ny - 2) + gy0 + p * RY - 1) * (s.nx - 2) + gx - 1, Fx, Fy);
 #pragma unroll
         for (int fi = 0; fi < CZC_NDERIV; fi++) {
           const double d = Fy[fi] - Fx[fi];
@@ -1064,14 +1084,17 @@ int64_t deriv_blocks(const Field3<T>& s0, int zchunk) {
 
 template <typename T>
 cudaError_t launch_deriv(const Field3<T>& s0, int zchunk, double* parts, DevResults* res,
-                         unsigned int* ticket, cudaStream_t st) {
+                         unsigned int* ticket, double* dbg, cudaStream_t st) {
   const Field3<T> s = deriv_view(s0);
   int zc;
   const dim3 grid = deriv_grid(s, zchunk, &zc);
-  if (s.ny > 1 && s.nz > 2) deriv3_kernel<T, 2><<<grid, dim3(kTX, kTY / 2), 0, st>>>(s, zc, parts, res, ticket);
-  else if (s.ny > 1) deriv_kernel<T, true, true, kTX, kTY><<<grid, dim3(kTX, kTY), 0, st>>>(s, zc, parts, res, ticket);
-  else if (s.nz > 1) deriv2_kernel<T><<<grid, 256, 0, st>>>(s, zc, parts, res, ticket);
-  else deriv_kernel<T, false, false, 256, 1><<<grid, dim3(256, 1), 0, st>>>(s, zc, parts, res, ticket);
+  if (s.ny > 1 && s.nz > 2) {
+    if (dbg) deriv3_kernel<T, 2, true><<<grid, dim3(kTX, kTY / 2), 0, st>>>(s, zc, parts, res, ticket, dbg);
+    else deriv3_kernel<T, 2, false><<<grid, dim3(kTX, kTY / 2), 0, st>>>(s, zc, parts, res, ticket, dbg);
+  }
+  else if (s.ny > 1) deriv_kernel<T, true, true, kTX, kTY><<<grid, dim3(kTX, kTY), 0, st>>>(s, zc, parts, res, ticket, dbg);
+  else if (s.nz > 1) deriv2_kernel<T><<<grid, 256, 0, st>>>(s, zc, parts, res, ticket, dbg);
+  else deriv_kernel<T, false, false, 256, 1><<<grid, dim3(256, 1), 0, st>>>(s, zc, parts, res, ticket, dbg);
   return cudaGetLastError();
 }
 
@@ -1196,7 +1219,7 @@ cudaError_t launch_ac(const Field3<E>& s, int T, int, double* parts, DevResults*
   template int64_t deriv_blocks<E>(const Field3<E>&, int);                                          \
   template int64_t ac_blocks<E>(const Field3<E>&, int);                                             \
   template cudaError_t launch_deriv<E>(const Field3<E>&, int, double*, DevResults*, unsigned int*,  \
-                                       cudaStream_t);                                               \
+                                       double*, cudaStream_t);                                      \
   template cudaError_t launch_ac<E>(const Field3<E>&, int, int, double*, DevResults*, unsigned int*, \
                                     cudaStream_t);
 CZC_P2_INST(float)

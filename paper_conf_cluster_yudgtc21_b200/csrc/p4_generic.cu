@@ -63,7 +63,8 @@ __device__ __forceinline__ void fields4(const T* __restrict__ f, int64_t c, cons
 
 template <typename T>
 __global__ void __launch_bounds__(kG4Threads)
-deriv4_kernel(Field4<T> s, double* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket) {
+deriv4_kernel(Field4<T> s, double* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket,
+              double* __restrict__ dbg) {
   double acc[kDerivSlots];
 #pragma unroll
   for (int k = 0; k < kDerivSlots; k++) acc[k] = op_identity(deriv_op(k));
@@ -79,6 +80,7 @@ deriv4_kernel(Field4<T> s, double* __restrict__ parts, DevResults* __restrict__ 
 #pragma unroll
     for (int fi = 0; fi < CZC_NDERIV; fi++) {
       const double d = Fy[fi] - Fx[fi];
+      if (dbg) dbg[fi * nI + i] = d;               // czc_config.debug_der: C order of the interior
       acc[fi * kDerivStats + 0] = fmax(acc[fi * kDerivStats + 0], fabs(d));
       acc[fi * kDerivStats + 1] += fabs(d);
       acc[fi * kDerivStats + 2] = fma(d, d, acc[fi * kDerivStats + 2]);
@@ -222,10 +224,10 @@ int64_t g4_max_blocks(int sms) { return (int64_t)sms * 8; }
 
 template <typename T>
 cudaError_t launch_deriv4(const T* x, const T* y, const int64_t n[4], int sms, double* parts, DevResults* res,
-                          unsigned int* ticket, cudaStream_t st) {
+                          unsigned int* ticket, double* dbg, cudaStream_t st) {
   const Field4<T> f = field4(x, y, n);
   const int64_t nI = (n[0] - 2) * (n[1] - 2) * (n[2] - 2) * (n[3] - 2);
-  deriv4_kernel<T><<<g4_grid(nI, sms), kG4Threads, 0, st>>>(f, parts, res, ticket);
+  deriv4_kernel<T><<<g4_grid(nI, sms), kG4Threads, 0, st>>>(f, parts, res, ticket, dbg);
   return cudaGetLastError();
 }
 
@@ -261,7 +263,7 @@ cudaError_t launch_ssim4(const T* x, const T* y, const int64_t n[4], const int w
 
 #define CZC_G4_INST(T)                                                                                         \
   template cudaError_t launch_deriv4<T>(const T*, const T*, const int64_t*, int, double*, DevResults*,         \
-                                        unsigned int*, cudaStream_t);                                          \
+                                        unsigned int*, double*, cudaStream_t);                                 \
   template cudaError_t launch_ac4<T>(const T*, const T*, const int64_t*, int, int, double*, DevResults*,       \
                                      unsigned int*, cudaStream_t);                                             \
   template cudaError_t launch_ssim4<T>(const T*, const T*, const int64_t*, const int*, const int*, int, int,   \

@@ -223,6 +223,20 @@ class TestDeriv:
             assert abs(r[f"{k}_mae"] - np.abs(d).mean()) < 1e-13 * scale, k
             assert abs(r[f"{k}_mse"] - (d * d).mean()) < 1e-12 * max(r[f"{k}_mse"], 1e-30) + 1e-26, k
 
+    @pytest.mark.parametrize("shape", [(9, 11, 13), (25, 31), (40,), (6, 1, 17)])
+    def test_points_against_numpy_scipy(self, orc, shape):
+        """czco_deriv_points (per-point dF, the reference of the CUDA debug_der output) against the
+        numpy.gradient / scipy.ndimage.laplace formulation, point by point."""
+        x, y = synth.make_pair(synth.config("C2", dims=shape))
+        x, y = x.numpy(), y.numpy()
+        got = orc.deriv_points(x, y)
+        Fx, Fy = _fields_numpy(x), _fields_numpy(y)
+        for i, k in enumerate(("der1", "der2", "grad", "div", "lap")):
+            want = (Fy[k] - Fx[k]).ravel()
+            scale = max(1.0, float(np.abs(Fx[k]).max()))
+            assert got.shape[1] == want.size
+            np.testing.assert_allclose(got[i], want, rtol=0, atol=1e-12 * scale, err_msg=k)
+
     def test_no_interior(self, orc):
         x = dyadic_field((2, 5, 5))
         r = orc.deriv(x, x)
