@@ -276,17 +276,26 @@ deriv2_kernel(Field3<T> s, int zchunk, double* __restrict__ parts, DevResults* _
   if (threadIdx.x == 0) *ticket = 0;
 }
 
+// Tile of the 3-D derivative kernel: kDerivTY rows, kDerivPTS points per thread (rows ty, ty + RY,
+// ...), kDerivMinB resident blocks per SM (float32; float64: one less).
+#ifndef CZC_DERIV_PTS
+#define CZC_DERIV_PTS 2
+#endif
+constexpr int kDerivPTS = CZC_DERIV_PTS;
+constexpr int kDerivTY = 4 * kDerivPTS;
+template <typename T> constexpr int deriv_minb() { return (kDerivPTS <= 2 ? 4 : 3) - (sizeof(T) == 8 ? 1 : 0); }
+
 // 3-D variant with two points per thread: threads (32, 4) cover a 32 x 8 tile, thread (tx, ty)
 // owns rows ty and ty + 4.  The 25 accumulators are shared by both points (half the registers
 // per point) and the two independent stencils double each warp's instruction-level parallelism.
-template <typename T, int PTS, bool DBG>
-__global__ void __launch_bounds__(kTX * kTY / PTS, sizeof(T) == 4 ? 4 : 3)
+template <typename T, int PTS, bool DBG, int TYD, int MINB>
+__global__ void __launch_bounds__(kTX * TYD / PTS, MINB)
 deriv3_kernel(Field3<T> s, int zc, double* __restrict__ parts, DevResults* __restrict__ res,
               unsigned int* __restrict__ ticket, double* __restrict__ dbg) {
-  constexpr int RY = kTY / PTS;                    // thread rows
-  constexpr int kHalo = 2 * (kTX + 2) + 2 * kTY;
+  constexpr int RY = TYD / PTS;                    // thread rows
+  constexpr int kHalo = 2 * (kTX + 2) + 2 * TYD;
   static_assert(kHalo <= kTX * RY, "halo larger than the block");
-  __shared__ double2 pl[2][kTY + 2][kTX + 2];
+  __shared__ double2 pl[2][TYD + 2][kTX + 2];
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * kTX + tx;
   int64_t zlo = 1, zhi = s.nz - 1;
   if (zlo < s.zown0) zlo = s.zown0;
@@ -298,7 +307,7 @@ deriv3_kernel(Field3<T> s, int zc, double* __restrict__ parts, DevResults* __res
   // DRAM once and from L2 by the neighbour (contiguous tile-major ranges left
   // neighbouring tiles planes apart and read the pair 2.13x per launch).  The chunk count is
   // chosen on the host so the rounds are nearly full.  The accumulators carry across units.
-  const int64_t ntxd = (s.nx + kTX - 1) / kTX, ntiles = ntxd * ((s.ny + kTY - 1) / kTY);
+  const int64_t ntxd = (s.nx + kTX - 1) / kTX, ntiles = ntxd * ((s.ny + TYD - 1) / TYD);
   const int64_t planes = zhi > zlo ? zhi - zlo : 0;
   const int64_t nch = planes > 0 ? (planes + zc - 1) / zc : 0, U = ntiles * nch;
 
@@ -310,7 +319,7 @@ deriv3_kernel(Field3<T> s, int zc, double* __restrict__ parts, DevResults* __res
   const int64_t bxi = tile % ntxd, byi = tile / ntxd;
   const int64_t zb = zlo + chunk * zc;
   const int64_t ze = zb + zc < zhi ? zb + zc : zhi;
-  const int64_t gx = bxi * kTX + tx, gy0 = byi * kTY + ty;
+  const int64_t gx = bxi * kTX + tx, gy0 = byi * TYD + ty;
   __syncthreads();                                   // the previous unit's readers are done with pl
 
   bool own[PTS], inxy[PTS];
@@ -323,9 +332,9 @@ deriv3_kernel(Field3<T> s, int zc, double* __restrict__ parts, DevResults* __res
   const int64_t col = own[0] ? gy0 * s.nx + gx : 0;  // point p: col + p * RY * nx
   const int64_t rstep = (int64_t)RY * s.nx;
   int hr = 0, hc = 0;
-  if (tid < 2 * (kTX + 2)) { hr = tid < kTX + 2 ? 0 : kTY + 1; hc = tid % (kTX + 2); }
-  else if (tid < kHalo) { const int t = tid - 2 * (kTX + 2); hr = 1 + t % kTY; hc = t < kTY ? 0 : kTX + 1; }
-  const int64_t hy = byi * kTY + hr - 1, hx = bxi * kTX + hc - 1;
+  if (tid < 2 * (kTX + 2)) { hr = tid < kTX + 2 ? 0 : TYD + 1; hc = tid % (kTX + 2); }
+  else if (tid < kHalo) { const int t = tid - 2 * (kTX + 2); hr = 1 + t % TYD; hc = t < TYD ? 0 : kTX + 1; }
+  const int64_t hy = byi * TYD + hr - 1, hx = bxi * kTX + hc - 1;
   const bool hown = tid < kHalo && hy >= 0 && hy < s.ny && hx >= 0 && hx < s.nx;
   const int64_t hcol = hown ? hy * s.nx + hx : 0;
 
@@ -1047,7 +1056,7 @@ static Field3<T> deriv_view(const Field3<T>& s) {
 // (4 rather than 8: C2 runs one 98-plane chunk per tile, derivatives 0.307 -> 0.290 ms).
 template <typename T>
 static dim3 deriv_grid(const Field3<T>& s, int zchunk, int* zc) {
-  const int bx = s.ny > 1 ? kTX : 256, by = s.ny > 1 ? kTY : 1;
+  const int bx = s.ny > 1 ? kTX : 256, by = s.ny > 1 ? (s.nz > 2 ? kDerivTY : kTY) : 1;
   const int64_t tiles = cdiv(s.nx, bx) * cdiv(s.ny, by), planes = deriv_zplanes(s);
   if (s.ny > 1 && s.nz > 2) {                 // deriv3_kernel: persistent, resident block count
     // z-chunks: the count whose round-robin rounds are fullest; a unit costs its planes plus ~1
@@ -1055,7 +1064,7 @@ static dim3 deriv_grid(const Field3<T>& s, int zchunk, int* zc) {
     // units: on C2, 12 units of 14 planes per block ran 0.281 ms against 0.268 ms for the old
     // contiguous split, 167 planes in ~2 pieces, at 2.1x the DRAM traffic); at most planes / 8
     // chunks
-    const int64_t G = (int64_t)sm_count() * (sizeof(T) == 4 ? 4 : 3);
+    const int64_t G = (int64_t)sm_count() * deriv_minb<T>();
     int64_t best = 1;
     double best_cost = 1e300;
     for (int64_t nch = 1; nch <= (planes / 8 > 1 ? planes / 8 : 1); nch++) {
@@ -1089,8 +1098,9 @@ cudaError_t launch_deriv(const Field3<T>& s0, int zchunk, double* parts, DevResu
   int zc;
   const dim3 grid = deriv_grid(s, zchunk, &zc);
   if (s.ny > 1 && s.nz > 2) {
-    if (dbg) deriv3_kernel<T, 2, true><<<grid, dim3(kTX, kTY / 2), 0, st>>>(s, zc, parts, res, ticket, dbg);
-    else deriv3_kernel<T, 2, false><<<grid, dim3(kTX, kTY / 2), 0, st>>>(s, zc, parts, res, ticket, dbg);
+    const dim3 blk(kTX, kDerivTY / kDerivPTS);
+    if (dbg) deriv3_kernel<T, kDerivPTS, true, kDerivTY, deriv_minb<T>()><<<grid, blk, 0, st>>>(s, zc, parts, res, ticket, dbg);
+    else deriv3_kernel<T, kDerivPTS, false, kDerivTY, deriv_minb<T>()><<<grid, blk, 0, st>>>(s, zc, parts, res, ticket, dbg);
   }
   else if (s.ny > 1) deriv_kernel<T, true, true, kTX, kTY><<<grid, dim3(kTX, kTY), 0, st>>>(s, zc, parts, res, ticket, dbg);
   else if (s.nz > 1) deriv2_kernel<T><<<grid, 256, 0, st>>>(s, zc, parts, res, ticket, dbg);
