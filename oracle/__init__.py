@@ -80,9 +80,12 @@ def _load():
         lib.czco_pdf.argtypes = [P, P, ctypes.c_uint64, ctypes.c_int, DP, DP, UP, DP, DP, UP, UP]
         lib.czco_ssim_windows.argtypes = [P, P, ctypes.c_int, I64P, I64P, I64P, ctypes.c_int, P]
         lib.czco_deriv_points.argtypes = [P, P, ctypes.c_int, I64P, P]
+        lib.czco_ssim_separable.argtypes = [P, P, ctypes.c_int, I64P, I64P, ctypes.c_int,
+                                            ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_uint64),
+                                            ctypes.POINTER(ctypes.c_uint64)]
         lib.czco_threads.restype = ctypes.c_int
         for name in ("czco_p1", "czco_deriv", "czco_autocorr", "czco_ssim_window", "czco_ssim", "czco_pdf",
-                     "czco_ssim_windows", "czco_deriv_points"):
+                     "czco_ssim_windows", "czco_deriv_points", "czco_ssim_separable"):
             f32, f64 = getattr(lib, name), getattr(lib, name + "_f64")
             f64.argtypes = f32.argtypes
             f64.restype = f32.restype
@@ -214,6 +217,23 @@ def ssim_windows(x, y, window, step=None, range_mode: int = 0, dims=None) -> np.
     if rc:
         raise ValueError(f"czco_ssim_windows failed ({rc})")
     return out.reshape(nw)
+
+
+def ssim_separable(x, y, window, range_mode: int = 0, dims=None):
+    """Separable SSIM (step 1, <= 3 active axes) for large fields: returns (ssim, n_windows,
+    n_brute), n_brute = windows recomputed by the brute force (czco_ssim_separable)."""
+    x, y = _pair(x, y)
+    nd, d = _dims(x, dims)
+    out = ctypes.c_double()
+    nw = ctypes.c_uint64()
+    nb = ctypes.c_uint64()
+    rc = _fn("czco_ssim_separable", x)(x.ctypes.data, y.ctypes.data, nd, d, _i64(window), range_mode,
+                                       ctypes.byref(out), ctypes.byref(nw), ctypes.byref(nb))
+    if rc == 3:
+        return float("nan"), 0, 0
+    if rc:
+        raise ValueError(f"czco_ssim_separable failed ({rc})")
+    return out.value, int(nw.value), int(nb.value)
 
 
 def pdf(x, y, nbins: int = 100) -> Dict:

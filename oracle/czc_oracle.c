@@ -9,6 +9,7 @@
  */
 #include "czc_oracle.h"
 
+#include <float.h>
 #include <math.h>
 #include <stdlib.h>
 #include <string.h>

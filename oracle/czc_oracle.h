@@ -67,6 +67,13 @@ double czco_ssim_window(const float* x, const float* y, int ndim, const int64_t*
 int czco_ssim(const float* x, const float* y, int ndim, const int64_t* dims, const int64_t* window,
               const int64_t* step, int range_mode, double* ssim, uint64_t* n_windows);
 
+/* Separable SSIM (step 1, up to three active axes) for fields too large for the brute force;
+ * the same definition as czco_ssim; *n_brute = windows recomputed by the brute force. */
+int czco_ssim_separable(const float* x, const float* y, int ndim, const int64_t* dims, const int64_t* window,
+                        int range_mode, double* ssim, uint64_t* n_windows, uint64_t* n_brute);
+int czco_ssim_separable_f64(const double* x, const double* y, int ndim, const int64_t* dims, const int64_t* window,
+                            int range_mode, double* ssim, uint64_t* n_windows, uint64_t* n_brute);
+
 /* Local SSIM of every valid window, C order of the window-origin grid (out: n_windows doubles);
  * returns 3 when there is no valid window. */
 int czco_ssim_windows(const float* x, const float* y, int ndim, const int64_t* dims, const int64_t* window,

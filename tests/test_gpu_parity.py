@@ -759,12 +759,17 @@ def test_full_size_2048_cubed_smooth_pair(czc, orc):
     org = rng.integers(0, n - 7, size=(1500, 3))
     oi = torch.from_numpy(org).cuda()
     gw = dbg[oi[:, 0], oi[:, 1], oi[:, 2]].cpu().numpy()
+    slab_mean = float(dbg[:256].sum(dtype=torch.float64).item()) / dbg[:256].numel()
     del dbg
     xn, yn = xd.cpu().numpy(), yd.cpu().numpy()
     del xd, yd
     torch.cuda.empty_cache()
     worst = max(abs(gw[i] - orc.ssim_window(xn, yn, list(org[i]), [8, 8, 8])) for i in range(len(org)))
     assert worst < 1e-6, worst
+    # the mean of the 1.06e9 windows with origin planes 0..255 (an eighth of the field) against the
+    # separable oracle (brute force would take ~5e11 element visits)
+    sep, nws, nbr = orc.ssim_separable(xn[:263], yn[:263], [8, 8, 8])
+    assert nws == 256 * (n - 7) ** 2 and abs(slab_mean - sep) < 1e-9, (slab_mean, sep, nbr)
     import time
     t0 = time.perf_counter()
     errors = []
@@ -775,4 +780,5 @@ def test_full_size_2048_cubed_smooth_pair(czc, orc):
     report(errors)
     print(f"oracle over 2048^3: {time.perf_counter() - t0:.0f} s on {orc.threads()} threads")
     print(f"C5 2048^3: psnr {g['psnr']:.4f} ssim {g['ssim']:.9f} exact windows {g['n_ssim_exact']} "
-          f"worst sampled window {worst:.2e}")
+          f"worst sampled window {worst:.2e}; planes 0..255: gpu mean {slab_mean:.15f} separable "
+          f"oracle {sep:.15f} ({nbr} brute-forced)")

@@ -383,6 +383,37 @@ class TestSSIM:
         np.testing.assert_allclose(got.ravel(), ref, rtol=0, atol=1e-12)
         assert abs(got.mean() - orc.ssim(x, y, [w] * len(shape), [s] * len(shape))[0]) < 1e-14
 
+    @pytest.mark.parametrize("cfg,shape,w,kw", [("C1", (20, 24, 28), 7, {}), ("C2q", (18, 30, 33), 8, {}),
+                                                ("C3", (17, 20, 25), 5, {}), ("C4", (60, 90), 8, {}),
+                                                ("C2", (10, 11, 40), 8, {}), ("C4", (1, 300), 9, {}),
+                                                ("C1", (10, 9, 14), 5, {"kind": "step", "eb": 0.1})])
+    def test_separable_equals_brute_force(self, orc, cfg, shape, w, kw):
+        """czco_ssim_separable (the C5-scale SSIM oracle: separable direct box sums in long double,
+        textbook formula) reproduces the per-window brute force czco_ssim; on the step field the
+        windows its cancellation bound rejects are recomputed by the brute force."""
+        x, y = synth.make_pair(synth.config(cfg, dims=shape, **kw))
+        x, y = x.numpy(), y.numpy()
+        if shape[0] == 1:
+            x, y = x[0].copy(), y[0].copy()
+        win = [w] * x.ndim
+        ref, nw = orc.ssim(x, y, win)
+        got, nw2, nb = orc.ssim_separable(x, y, win)
+        assert nw2 == nw and abs(got - ref) < 1e-13
+        gr, _ = orc.ssim(x, y, win, range_mode=1)
+        assert abs(orc.ssim_separable(x, y, win, range_mode=1)[0] - gr) < 1e-13
+        if kw.get("kind") == "step":
+            assert nb > 0
+
+    def test_separable_closed_forms(self, orc):
+        """Zero error -> 1; constant field x = v, y = v + c -> A / (A + c^2) (L = 0 -> 1)."""
+        x, _ = synth.make_pair(synth.config("C2", dims=(12, 16, 20)))
+        assert abs(orc.ssim_separable(x, x, [5, 5, 5])[0] - 1.0) < 1e-15
+        v, c = 0.75, 2.0 ** -8
+        xc = np.full((9, 10, 11), v, np.float32)
+        yc = np.full((9, 10, 11), v + c, np.float32)
+        A = 2 * v * (v + c) + 1e-4
+        assert abs(orc.ssim_separable(xc, yc, [4, 4, 4])[0] - A / (A + c * c)) < 1e-15
+
     def test_no_window(self, orc):
         x = dyadic_field((5, 5, 5))
         s, nw = orc.ssim(x, x, [6, 6, 6])
