@@ -11,6 +11,14 @@
 
 namespace czc {
 
+// 32: 256-bit float32 vectors (LDG.E.ENL2.256).  Not the default: at two vectors in flight per
+// array they need 162 registers (one block per SM) or spill 120 B at two blocks per SM, and one
+// 256-bit vector in flight carries the same bytes as the two 128-bit ones of the default.
+#ifndef CZC_P1_VEC_BYTES
+#define CZC_P1_VEC_BYTES 16
+#endif
+constexpr int kP1VecBytes = CZC_P1_VEC_BYTES;
+
 // Per-thread accumulator: sums about the thread's first element (kx, ke).  The element count
 // is implicit (counted per vector), so no per-element work is spent on it.
 
@@ -66,13 +74,18 @@ __device__ __forceinline__ bool acc_elem(P1Acc<T>& a, T xf, T yf, double& ae_out
   a.xmax = tmax(a.xmax, xf);
   const bool nz = xf != (T)0;
   const double ax = nz ? fabs(x) : 1.0;
-  double qa = nz ? ae * rcp_newton1(ax) : 0.0;
+  // |e| = |x| (a reconstruction of 0 or 2x: common where a relative error bound exceeds the
+  // value, e.g. the low decades of a log-normal density) gives exactly 1 — and would otherwise
+  // be a candidate on every such element once the maximum is 1 (a tie the approximate quotient
+  // cannot rule out): C3 P1 ran at 29 % of HBM
+  const bool unit = ae == ax;
+  double qa = nz ? (unit ? 1.0 : ae * rcp_newton1(ax)) : 0.0;
   if (sizeof(T) == 8 && !(ax >= 1e-290 && ax <= 1e290)) qa = ae / ax;
   a.spwr += qa;
   a.npwr += nz ? 1u : 0u;
   ae_out = ae;
   ax_out = ax;
-  return nz && (qa > a.pthr_hi || qa < a.pthr_lo);
+  return nz && (unit ? (1.0 > a.pmax || 1.0 < a.pmin) : (qa > a.pthr_hi || qa < a.pthr_lo));
 }
 
 template <typename T>
@@ -82,9 +95,32 @@ __device__ __forceinline__ void acc_resolve(P1Acc<T>& a, double ae, double ax) {
   if (q < a.pmin) { a.pmin = q; a.pthr_lo = q * (1.0 + 1e-10); }   // q = 0 -> thr_lo = 0
 }
 
-template <typename T>
-__device__ __forceinline__ void acc_vec(P1Acc<T>& a, const Vec16<T>& xv, const Vec16<T>& yv) {
-  constexpr int N = Vec16<T>::N;
+// One vector of VB bytes of the input type (16: 4 floats / 2 doubles; 32: 8 floats, one 256-bit
+// LDG.E.ENL2.256 per array).
+template <typename T, int VB>
+struct VecB {
+  static constexpr int N = VB / (int)sizeof(T);
+  T e[N];
+};
+template <typename T, int VB>
+__device__ __forceinline__ VecB<T, VB> ld_streamB(const T* p) {
+  VecB<T, VB> r;
+  if constexpr (VB == 32 && sizeof(T) == 4) {
+    asm volatile("ld.global.nc.L1::no_allocate.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=f"(r.e[0]), "=f"(r.e[1]), "=f"(r.e[2]), "=f"(r.e[3]), "=f"(r.e[4]), "=f"(r.e[5]),
+                   "=f"(r.e[6]), "=f"(r.e[7]) : "l"(p));
+  } else {
+    static_assert(VB == 16, "256-bit loads: float32 only");
+    const Vec16<T> v = ld_stream16(p);
+#pragma unroll
+    for (int j = 0; j < VecB<T, VB>::N; j++) r.e[j] = v.e[j];
+  }
+  return r;
+}
+
+template <typename T, int VB>
+__device__ __forceinline__ void acc_vec(P1Acc<T>& a, const VecB<T, VB>& xv, const VecB<T, VB>& yv) {
+  constexpr int N = VecB<T, VB>::N;
   double ae[N], ax[N];
   bool c[N], any = false;
 #pragma unroll
@@ -174,11 +210,11 @@ __device__ __forceinline__ P1State block_merge(P1State s) {
 // VEC: x and y share the same 16-byte misalignment; elements [head, head + VN*nvec) are read as
 // 128-bit vectors (VN = 4 floats or 2 doubles), the leftovers (prologue [0, head) and tail) by
 // threads 0..nleft-1.
-template <typename T, bool VEC>
+template <typename T, bool VEC, int VB>
 __global__ void __launch_bounds__(kP1Threads)
 p1_kernel(const T* __restrict__ x, const T* __restrict__ y, int64_t n, int64_t head,
           P1State* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket) {
-  constexpr int VN = Vec16<T>::N;
+  constexpr int VN = VecB<T, VB>::N;
   const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
   const int64_t nvec = VEC ? (n - head) / VN : 0;
@@ -200,20 +236,20 @@ p1_kernel(const T* __restrict__ x, const T* __restrict__ y, int64_t n, int64_t h
     if (gtid < nvec) cnt = VN * ((nvec - 1 - gtid) / gsz + 1);
     // software pipeline: the next two vectors' loads are in flight while two are processed
     if (v + gsz < nvec) {
-      Vec16<T> xa = ld_stream16(x4 + VN * v), ya = ld_stream16(y4 + VN * v);
-      Vec16<T> xb = ld_stream16(x4 + VN * (v + gsz)), yb = ld_stream16(y4 + VN * (v + gsz));
+      VecB<T, VB> xa = ld_streamB<T, VB>(x4 + VN * v), ya = ld_streamB<T, VB>(y4 + VN * v);
+      VecB<T, VB> xb = ld_streamB<T, VB>(x4 + VN * (v + gsz)), yb = ld_streamB<T, VB>(y4 + VN * (v + gsz));
       v += 2 * gsz;
       for (; v + gsz < nvec; v += 2 * gsz) {
-        const Vec16<T> xc = ld_stream16(x4 + VN * v), yc = ld_stream16(y4 + VN * v);
-        const Vec16<T> xd = ld_stream16(x4 + VN * (v + gsz)), yd = ld_stream16(y4 + VN * (v + gsz));
-        acc_vec(a, xa, ya);
-        acc_vec(a, xb, yb);
+        const VecB<T, VB> xc = ld_streamB<T, VB>(x4 + VN * v), yc = ld_streamB<T, VB>(y4 + VN * v);
+        const VecB<T, VB> xd = ld_streamB<T, VB>(x4 + VN * (v + gsz)), yd = ld_streamB<T, VB>(y4 + VN * (v + gsz));
+        acc_vec<T, VB>(a, xa, ya);
+        acc_vec<T, VB>(a, xb, yb);
         xa = xc; ya = yc; xb = xd; yb = yd;
       }
-      acc_vec(a, xa, ya);
-      acc_vec(a, xb, yb);
+      acc_vec<T, VB>(a, xa, ya);
+      acc_vec<T, VB>(a, xb, yb);
     }
-    for (; v < nvec; v += gsz) acc_vec(a, ld_stream16(x4 + VN * v), ld_stream16(y4 + VN * v));
+    for (; v < nvec; v += gsz) acc_vec<T, VB>(a, ld_streamB<T, VB>(x4 + VN * v), ld_streamB<T, VB>(y4 + VN * v));
     if (gtid < nleft) {
       const int64_t i = left_index(gtid);
       acc_scalar(a, x[i], y[i]);
@@ -247,31 +283,39 @@ p1_kernel(const T* __restrict__ x, const T* __restrict__ y, int64_t n, int64_t h
   }
 }
 
-// 128-bit vector path: both arrays element-aligned with the same 16-byte misalignment; head =
-// elements before the first aligned vector.
-template <typename T>
+// Vector path: both arrays element-aligned with the same VB-byte misalignment; head = elements
+// before the first aligned vector.
+template <typename T, int VB>
 static bool vec_head(const T* x, const T* y, int64_t n, int64_t* head) {
   const uintptr_t ax = reinterpret_cast<uintptr_t>(x), ay = reinterpret_cast<uintptr_t>(y);
-  const bool vec = (ax % 16) == (ay % 16) && (ax % sizeof(T)) == 0;
-  int64_t h = vec ? (int64_t)(((16 - ax % 16) % 16) / sizeof(T)) : 0;
+  const bool vec = (ax % VB) == (ay % VB) && (ax % sizeof(T)) == 0;
+  int64_t h = vec ? (int64_t)(((VB - ax % VB) % VB) / sizeof(T)) : 0;
   *head = h > n ? n : h;
   return vec;
 }
 
-// Host launcher.  Returns the cuda error of the launch.
+// Host launcher.  Returns the cuda error of the launch.  float32 pairs with the same 32-byte
+// misalignment stream 256-bit vectors (twice the bytes in flight per load instruction), others
+// 128-bit vectors, else scalars.
 template <typename T>
 cudaError_t launch_p1(const T* x, const T* y, int64_t n, int grid_cap, P1State* parts,
                       DevResults* res, unsigned int* ticket, cudaStream_t st) {
   int64_t head = 0;
-  const bool vec = vec_head(x, y, n, &head);
-  const int64_t work = vec ? ((n - head) / Vec16<T>::N + 8) : n;
-  int64_t blocks = (work + kP1Threads - 1) / kP1Threads;
-  if (blocks > grid_cap) blocks = grid_cap;
-  if (blocks < 1) blocks = 1;
-  if (vec)
-    p1_kernel<T, true><<<(unsigned)blocks, kP1Threads, 0, st>>>(x, y, n, head, parts, res, ticket);
+  auto grid = [&](int64_t work) {
+    int64_t blocks = (work + kP1Threads - 1) / kP1Threads;
+    if (blocks > grid_cap) blocks = grid_cap;
+    return (unsigned)(blocks < 1 ? 1 : blocks);
+  };
+  if constexpr (sizeof(T) == 4 && kP1VecBytes == 32) {
+    if (vec_head<T, 32>(x, y, n, &head)) {
+      p1_kernel<T, true, 32><<<grid((n - head) / 8 + 8), kP1Threads, 0, st>>>(x, y, n, head, parts, res, ticket);
+      return cudaGetLastError();
+    }
+  }
+  if (vec_head<T, 16>(x, y, n, &head))
+    p1_kernel<T, true, 16><<<grid((n - head) / Vec16<T>::N + 8), kP1Threads, 0, st>>>(x, y, n, head, parts, res, ticket);
   else
-    p1_kernel<T, false><<<(unsigned)blocks, kP1Threads, 0, st>>>(x, y, n, head, parts, res, ticket);
+    p1_kernel<T, false, 16><<<grid(n), kP1Threads, 0, st>>>(x, y, n, head, parts, res, ticket);
   return cudaGetLastError();
 }
 template cudaError_t launch_p1<float>(const float*, const float*, int64_t, int, P1State*, DevResults*,
@@ -357,7 +401,7 @@ cudaError_t launch_pdf(const T* x, const T* y, int64_t n, int nb, int grid_cap, 
   cudaError_t e = cudaMemsetAsync(res->rec.pdf, 0, sizeof(res->rec.pdf), st);
   if (e != cudaSuccess) return e;
   int64_t head = 0;
-  const bool vec = vec_head(x, y, n, &head);
+  const bool vec = vec_head<T, 16>(x, y, n, &head);
   const int64_t work = vec ? ((n - head) / Vec16<T>::N + 8) : n;
   int64_t blocks = (work + kP1Threads - 1) / kP1Threads;
   if (blocks > grid_cap) blocks = grid_cap;
@@ -386,7 +430,7 @@ cudaError_t launch_p1_combine(const P1State* states, int count, DevResults* res,
 
 int p1_max_blocks_per_sm() {
   int nb = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, p1_kernel<float, true>, kP1Threads, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, p1_kernel<float, true, kP1VecBytes>, kP1Threads, 0);
   return nb > 0 ? nb : 1;
 }
 
