@@ -78,8 +78,14 @@ struct czc_ctx {
   DevResults* dres = nullptr;      // device
   Record* hrec = nullptr;          // pinned host, max_records records
   unsigned int* tickets = nullptr; // device
-  void* parts = nullptr;           // per-block partial records
+  void* parts = nullptr;           // per-block partial records: one region per kernel kind
   size_t parts_cap = 0;
+  size_t off_deriv = 0, off_ac = 0, off_ssim = 0;   // byte offsets (P1 at 0) set by ensure_scratch
+  // the single-GPU sequence as two concurrent branches (P1 -> AC | derivatives -> SSIM)
+  cudaStream_t stream2 = nullptr, stream3 = nullptr;
+  cudaEvent_t fork_ev = nullptr, join_ev = nullptr, join3_ev = nullptr, p1_ev = nullptr;
+  bool concurrent = true;          // CZC_SEQUENTIAL=1: one stream (A/B timing)
+  int layout = 0;                  // CZC_BRANCHES (A/B): 0 P1>AC | deriv>SSIM, 1 P1>AC>deriv | SSIM, 2 P1>AC | deriv | SSIM
   void* din[2] = {nullptr, nullptr};    // staging for czc_assess_host
   size_t din_cap = 0;
   cudaEvent_t ev[6] = {};   // P1 start, P1 end, deriv end, AC end, SSIM end, call end
@@ -165,6 +171,10 @@ extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
   {
     const char* ng = getenv("CZC_NO_GRAPHS");
     ctx->use_graphs = !(ng && ng[0] == '1');
+    const char* sq = getenv("CZC_SEQUENTIAL");
+    ctx->concurrent = !(sq && sq[0] == '1');
+    const char* br = getenv("CZC_BRANCHES");
+    ctx->layout = br ? atoi(br) : 0;
   }
   ctx->max_records = std::max(kMaxHostChunks, std::max(c.nranks, c.loopback_slabs));
   do {
@@ -201,6 +211,15 @@ extern "C" czc_status czc_init(czc_ctx** out, const czc_config* cfg) {
     for (int i = 0; i < 6 && st == CZC_OK; i++)
       if ((e = cudaEventCreate(&ctx->ev[i])) != cudaSuccess) st = cuda_fail(ctx, e, "cudaEventCreate");
     if (st != CZC_OK) break;
+    if ((e = cudaStreamCreateWithFlags(&ctx->stream2, cudaStreamNonBlocking)) != cudaSuccess ||
+        (e = cudaStreamCreateWithFlags(&ctx->stream3, cudaStreamNonBlocking)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&ctx->join3_ev, cudaEventDisableTiming)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&ctx->fork_ev, cudaEventDisableTiming)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&ctx->join_ev, cudaEventDisableTiming)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&ctx->p1_ev, cudaEventDisableTiming)) != cudaSuccess) {
+      st = cuda_fail(ctx, e, "second stream");
+      break;
+    }
     {
       if ((e = cudaMalloc(&ctx->dgather_in, 64)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(gather)"); break; }
       if ((e = cudaMalloc(&ctx->dgather, rb)) != cudaSuccess) { st = cuda_fail(ctx, e, "cudaMalloc(gather)"); break; }
@@ -249,6 +268,10 @@ extern "C" void czc_free(czc_ctx* ctx) {
     if (ctx->copy_stream[c]) cudaStreamDestroy(ctx->copy_stream[c]);
   }
   if (ctx->gexec) cudaGraphExecDestroy(ctx->gexec);
+  for (cudaStream_t sx : {ctx->stream2, ctx->stream3})
+    if (sx) { cudaStreamSynchronize(sx); cudaStreamDestroy(sx); }
+  for (cudaEvent_t ev : {ctx->fork_ev, ctx->join_ev, ctx->join3_ev, ctx->p1_ev})
+    if (ev) cudaEventDestroy(ev);
   for (int i = 0; i < 2; i++)
     if (ctx->halo_ev[i]) cudaEventDestroy(ctx->halo_ev[i]);
   if (ctx->halo_stream) cudaStreamDestroy(ctx->halo_stream);
@@ -500,45 +523,65 @@ int64_t halo_depth(const Plan& P) {
 }
 }  // namespace
 
-// Scratch for the largest launch over the given field view.
+// Scratch for every launch over the given field view: one region per kernel kind (P1 at offset
+// 0, then derivatives, AC, SSIM), so kernels of different kinds may run concurrently.
 template <typename E>
 static czc_status ensure_scratch(czc_ctx* ctx, const Plan& P, const Field3<E>& F, const SsimParams& sp) {
-  size_t need = (size_t)ctx->p1_grid_cap * sizeof(P1State);
-  if (P.run_deriv) need = std::max(need, (size_t)deriv_blocks(F, kZchunkDeriv) * kDerivSlots * sizeof(double));
-  if (P.run_ac) need = std::max(need, (size_t)ac_blocks(F, P.T) * kAcSlots * sizeof(double));
+  auto al = [](size_t b) { return (b + 255) / 256 * 256; };
+  const size_t p1 = al((size_t)ctx->p1_grid_cap * sizeof(P1State));
+  const size_t dv = P.run_deriv ? al((size_t)deriv_blocks(F, kZchunkDeriv) * kDerivSlots * sizeof(double)) : 0;
+  const size_t ac = P.run_ac ? al((size_t)ac_blocks(F, P.T) * kAcSlots * sizeof(double)) : 0;
+  size_t ss = 0;
   if (P.run_ssim) {
     int64_t nb = 0;
     if (launch_ssim(P.kind, P.W, F, sp, nullptr, nullptr, nullptr, nullptr, ctx->stream, &nb) != cudaSuccess) {
       ctx->last_error = "unsupported SSIM window";
       return CZC_ERR_UNSUPPORTED;
     }
-    need = std::max(need, (size_t)nb * kSsimSlots * sizeof(double));
+    ss = al((size_t)nb * kSsimSlots * sizeof(double));
   }
-  return ensure_buf(ctx, &ctx->parts, &ctx->parts_cap, need);
+  czc_status st = ensure_buf(ctx, &ctx->parts, &ctx->parts_cap, p1 + dv + ac + ss);
+  if (st != CZC_OK) return st;
+  ctx->off_deriv = p1;
+  ctx->off_ac = p1 + dv;
+  ctx->off_ssim = p1 + dv + ac;
+  return CZC_OK;
+}
+static double* parts_at(czc_ctx* ctx, size_t off) { return reinterpret_cast<double*>(static_cast<char*>(ctx->parts) + off); }
+
+// The kernels of P2 / P3 over one field view (the owned planes of F); results land in dres->rec.
+template <typename E>
+static czc_status launch_deriv_k(czc_ctx* ctx, const Field3<E>& F, cudaStream_t s) {
+  NvtxRange r_("czc/P2 derivatives");
+  CZC_CUDA(ctx, launch_deriv(F, kZchunkDeriv, parts_at(ctx, ctx->off_deriv), ctx->dres, ctx->tickets + TICKET_DERIV,
+                             ctx->cfg.debug_der, s));
+  return CZC_OK;
+}
+template <typename E>
+static czc_status launch_ac_k(czc_ctx* ctx, const Plan& P, const Field3<E>& F, cudaStream_t s) {
+  NvtxRange r_("czc/P2 autocorrelation");
+  CZC_CUDA(ctx, launch_ac(F, P.T, 0, parts_at(ctx, ctx->off_ac), ctx->dres, ctx->tickets + TICKET_ACZ, s));
+  return CZC_OK;
+}
+template <typename E>
+static czc_status launch_ssim_k(czc_ctx* ctx, const Plan& P, const Field3<E>& F, const SsimParams& sp, cudaStream_t s) {
+  NvtxRange r_("czc/P3 SSIM");
+  CZC_CUDA(ctx, launch_ssim(P.kind, P.W, F, sp, parts_at(ctx, ctx->off_ssim), ctx->dres, ctx->tickets + TICKET_SSIM,
+                            ctx->cfg.debug_wssim, s, nullptr));
+  return CZC_OK;
 }
 
-// P2 + P3 over one field view (the owned planes of F); results land in dres->rec.
+// P2 + P3 in sequence on the context stream.
 template <typename E>
 static czc_status run_p23(czc_ctx* ctx, const Plan& P, const Field3<E>& F, const SsimParams& sp) {
   const cudaStream_t s = ctx->stream;
   czc_status st = ensure_scratch(ctx, P, F, sp);
   if (st != CZC_OK) return st;
-  if (P.run_deriv) {
-    NvtxRange r_("czc/P2 derivatives");
-    CZC_CUDA(ctx, launch_deriv(F, kZchunkDeriv, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_DERIV,
-                               ctx->cfg.debug_der, s));
-  }
+  if (P.run_deriv && (st = launch_deriv_k(ctx, F, s)) != CZC_OK) return st;
   if (ctx->cfg.timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
-  if (P.run_ac) {
-    NvtxRange r_("czc/P2 autocorrelation");
-    CZC_CUDA(ctx, launch_ac(F, P.T, 0, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_ACZ, s));
-  }
+  if (P.run_ac && (st = launch_ac_k(ctx, P, F, s)) != CZC_OK) return st;
   if (ctx->cfg.timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));
-  if (P.run_ssim) {
-    NvtxRange r_("czc/P3 SSIM");
-    CZC_CUDA(ctx, launch_ssim(P.kind, P.W, F, sp, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_SSIM,
-                              ctx->cfg.debug_wssim, s, nullptr));
-  }
+  if (P.run_ssim && (st = launch_ssim_k(ctx, P, F, sp, s)) != CZC_OK) return st;
   return CZC_OK;
 }
 
@@ -566,7 +609,11 @@ static void finish_timing(czc_ctx* ctx, czc_result* out) {
   out->kernel_ms[5] = 0.f;
 }
 
-// The single-GPU launch sequence: P1 (+ PDF), P2, P3, the D2H copy of the record.
+// The single-GPU launch sequence: P1 (+ PDF), P2, P3, the D2H copy of the record.  Without
+// per-kernel timing it runs as two concurrent branches joined before the record copy — the
+// context stream: P1 (+ PDF) -> AC (which needs P1's mean / variance of the error, Alg. 2);
+// the second stream: derivatives -> SSIM (which needs P1 only for the global range mode) — so
+// the memory-latency-bound P1 and the FP64-bound stencil / window kernels can share the SMs.
 template <typename E>
 static czc_status enqueue_single(czc_ctx* ctx, const Plan& P, const E* x, const E* y, const Field3<E>& F,
                                  const SsimParams& sp) {
@@ -574,6 +621,36 @@ static czc_status enqueue_single(czc_ctx* ctx, const Plan& P, const E* x, const 
   const bool timing = ctx->cfg.timing != 0;
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
   NvtxRange r_("czc/enqueue");
+  if (!timing && ctx->concurrent && (P.run_deriv || P.run_ssim)) {
+    const int L = ctx->layout;
+    const cudaStream_t s2 = ctx->stream2, s3 = ctx->stream3;
+    const cudaStream_t sd = L == 1 ? s : s2;            // derivatives
+    const cudaStream_t ss = L == 2 ? s3 : s2;           // SSIM
+    czc_status st = ensure_scratch(ctx, P, F, sp);
+    if (st != CZC_OK) return st;
+    CZC_CUDA(ctx, cudaEventRecord(ctx->fork_ev, s));
+    CZC_CUDA(ctx, cudaStreamWaitEvent(s2, ctx->fork_ev, 0));
+    if (L == 2) CZC_CUDA(ctx, cudaStreamWaitEvent(s3, ctx->fork_ev, 0));
+    if (P.run_deriv && sd != s && (st = launch_deriv_k(ctx, F, sd)) != CZC_OK) return st;
+    if (P.run_ssim && sp.range_mode == 0 && (st = launch_ssim_k(ctx, P, F, sp, ss)) != CZC_OK) return st;
+    if ((st = p1_local(ctx, P, x, y, F.nz * F.ny * F.nx)) != CZC_OK) return st;
+    if (P.run_pdf) CZC_CUDA(ctx, launch_pdf(x, y, F.nz * F.ny * F.nx, P.nb, ctx->p1_grid_cap, ctx->dres, s));
+    if (P.run_ssim && sp.range_mode != 0) {            // the global range comes from P1
+      CZC_CUDA(ctx, cudaEventRecord(ctx->p1_ev, s));
+      CZC_CUDA(ctx, cudaStreamWaitEvent(ss, ctx->p1_ev, 0));
+      if ((st = launch_ssim_k(ctx, P, F, sp, ss)) != CZC_OK) return st;
+    }
+    if (P.run_ac && (st = launch_ac_k(ctx, P, F, s)) != CZC_OK) return st;
+    if (P.run_deriv && sd == s && (st = launch_deriv_k(ctx, F, s)) != CZC_OK) return st;
+    CZC_CUDA(ctx, cudaEventRecord(ctx->join_ev, s2));
+    CZC_CUDA(ctx, cudaStreamWaitEvent(s, ctx->join_ev, 0));
+    if (L == 2) {
+      CZC_CUDA(ctx, cudaEventRecord(ctx->join3_ev, s3));
+      CZC_CUDA(ctx, cudaStreamWaitEvent(s, ctx->join3_ev, 0));
+    }
+    CZC_CUDA(ctx, copy_records(ctx->hrec, &ctx->dres->rec, 1, P.run_pdf, s));
+    return CZC_OK;
+  }
   czc_status st = p1_local(ctx, P, x, y, F.nz * F.ny * F.nx);
   if (st != CZC_OK) return st;
   if (P.run_pdf) CZC_CUDA(ctx, launch_pdf(x, y, F.nz * F.ny * F.nx, P.nb, ctx->p1_grid_cap, ctx->dres, s));
@@ -1077,7 +1154,7 @@ static czc_status assess_host_pipelined(czc_ctx* ctx, const Plan& P, const E* hx
     F.zown1 = nz;
     czc_status st = ensure_scratch(ctx, P, F, sp);
     if (st != CZC_OK) return st;
-    CZC_CUDA(ctx, launch_ac(F, P.T, 0, (double*)ctx->parts, ctx->dres, ctx->tickets + TICKET_ACZ, s));
+    CZC_CUDA(ctx, launch_ac(F, P.T, 0, parts_at(ctx, ctx->off_ac), ctx->dres, ctx->tickets + TICKET_ACZ, s));
     CZC_CUDA(ctx, cudaMemcpyAsync(drec[0].ac, ctx->dres->rec.ac, sizeof(drec[0].ac), cudaMemcpyDeviceToDevice, s));
   }
   if (timing) CZC_CUDA(ctx, cudaEventRecord(ctx->ev[3], s));

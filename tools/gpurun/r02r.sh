@@ -1,0 +1,2 @@
+python tools/ab_concurrent.py C2 C3
+timeout 1500 python -m pytest tests -m gpu -q -x --deselect tests/test_gpu_parity.py::test_full_size_2048_cubed_smooth_pair 2>&1 | tail -2
