@@ -849,7 +849,9 @@ static czc_status assess_ranks(czc_ctx* ctx, const Plan& P, const E* x, const E*
   const size_t pb = (size_t)plane * sizeof(E);
   const SsimParams sp = ssim_params(P, ctx->cfg);
   E *xlo, *ylo, *xhi, *yhi;
-  const std::vector<int64_t> key = {z0, nzl, nz, P.g3[1], P.g3[2], H, P.run_deriv, (int64_t)sizeof(E)};
+  // the call signature: everything the buffers and the scratch layout depend on
+  const std::vector<int64_t> key = {z0, nzl, nz, P.g3[1], P.g3[2], H, (int64_t)sizeof(E), P.run_p1, P.run_deriv,
+                                    P.run_ac, P.run_ssim, P.run_pdf, P.W, P.T, P.kind, P.step[0], P.step[1], P.step[2]};
   if (key != ctx->slab_key) {
     ctx->slab_key.clear();
     // allocate first (halo planes, kernel scratch), then one collective decision
@@ -917,6 +919,17 @@ static czc_status assess_ranks(czc_ctx* ctx, const Plan& P, const E* x, const E*
   }
   if (!comm_group_end(&ctx->last_error) || !ok) return fail(CZC_ERR_COMM);
   CZC_SLAB(cudaEventRecord(ctx->halo_ev[1], hs));
+  // The derivatives and local-range SSIM need only the slab and its halo: without per-kernel
+  // timing they run on the second stream as soon as the halo is in (the single-GPU branch
+  // layout, enqueue_single), concurrently with P1, its allgather and AC on the compute stream.
+  const bool branch = !timing && ctx->concurrent;
+  const bool ssim_early = P.run_ssim && sp.range_mode == 0;
+  czc_status st = CZC_OK;
+  if (branch) {
+    CZC_SLAB(cudaStreamWaitEvent(ctx->stream2, ctx->halo_ev[1], 0));
+    if (P.run_deriv && (st = launch_deriv_k(ctx, F, ctx->stream2)) != CZC_OK) return fail(st);
+    if (ssim_early && (st = launch_ssim_k(ctx, P, F, sp, ctx->stream2)) != CZC_OK) return fail(st);
+  }
   // P1 on the local slab (overlaps the halo transfer), one small allgather of the states, merged
   // in rank order on the device
   if (P.run_p1) {
@@ -927,8 +940,14 @@ static czc_status assess_ranks(czc_ctx* ctx, const Plan& P, const E* x, const E*
   if (P.run_pdf) CZC_SLAB(launch_pdf(x, y, nzl * plane, P.nb, ctx->p1_grid_cap, ctx->dres, s));
   if (timing) CZC_SLAB(cudaEventRecord(ctx->ev[1], s));
   CZC_SLAB(cudaStreamWaitEvent(s, ctx->halo_ev[1], 0));
-  czc_status st = run_p23(ctx, P, F, sp);               // scratch sized above: no allocation
-  if (st != CZC_OK) return fail(st);
+  if (branch) {                                          // scratch sized above: no allocation
+    if (P.run_ac && (st = launch_ac_k(ctx, P, F, s)) != CZC_OK) return fail(st);
+    if (P.run_ssim && !ssim_early && (st = launch_ssim_k(ctx, P, F, sp, s)) != CZC_OK) return fail(st);
+    CZC_SLAB(cudaEventRecord(ctx->join_ev, ctx->stream2));
+    CZC_SLAB(cudaStreamWaitEvent(s, ctx->join_ev, 0));
+  } else if ((st = run_p23(ctx, P, F, sp)) != CZC_OK) {
+    return fail(st);
+  }
   if (timing) CZC_SLAB(cudaEventRecord(ctx->ev[4], s));
   // every rank's record, combined in rank order on the host; plus the slab check of this call
   if (!comm_allgather(ctx->comm, &ctx->dres->rec, ctx->dgather, sizeof(Record), s, &ctx->last_error)) return fail(CZC_ERR_COMM);

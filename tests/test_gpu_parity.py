@@ -244,12 +244,22 @@ def test_nccl_slab_path_single_rank(czc):
         g1 = a.assess(xd, yd)
     uid = bench.czc_nccl_uid()
     with czc.Assessor(ssim_window=8, rank=0, nranks=1, nccl_uid=uid) as a:
-        g = a.assess(xd, yd, dims=xd.shape, z0=0)
+        # repeated calls (cached slab signature), a mask change (new signature: re-validated and
+        # re-allocated before any collective), then the first mask again
+        for mask in (czc.M_ALL, czc.M_ALL, czc.M_SSIM | czc.M_DERIV, czc.M_ALL):
+            g = a.assess(xd, yd, mask, dims=xd.shape, z0=0)
+            assert g["computed_mask"] == mask
+            for k in ("n_windows", "der1_maxabs", "grad_f_max"):
+                assert g[k] == g1[k], k
+            assert abs(g["ssim"] - g1["ssim"]) <= 1e-12
     for k in ("x_min", "x_max", "err_min", "err_max", "pwr_max", "n_pwr", "n_windows", "der1_maxabs"):
         assert g[k] == g1[k], k
     for k in ("mse", "psnr", "pearson", "ssim", "der1_mae", "lap_mse"):
         assert abs(g[k] - g1[k]) <= 1e-12 * max(1.0, abs(g1[k])), k
     assert np.allclose(g["ac"], g1["ac"], rtol=0, atol=1e-13)
+    with czc.Assessor(ssim_window=8, rank=0, nranks=1, nccl_uid=bench.czc_nccl_uid(), timing=True) as a:
+        gt = a.assess(xd, yd, dims=xd.shape, z0=0)                  # per-kernel timing: one stream
+    assert gt["ssim"] == g["ssim"] and gt["mse"] == g["mse"] and all(v > 0 for v in gt["kernel_ms"][:5])
 
 
 @pytest.mark.parametrize("dims,w", [((100, 120, 96), 8), ((23, 31, 40), 5), ((9, 300, 41), 3)])
