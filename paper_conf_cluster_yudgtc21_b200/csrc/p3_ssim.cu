@@ -134,6 +134,9 @@ __device__ __forceinline__ T lane_window_ext(T v) {
 //   |d ssim| <= n2 / D2 + n1 / D1 + 14 u,
 //   n2 = 2 [(5 cV + 19) u V^2 + cV u V q],
 //   n1 = 2 [6 cV u m V + 10 u m^2 + 2 cV u V (|mu_e| + s) + (cV u V)^2].
+// Evaluated in the cheaper dominating form q' = 8 |mu_a| + 6 |mu_e| + 10 s >= q (|mu_b| <= |mu_a| +
+// |mu_e|) and n1' = m (20 u m + 17 cV u V) + 18 (cV u V)^2 >= n1 (the computed |mu_e| <= (|mu_x| +
+// |mu_y|)(1 + u) + s since mu_y = mu_x + mu_e is formed from it, and s = 2 cV u V).
 // The window is certified when this is <= kSsimTau (cross-multiplied, no division; NaN / inf /
 // non-positive denominators fail the test and take the exact path).  Using the computed means
 // (not their worst case |K| + 2V) keeps windows near zero (QCLOUD-like fields) certified.
@@ -147,11 +150,11 @@ __host__ __device__ constexpr SsimCert ssim_cert(double cV) {
 __device__ __forceinline__ bool ssim_certified(const SsimCert& c, float Vf, double mua, double mue, double mux,
                                                double muy, double D1, double D2) {
   const double V = (double)Vf * (1.0 + 0x1p-22);
-  const double cuV = c.cvu * V, s = 2.0 * cuV;
-  const double q = fma(4.0, fabs(mua) + fabs(mua + mue), fma(2.0, fabs(mue), 10.0 * s));
-  const double m = fabs(mux) + fabs(muy) + 2.0 * s;
-  const double n2 = fma(c.ka * V, V, 2.0 * cuV * q);
-  const double n1 = 2.0 * fma(6.0 * cuV, m, fma(2.0 * cuV, fabs(mue) + s, cuV * cuV)) + c.kc * m * m;
+  const double cuV = c.cvu * V;
+  const double q = fma(8.0, fabs(mua), fma(6.0, fabs(mue), 20.0 * cuV));        // >= q above
+  const double m = fma(4.0, cuV, fabs(mux) + fabs(muy));
+  const double n2 = V * fma(c.ka, V, 2.0 * c.cvu * q);
+  const double n1 = fma(m, fma(c.kc, m, 17.0 * cuV), 18.0 * cuV * cuV);          // >= n1 above
   return D1 > 0.0 && D2 > 0.0 && fma(n2, D1, n1 * D2) <= c.tau * D1 * D2;
 }
 
