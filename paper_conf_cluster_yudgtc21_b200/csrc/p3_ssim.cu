@@ -542,17 +542,12 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
     step_body(s, s, false, false);
   }
   // steady state: a resync every kResync WZ planes (step = WZ, (1 + kResync) WZ, ...)
-  // in pairs of planes: the resync period is even, so the second plane of a pair never resyncs,
-  // and the ring shifts of the pair fold into one set of register moves
-  static_assert((kResync * WZ) % 2 == 0, "resync period must be even");
-  int rph = 0, step = WZ;
+  int rph = 0;
 #pragma unroll 1
-  for (; step + 1 < nsteps; step += 2) {
+  for (int step = WZ; step < nsteps; step++) {
     step_body(step, 0, true, rph == 0);
-    step_body(step + 1, 0, true, false);
-    rph = rph + 2 == kResync * WZ ? 0 : rph + 2;
+    rph = rph + 1 == kResync * WZ ? 0 : rph + 1;
   }
-  if (step < nsteps) step_body(step, 0, true, rph == 0);
 
   double rec[kSsimSlots] = {ssum, (double)scnt, (double)nexact};
   const unsigned bid = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
