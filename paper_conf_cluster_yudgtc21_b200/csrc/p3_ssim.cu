@@ -41,7 +41,13 @@
 
 namespace czc {
 
-constexpr int kP3Warps = 8;
+// Warps per block (A/B, C3 SSIM): 8 (two blocks per SM) 2.94 ms; 12 (one block, 168 registers)
+// 3.73 ms; 16 (one block, 128 registers, 1.56 footprint cells per window instead of 1.92) 3.35 ms —
+// the per-plane barrier of a single resident block is not hidden by a second one.
+#ifndef CZC_P3_WARPS
+#define CZC_P3_WARPS 8
+#endif
+constexpr int kP3Warps = CZC_P3_WARPS;
 constexpr int kP3Threads = 32 * kP3Warps;
 constexpr double kU = 1.1102230246251565e-16;   // unit roundoff of FP64, 2^-53
 // Per-window error budget of the fast path.  The parity tolerance of SSIM is 1e-6 absolute on
