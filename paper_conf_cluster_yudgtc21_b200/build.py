@@ -16,8 +16,10 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-OBJ = os.path.join(HERE, "build_obj")
-SO = os.path.join(HERE, "libczc.so")
+# development A/B builds (tools/ab_build.py): extra nvcc flags and another output path
+EXTRA = os.environ.get("CZC_NVCC_EXTRA", "").split()
+OBJ = os.environ.get("CZC_OBJ_DIR") or os.path.join(HERE, "build_obj")
+SO = os.environ.get("CZC_SO_OUT") or os.path.join(HERE, "libczc.so")
 ROOT = os.path.dirname(HERE)
 SOURCES = ["czc_api.cu", "czc_comm.cu", "p1_reduce.cu", "p2_stencil.cu", "p3_ssim.cu", "p4_generic.cu"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -53,7 +55,7 @@ def _have_nccl() -> bool:
 
 def _flags():
     f = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "-Xptxas", "-O3",
-                "-I" + os.path.join(ROOT, "include")]
+                "-I" + os.path.join(ROOT, "include")] + EXTRA
     if _have_nccl():
         f.append("-DCZC_WITH_NCCL")
         tn = _torch_nccl()
