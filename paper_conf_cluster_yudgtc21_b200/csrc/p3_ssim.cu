@@ -57,7 +57,15 @@ constexpr double kSsimTau = 2.5e-7;
 // The streamed window sums are re-summed from scratch every kResync x (window extent) planes /
 // rows and slide in between, so a rounding error lives at most (kResync + 1) w - 1 planes.
 // 2: C2 SSIM 0.570 -> 0.554 ms (A/B) against 1, with the same flags on the test fields.
-constexpr int kResync = 2;
+// 3: C5 SSIM 169.9 -> 168.1 ms, C3 2.856 -> 2.822 ms against 2 (A/B), the same flags on every
+// test field (tests/test_gpu_ssim_cert.py)
+#ifndef CZC_P3_RESYNC
+#define CZC_P3_RESYNC 3
+#endif
+constexpr int kResync = CZC_P3_RESYNC;
+#ifndef CZC_P3_LONG_CHUNKS
+#define CZC_P3_LONG_CHUNKS 1
+#endif
 
 template <typename T, int WX, int WY, int WZ, int G>
 struct SsimGeom {
@@ -591,6 +599,24 @@ static cudaError_t launch_t(const Field3<T>& f, const SsimParams& p, double* par
   }
   const int64_t slots = (int64_t)(sms > 0 ? sms : 148) * occ;
   const int64_t n0 = cdiv(noz, p.zchunk);
+#if CZC_P3_LONG_CHUNKS
+  // Any chunk count from the one giving chunks of at most kMaxChunk planes up to n0 + 2: a
+  // block's cost is its zc window planes plus its WZ - 1 warm-up planes (z-walk only, ~0.3 of a
+  // window plane) plus ~1 plane of prologue / epilogue, times the waves.  Long chunks amortise
+  // the warm-up where the grid is large anyway (C3, C5); short ones balance small grids (C2).
+#ifndef CZC_P3_MAX_CHUNK
+#define CZC_P3_MAX_CHUNK 512
+#endif
+  constexpr int64_t kMaxChunk = CZC_P3_MAX_CHUNK;
+  const int64_t nlo = cdiv(noz, kMaxChunk);
+  int64_t best_n = n0, best_cost = INT64_MAX;
+  for (int64_t nch = nlo; nch <= n0 + 2 && nch <= noz; nch++) {
+    const int64_t zc = cdiv(noz, nch);
+    if (cdiv(noz, zc) != nch) continue;               // the same chunking as a smaller count
+    const int64_t cost = cdiv(tiles * nch, slots) * (10 * zc + 3 * (WZ - 1) + 10);
+    if (cost < best_cost) { best_cost = cost; best_n = nch; }
+  }
+#else
   int64_t best_n = n0, best_cost = INT64_MAX;
   for (int64_t nch = n0 > 2 ? n0 - 2 : 1; nch <= n0 + 2 && nch <= noz; nch++) {
     const int64_t zc = cdiv(noz, nch);
@@ -598,6 +624,7 @@ static cudaError_t launch_t(const Field3<T>& f, const SsimParams& p, double* par
     const int64_t cost = cdiv(tiles * nch, slots) * (zc + WZ - 1);
     if (cost < best_cost) { best_cost = cost; best_n = nch; }
   }
+#endif
   SsimParams q = p;
   q.zchunk = (int)cdiv(noz, best_n);
   dim3 grid((unsigned)cdiv(f.nx - WX + 1, Gm::TX), (unsigned)cdiv(f.ny - WY + 1, Gm::TY),

@@ -2,6 +2,8 @@
 samples by opcode, the top instructions, shared-memory excess wavefronts (development aid)."""
 import csv, collections, sys
 rows = list(csv.reader(open(sys.argv[1])))
+ends = [i for i, r in enumerate(rows) if i > 0 and r and r[0] == "Kernel Name"]
+rows = rows[:ends[0]] if ends else rows   # first kernel section only
 h = rows[1]
 ix = {k: h.index(k) for k in ("Address", "Source", "Warp Stall Sampling (All Samples)", "Instructions Executed",
                               "L1 Wavefronts Shared Excessive")}

@@ -30,6 +30,8 @@ for cub in sorted(os.listdir(tmp)):
             off2src[int(m.group(1), 16)] = cur
     break
 rows = list(csv.reader(open(dump)))
+ends = [i for i, r in enumerate(rows) if i > 0 and r and r[0] == "Kernel Name"]
+rows = rows[:ends[0]] if ends else rows   # first kernel section only
 h = rows[1]
 a, n, st = h.index("Address"), h.index("Instructions Executed"), h.index("Warp Stall Sampling (All Samples)")
 base = int(rows[2][a], 16)
