@@ -153,3 +153,22 @@ def test_adversarial_result_deterministic(czc):
     x, y = step_pair((30, 40, 57), 2, 37)
     outs = [gpu_windows(czc, x, y, 8)[1] for _ in range(3)]
     assert all(o["ssim"] == outs[0]["ssim"] and o["n_ssim_exact"] == outs[0]["n_ssim_exact"] for o in outs)
+
+
+@pytest.mark.parametrize("dims,step", [((1100, 160, 160), 1), ((600, 26, 33), 3)])
+def test_tall_fields_long_chunks(czc, orc, dims, step):
+    """Tall fields: with 70 tiles the launcher's cost model (p3_ssim.cu launch_t) walks the
+    1100-plane field in 4 chunks of 274 origin planes (one wave), so one block's z-sums slide and
+    resync across hundreds of planes and the chunk boundaries fall mid-field; the small field
+    takes many short chunks with a z step of 3.  Every window is compared with the oracle on a
+    log-normal recipe field and on a z-step field whose steps repeat every 97 planes (each block
+    meets several)."""
+    x, y = synth.make_pair(synth.config("C3", dims=dims))
+    r, worst = check_all_windows(czc, orc, x.numpy(), y.numpy(), 8, step)
+    assert r["n_ssim_exact"] == 0
+    rng = np.random.default_rng(11)
+    z = np.arange(dims[0])[:, None, None]
+    xs = (np.where((z // 97) % 2 == 0, 1.0, 1000.0) + 1e-3 * rng.standard_normal(dims)).astype(np.float32)
+    ys = (0.2 * np.rint(xs.astype(np.float64) / 0.2)).astype(np.float32)
+    r2, worst2 = check_all_windows(czc, orc, xs, ys, 8, step)
+    print(f"tall {dims} step {step}: worst {worst:.2e} / {worst2:.2e}, exact recomputes {r2['n_ssim_exact']}")
