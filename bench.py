@@ -416,11 +416,12 @@ def run_ours(args, rank, world, local):
             xo, yo = make_slab_device(sp, 0, sp.dims[0], dev, 1)
             nb = 2 * xo.numel() * 4
             with czc.Assessor(ndim=xo.dim(), device=local, stream=stream, **cfg) as ao:
-                ms, _ = time_steps(czc, ao, xo, yo, {}, args.steps, args.warmup, stream, flush, clean)
+                ms, ro = time_steps(czc, ao, xo, yo, {}, args.steps, args.warmup, stream, flush, clean)
             sh = pattern_split(czc, xo, yo, {}, cfg, max(3, args.steps // 2), 3, stream, flush, clean, local) \
                 if xo.dim() == 3 else {}
             others[name] = {"workload": sp.name, "dims": list(sp.dims), "value": round(nb * len(ms) / (sum(ms) * 1e-3) / 1e9, 3),
                             "unit": UNIT, "ms_per_step": round(sum(ms) / len(ms), 4),
+                            "ssim_exact_windows": int(ro.get("n_ssim_exact", 0)),
                             "per_pattern_ms": {k: round(v, 4) for k, v in sh.items()},
                             "per_pattern_hbm_frac": {k: round(nb / (v * 1e-3) / 1e9 / peak, 4) for k, v in sh.items() if v > 0}}
             del xo, yo

@@ -57,14 +57,18 @@ constexpr double kSsimTau = 2.5e-7;
 // The streamed window sums are re-summed from scratch every kResync x (window extent) planes /
 // rows and slide in between, so a rounding error lives at most (kResync + 1) w - 1 planes.
 // 2: C2 SSIM 0.570 -> 0.554 ms (A/B) against 1, with the same flags on the test fields.
-// 3: C5 SSIM 169.9 -> 168.1 ms, C3 2.856 -> 2.822 ms against 2 (A/B), the same flags on every
-// test field (tests/test_gpu_ssim_cert.py)
+// 3 measured ~1 % faster (C5 169.9 -> 168.1 ms, C3 2.856 -> 2.822 ms) but sends 448 windows of
+// the C3 512^3 recipe to the exact path (0 with 2), so 2 stays.
 #ifndef CZC_P3_RESYNC
-#define CZC_P3_RESYNC 3
+#define CZC_P3_RESYNC 2
 #endif
 constexpr int kResync = CZC_P3_RESYNC;
 #ifndef CZC_P3_LONG_CHUNKS
 #define CZC_P3_LONG_CHUNKS 1
+#endif
+// a new tile anchor at every resync (1) or one per block (0)
+#ifndef CZC_P3_REANCHOR
+#define CZC_P3_REANCHOR 1
 #endif
 
 template <typename T, int WX, int WY, int WZ, int G>
@@ -341,10 +345,12 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
     vm[k] = 0.f;
   }
   load(0, false);
-  // the block's anchor (tile_anchor) from the first plane's footprint: one barrier
-  T Kt = (T)0;
-  {
-    __shared__ T s_ext[2][kP3Warps];
+  // The block's anchor (tile_anchor) from the footprint of the plane in `nxt` (one barrier): at
+  // the first plane, and again at every resync — the z-sums are re-summed from scratch there, so
+  // they can take a new anchor, which keeps K near the values of long z-chunks (a log-normal
+  // density changes by decades along z).
+  __shared__ T s_ext[2][kP3Warps];
+  auto block_anchor = [&](int64_t z) -> T {
     T mn = nxt[0].x, mx = nxt[0].x;
 #pragma unroll
     for (int k = 1; k < KC; k++)
@@ -352,13 +358,18 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
     mn = warp_min_t(mn);
     mx = warp_max_t(mx);
     if (lane == 0) { s_ext[0][warp] = mn; s_ext[1][warp] = mx; }
-    __syncthreads();
+    __syncthreads();                                     // (the previous readers passed a barrier)
 #pragma unroll
     for (int w = 0; w < kP3Warps; w++) { mn = tmin(mn, s_ext[0][w]); mx = tmax(mx, s_ext[1][w]); }
-    if (nsteps > 0) Kt = tile_anchor<T>(f.xp(zb)[ky * f.nx + kx], mn, mx);
+    return tile_anchor<T>(f.xp(z)[ky * f.nx + kx], mn, mx);
+  };
+  T Kt = (T)0;
+  {
+    const T k0 = block_anchor(zb < zend ? zb : f.zown0);
+    if (nsteps > 0) Kt = k0;
   }
-  const double K = (double)Kt;
-  const float K32 = (float)Kt;
+  double K = (double)Kt;
+  float K32 = (float)Kt;
 
   double ssum = 0;
   unsigned scnt = 0, nexact = 0;
@@ -401,7 +412,13 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
     // ---- (a) z-walk --------------------------------------------------------------------
     if (resync) {
       // window planes zb+step-WZ+1 .. zb+step: ring slots 1..WZ-1 (x) with their y re-read,
-      // plus the entering plane; V restarts from the window's own samples
+      // plus the entering plane, about a new anchor from the entering plane; V restarts from
+      // the window's own samples
+#if CZC_P3_REANCHOR
+      Kt = block_anchor(zb + step);
+      K = (double)Kt;
+      K32 = (float)Kt;
+#endif
 #pragma unroll
       for (int k = 0; k < KC; k++) {
         if (!row_live(k)) continue;
@@ -665,9 +682,9 @@ p3_rows_kernel(Field3<T> f, SsimParams p, int rchunk, double* __restrict__ parts
   const int64_t kx = x0 + 16 < nx ? x0 + 16 : nx - 1, ky = rb + W / 2 < ny ? rb + W / 2 : ny - 1;
   // anchor of this warp's tile (tile_anchor) from its first row
   const T fr = X[rb * nx + gxc];
-  const T Kt = tile_anchor<T>(X[ky * nx + kx], warp_min_t(fr), warp_max_t(fr));
-  const double K = (double)Kt;
-  const float K32 = (float)Kt;
+  T Kt = tile_anchor<T>(X[ky * nx + kx], warp_min_t(fr), warp_max_t(fr));
+  double K = (double)Kt;
+  float K32 = (float)Kt;
   const double Lglob = res->p1g.xmax - res->p1g.xmin;
   const bool range_global = p.range_mode != 0;
   const bool xok = lane < TX && gx <= nx - W && (gx % p.sx) == 0;
@@ -699,6 +716,12 @@ p3_rows_kernel(Field3<T> f, SsimParams p, int rchunk, double* __restrict__ parts
   auto step_body = [&](const int step, const int s, const bool warm, const bool resync) {
     const bool full = warm || s == W - 1;
     if (resync) {                                               // rows rb+step-W+1 .. rb+step
+#if CZC_P3_REANCHOR
+      // a new anchor from the entering row (the sums restart here), as the 3-D kernel
+      Kt = tile_anchor<T>(X[(rb + step) * nx + kx], warp_min_t(nx_), warp_max_t(nx_));
+      K = (double)Kt;
+      K32 = (float)Kt;
+#endif
       sm[0] = sm[1] = sm[2] = sm[3] = 0;
       vm = 0.f;
       const T* yr = Y + (rb + step - W + 1) * nx + gxc;
