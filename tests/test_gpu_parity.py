@@ -209,10 +209,13 @@ def test_full_size_hurricane(czc, orc):
 
 
 @pytest.mark.parametrize("cfg,dims,K,w", [("C2", (40, 70, 90), 2, 8), ("C1", (37, 13, 17), 3, 5),
-                                          ("C3", (44, 33, 40), 4, 6), ("C2q", (30, 50, 64), 3, 8)])
+                                          ("C3", (44, 33, 40), 4, 6), ("C2q", (30, 50, 64), 3, 8),
+                                          ("C5", (100, 40, 48), 8, 8)])
 def test_loopback_slabs(czc, orc, cfg, dims, K, w):
     """The multi-GPU algorithm (slab ownership, halo buffers, rank-ordered combine) on one GPU:
-    K slabs must agree with the oracle on the whole field, and with the single-slab run."""
+    K slabs must agree with the oracle on the whole field, and with the single-slab run.  The
+    C5 case is the bench's 8-GPU strong-scaling split in miniature: 8 uneven slabs (12-13 planes,
+    bench.slab_bounds), each barely deeper than the 10-plane AC halo."""
     x, y = synth.make_pair(synth.config(cfg, dims=dims))
     xn, yn = x.numpy(), y.numpy()
     xd, yd = x.cuda(), y.cuda()
