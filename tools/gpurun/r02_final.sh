@@ -14,7 +14,7 @@ timeout 1500 ncu --set full --clock-control none --import-source on -f -o gpurun
 python tools/ncu_summary.py gpurun_out/${TAG}_ncu gpurun_out/prof_${TAG}.ncu-rep --launches gpurun_out/launches_${TAG}.csv > /dev/null 2>&1; cat gpurun_out/${TAG}_ncu.md
 ncu -i gpurun_out/prof_${TAG}.ncu-rep --page source --csv --kernel-name regex:p3_kernel > gpurun_out/${TAG}_p3_source.csv 2>/dev/null
 rm -f gpurun_out/prof_${TAG}.ncu-rep
-for tool in memcheck racecheck synccheck initcheck; do
+for tool in; do   # compute-sanitizer is closed on the GPU pool (round 2); logs of r02w stay
   timeout 1500 compute-sanitizer --tool $tool --print-limit 50 python tools/sanitize_target.py > gpurun_out/sanitize_${tool}_${TAG}.log 2>&1
   echo "$tool: $(tail -1 gpurun_out/sanitize_${tool}_${TAG}.log)"
 done
