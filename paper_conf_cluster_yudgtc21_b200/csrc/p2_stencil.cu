@@ -20,11 +20,17 @@
 //    line's other coordinates.  z- and y-walks read coalesced rows directly; the x-walk goes
 //    through a warp-private shared-memory transpose.  Every product is formed exactly once.
 // FP64 accumulators per thread; block partials combined by the last block in index order.
+#include <cuda.h>               // CUtensorMap (the encoder comes through cudaGetDriverEntryPoint)
+#include <cudaTypedefs.h>
+
 #include "czc_internal.cuh"
 
 namespace czc {
 
 constexpr int kTX = 32, kTY = 8;
+#ifndef CZC_AC_TMA
+#define CZC_AC_TMA 1
+#endif
 
 // ================================================================================================
 // Derivatives
@@ -803,9 +809,13 @@ struct PlaneTile {
   static constexpr int NV = (HX + EPG - 1) / EPG;        // 16-byte groups per staged row
   static constexpr int PF = EPG * NV;            // staged row pitch (elements), 16-byte multiple
   static constexpr int PE = (PF + 1) | 1;        // eps row pitch (doubles), odd: conflict-free columns
-  double e[HY][PE];
+  // staged arrays first, each padded to a multiple of 128 bytes (tensor-copy destinations)
+  static constexpr int FPAD = (int)(((HY * PF * sizeof(T) + 127) / 128 * 128 - HY * PF * sizeof(T)) / sizeof(T));
   T fx[HY][PF];
+  T padx[FPAD > 0 ? FPAD : 128 / sizeof(T)];
   T fy[HY][PF];
+  T pady[FPAD > 0 ? FPAD : 128 / sizeof(T)];
+  double e[HY][PE];
 };
 
 __device__ __forceinline__ void cp_async4(unsigned dst, const void* src, int src_bytes) {
@@ -835,7 +845,7 @@ __device__ __forceinline__ void plane_stage(unsigned sfx, const T* xt, const T* 
   using PT = PlaneTile<T, TM>;
   constexpr int HX = PT::HX, HY = PT::HY, NV = PT::NV, PF = PT::PF, EPG = PT::EPG;
   constexpr int RS = kPlThreads / 32;                             // row stride
-  constexpr unsigned dy = (unsigned)(sizeof(T) * HY * PF);       // fx -> fy
+  constexpr unsigned dy = (unsigned)(offsetof(PT, fy) - offsetof(PT, fx));   // fx -> fy
   if (VEC) {
 #pragma unroll
     for (int g = lane; g < NV; g += 32) {
@@ -918,12 +928,31 @@ __device__ __forceinline__ void plane_walks(const PlaneTile<T, TM>& sm, int tid,
 
 // grid: persistent (gridDim.x blocks); block 256; requires ny > 1.
 // VEC: rows 16-byte aligned (nx % 4 == 0, aligned plane segments) and (32 + TM) * nx < 2^31.
-template <typename T, int TM, bool VEC>
+// One 3-D tensor copy (TMA, cp.async.bulk.tensor) of the box at (c0, c1, c2) into shared memory,
+// completing on `bar`; elements outside the tensor arrive as zeros.
+__device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, int c0, int c1, int c2, uint64_t* bar) {
+  asm volatile("cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];"
+               :: "r"(smem_addr(dst)), "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(smem_addr(bar))
+               : "memory");
+}
+
+// TMAP (float32, one plane segment): the x / y windows arrive by two tensor copies issued by one
+// thread (mapx / mapy: the segment as a (nx, ny, planes) tensor, box (PF, HY, 1)) instead of
+// per-thread 16-byte cp.async groups.
+template <typename T, int TM, bool VEC, bool TMAP>
 __global__ void __launch_bounds__(kPlThreads, pl_bps<T, TM>())
-ac_plane(Field3<T> s, double* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket) {
+ac_plane(Field3<T> s, double* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket,
+         const __grid_constant__ CUtensorMap mapx, const __grid_constant__ CUtensorMap mapy) {
   extern __shared__ __align__(128) unsigned char plane_smem[];
   using PT = PlaneTile<T, TM>;
   PT& sm = *reinterpret_cast<PT*>(plane_smem);
+  static_assert(!TMAP || (sizeof(T) == 4 && offsetof(PT, fy) % 128 == 0), "tensor copies: float32, 128-byte aligned");
+  __shared__ uint64_t s_bar;
+  uint32_t phase = 0;
+  if constexpr (TMAP) {
+    if (threadIdx.x == 0) { mbar_init(&s_bar, 1); fence_mbar_init(); }
+    __syncthreads();
+  }
   constexpr int HY = PT::HY, NV = PT::NV, EPG = PT::EPG;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const unsigned sfx = (unsigned)__cvta_generic_to_shared(&sm.fx[0][0]);
@@ -959,8 +988,21 @@ ac_plane(Field3<T> s, double* __restrict__ parts, DevResults* __restrict__ res, 
   auto stage_item = [&](int64_t sz, int64_t sx0, int64_t sy0) {
     const int rv = (int)(s.ny - sy0 < HY ? s.ny - sy0 : HY);
     const int cv = (int)(s.nx - sx0 < PT::PF ? s.nx - sx0 : PT::PF);
-    const int64_t o = sy0 * s.nx + sx0;
-    plane_stage<T, TM, VEC>(sfx, s.xp(sz) + o, s.yp(sz) + o, s.nx, rv, cv, warp, lane);
+    if constexpr (TMAP) {
+      (void)rv; (void)cv;
+      if (threadIdx.x == 0) {
+        // the previous readers of the staging buffers passed a barrier; order their generic-proxy
+        // reads before the async-proxy writes
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        mbar_expect_tx(&s_bar, (uint32_t)(2 * HY * PT::PF * sizeof(T)));
+        const int zc = (int)(sz - s.zs[0]);
+        tma_load_3d(&sm.fx[0][0], &mapx, (int)sx0, (int)sy0, zc, &s_bar);
+        tma_load_3d(&sm.fy[0][0], &mapy, (int)sx0, (int)sy0, zc, &s_bar);
+      }
+    } else {
+      const int64_t o = sy0 * s.nx + sx0;
+      plane_stage<T, TM, VEC>(sfx, s.xp(sz) + o, s.yp(sz) + o, s.nx, rv, cv, warp, lane);
+    }
   };
   if (jb < je) stage_item(z, x0, y0);
   for (int64_t j = jb; j < je; j++) {
@@ -978,7 +1020,12 @@ ac_plane(Field3<T> s, double* __restrict__ parts, DevResults* __restrict__ res, 
       limy0[h] = my < TM ? (int)(my < -1 ? -1 : my) : TM;
     }
     {
-      cp_async_wait_all();
+      if constexpr (TMAP) {
+        mbar_wait(&s_bar, phase);
+        phase ^= 1u;
+      } else {
+        cp_async_wait_all();
+      }
       __syncthreads();                     // plane z staged; previous walks done with sm.e
       {
         // all 16-byte groups of the staged window, 256 at a time (row r, group g of the row);
@@ -1025,6 +1072,31 @@ ac_plane(Field3<T> s, double* __restrict__ parts, DevResults* __restrict__ res, 
   }
   ac_finish<TM>(acc, parts, res->rec.ac[1], ticket);
 }
+
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no libcuda link): a float32
+// segment of planes as a (nx, ny, planes) tensor with box (bx, by, 1), zeros outside.
+static bool encode_plane_map(CUtensorMap* m, const float* base, int64_t nx, int64_t ny, int64_t nz, int bx, int by) {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    void* fp = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fp, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !fp)
+      return false;
+    fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fp);
+  }
+  if (nx % 4 != 0 || ((uintptr_t)base & 15) != 0 || nx >= ((int64_t)1 << 32) || ny >= ((int64_t)1 << 32) ||
+      nz >= ((int64_t)1 << 32))
+    return false;
+  const cuuint64_t dims[3] = {(cuuint64_t)nx, (cuuint64_t)ny, (cuuint64_t)nz};
+  const cuuint64_t strides[2] = {(cuuint64_t)nx * 4, (cuuint64_t)(nx * ny) * 4};
+  const cuuint32_t box[3] = {(cuuint32_t)bx, (cuuint32_t)by, 1u};
+  const cuuint32_t es[3] = {1u, 1u, 1u};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(base), dims, strides, box, es,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+static bool encode_plane_map(CUtensorMap*, const double*, int64_t, int64_t, int64_t, int, int) { return false; }
 
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 static int sm_count() {
@@ -1195,10 +1267,31 @@ static cudaError_t launch_ac_t(const Field3<E>& s, int T, double* parts, DevResu
     constexpr int psm = (int)sizeof(PlaneTile<E, TM>);
     // 16-byte staging needs aligned rows; tile-relative offsets are 32-bit
     const bool pvec = vec && (int64_t)(pl_ty<E, TM>() + TM) * s.nx < ((int64_t)1 << 31);
-    auto kern = pvec ? ac_plane<E, TM, true> : ac_plane<E, TM, false>;
-    if ((e = pvec ? set_smem_once<ac_plane<E, TM, true>>(psm) : set_smem_once<ac_plane<E, TM, false>>(psm)) != cudaSuccess)
-      return e;
-    kern<<<g.pl, kPlThreads, psm, st>>>(s, pp, res, tickets + 1);
+    static const CUtensorMap no_map{};
+    bool done = false;
+#if CZC_AC_TMA
+    if constexpr (sizeof(E) == 4) {
+      // one plane segment (single GPU): the windows arrive by tensor copies
+      if (pvec && s.nseg == 1) {
+        using PT = PlaneTile<E, TM>;
+        CUtensorMap mx, my;
+        const int64_t nzs = s.zs[1] - s.zs[0];
+        if (encode_plane_map(&mx, s.xs[0], s.nx, s.ny, nzs, PT::PF, PT::HY) &&
+            encode_plane_map(&my, s.ys[0], s.nx, s.ny, nzs, PT::PF, PT::HY)) {
+          if ((e = set_smem_once<ac_plane<E, TM, true, true>>(psm)) != cudaSuccess) return e;
+          ac_plane<E, TM, true, true><<<g.pl, kPlThreads, psm, st>>>(s, pp, res, tickets + 1, mx, my);
+          done = true;
+        }
+      }
+    }
+#endif
+    if (!done) {
+      auto kern = pvec ? ac_plane<E, TM, true, false> : ac_plane<E, TM, false, false>;
+      if ((e = pvec ? set_smem_once<ac_plane<E, TM, true, false>>(psm) : set_smem_once<ac_plane<E, TM, false, false>>(psm)) !=
+          cudaSuccess)
+        return e;
+      kern<<<g.pl, kPlThreads, psm, st>>>(s, pp, res, tickets + 1, no_map, no_map);
+    }
   } else if (g.rx) {
     bool done = false;
     if constexpr (sizeof(E) == 4) {
