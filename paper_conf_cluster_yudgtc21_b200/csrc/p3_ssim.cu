@@ -37,6 +37,11 @@
 // K is one anchor per block (tile_anchor: the tile-centre sample of its first plane, or 0 for
 // tiles spanning decades or crossing zero).  Window extents are
 // compile-time (cubic 3-D, square 2-D, 1-D).
+#include <type_traits>
+
+#include <cuda.h>               // CUtensorMap (encoded through cudaGetDriverEntryPoint)
+#include <cudaTypedefs.h>
+
 #include "czc_internal.cuh"
 
 namespace czc {
@@ -82,6 +87,15 @@ struct SsimGeom {
   // x FY x 32, double-buffered
   static constexpr size_t buf_bytes = (size_t)ZSTRIDE * (4 * sizeof(double) + 2 * sizeof(T) + sizeof(float));
   static constexpr size_t smem = 2 * buf_bytes;
+  // tensor-copy staging (TMAP): kStages planes of { x, y of the entering plane, y of the plane
+  // leaving the z-window }, each a BX x FY float box starting at the 16-byte-aligned column at or
+  // before the tile's first column (BX = 36 covers the 32 footprint columns from any offset 0..3)
+  static constexpr int BX = 36;
+  static constexpr size_t box_bytes = (size_t)BX * FY * sizeof(float);
+  static constexpr size_t box_pitch = (box_bytes + 127) / 128 * 128;
+  static constexpr size_t ring_off = (smem + 127) / 128 * 128;
+  static constexpr int kStages = 3;
+  static constexpr size_t smem_tma = ring_off + (size_t)kStages * 3 * box_pitch;
 };
 
 __device__ __forceinline__ double shd(double v, int d) { return __shfl_down_sync(0xffffffffu, v, d); }
@@ -274,15 +288,28 @@ __device__ __forceinline__ double ssim_exact_window(const Field3<T> f, int64_t o
 
 // T = float: the x ring and the exchanged extrema are floats (exact); T = double: doubles, one
 // block per SM for the larger register ring.
-template <typename T, int WX, int WY, int WZ, int G>
+// 3-D tensor copy (TMA) of the box at (c0, c1, c2) into shared memory, completing on `bar`;
+// elements outside the tensor arrive as zeros
+__device__ __forceinline__ void p3_tma_3d(void* dst, const CUtensorMap* map, int c0, int c1, int c2, uint64_t* bar) {
+  asm volatile("cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];"
+               :: "r"(smem_addr(dst)), "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(smem_addr(bar))
+               : "memory");
+}
+
+// TMAP (float32 fields in one plane segment): the footprint planes arrive by tensor copies issued
+// by one thread kStages - 1 planes ahead into a shared-memory ring (no per-thread addresses);
+// cells outside the field read zeros (they feed only masked windows, and the tile anchor skips
+// them).
+template <typename T, int WX, int WY, int WZ, int G, bool TMAP>
 __global__ void __launch_bounds__(kP3Threads, (kP3Warps <= 8 && SsimGeom<T, WX, WY, WZ, G>::KC * WZ * sizeof(T) <= 128) ? 2 : 1)
 p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __restrict__ res,
-          unsigned int* __restrict__ ticket, double* __restrict__ dbg) {
+          unsigned int* __restrict__ ticket, double* __restrict__ dbg, const __grid_constant__ CUtensorMap mapx,
+          const __grid_constant__ CUtensorMap mapy) {
   using Gm = SsimGeom<T, WX, WY, WZ, G>;
   constexpr int TX = Gm::TX, FY = Gm::FY, KC = Gm::KC, ZS = Gm::ZSTRIDE;
   constexpr double invM = 1.0 / (double)(WX * WY * WZ);
   constexpr SsimCert cert = ssim_cert((1.0 + 2.0 * kResync) * WZ + WY + 2.0 * G + 13.0);
-  extern __shared__ __align__(16) unsigned char smem_raw[];
+  extern __shared__ __align__(128) unsigned char smem_raw[];   // (128: tensor-copy destinations)
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int64_t x0 = (int64_t)blockIdx.x * TX, y0 = (int64_t)blockIdx.y * Gm::TY;
@@ -319,19 +346,61 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
   // footprint row warp + kP3Warps k exists (r < FY); warp-uniform, and constant for every k but
   // the last, so rows past the footprint cost nothing
   auto row_live = [&](const int k) { return kP3Warps * (k + 1) <= FY || warp + kP3Warps * k < FY; };
-  auto load = [&](int n, bool has_old) {                 // has_old: n >= WZ (constant per call site)
-    if (n < nsteps) {                                    // block-uniform
-#pragma unroll
-      for (int k = 0; k < KC; k++) {
-        if (!row_live(k)) continue;
-        nxt[k].x = __ldg(cin.x + off[k]);
-        nxt[k].y = __ldg(cin.y + off[k]);
-        nyo[k] = has_old ? __ldg(cold.y + off[k]) : (T)0;
+  __shared__ uint64_t s_tbar[Gm::kStages];
+  const int xs0 = (int)(x0 & ~(int64_t)3), xsh = (int)(x0 - xs0);   // aligned box column, lane shift
+  auto tma_issue = [&](int n) {                          // thread 0; plane n of this block
+    if constexpr (TMAP) {
+      if (threadIdx.x == 0 && n < nsteps) {
+        const int st = n % Gm::kStages;
+        const bool old = n >= WZ;
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        mbar_expect_tx(&s_tbar[st], (uint32_t)((old ? 3 : 2) * Gm::box_bytes));
+        unsigned char* d = smem_raw + Gm::ring_off + (size_t)3 * st * Gm::box_pitch;
+        const int zc = (int)(zb + n - f.zs[0]);
+        p3_tma_3d(d, &mapx, xs0, (int)y0, zc, &s_tbar[st]);
+        p3_tma_3d(d + Gm::box_pitch, &mapy, xs0, (int)y0, zc, &s_tbar[st]);
+        if (old) p3_tma_3d(d + 2 * Gm::box_pitch, &mapy, xs0, (int)y0, zc - WZ, &s_tbar[st]);
       }
-      cin.advance(f, zb + n + 1);
-      if (has_old) cold.advance(f, zb + n + 1 - WZ);
     }
   };
+  auto load = [&](int n, bool has_old) {                 // has_old: n >= WZ (constant per call site)
+    if (n < nsteps) {                                    // block-uniform
+      if constexpr (TMAP) {
+        const int st = n % Gm::kStages;
+        mbar_wait(&s_tbar[st], (uint32_t)((n / Gm::kStages) & 1));
+        constexpr int BP = (int)(Gm::box_pitch / sizeof(float));
+        const float* b = reinterpret_cast<const float*>(smem_raw + Gm::ring_off) + 3 * st * BP;
+#pragma unroll
+        for (int k = 0; k < KC; k++) {
+          if (!row_live(k)) continue;
+          const int c = (warp + kP3Warps * k) * Gm::BX + xsh + lane;
+          nxt[k].x = b[c];
+          nxt[k].y = b[BP + c];
+          nyo[k] = has_old ? b[2 * BP + c] : (T)0;
+        }
+      } else {
+#pragma unroll
+        for (int k = 0; k < KC; k++) {
+          if (!row_live(k)) continue;
+          nxt[k].x = __ldg(cin.x + off[k]);
+          nxt[k].y = __ldg(cin.y + off[k]);
+          nyo[k] = has_old ? __ldg(cold.y + off[k]) : (T)0;
+        }
+        cin.advance(f, zb + n + 1);
+        if (has_old) cold.advance(f, zb + n + 1 - WZ);
+      }
+    }
+  };
+  if constexpr (TMAP) {
+    if (threadIdx.x == 0) {
+#pragma unroll
+      for (int i = 0; i < Gm::kStages; i++) mbar_init(&s_tbar[i], 1);
+      fence_mbar_init();
+    }
+    __syncthreads();
+#pragma unroll
+    for (int n = 0; n + 1 < Gm::kStages; n++) tma_issue(n);
+  }
 
   double sm[KC][4];
   T ring[KC][WZ];                                        // x of the last WZ planes
@@ -350,11 +419,17 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
   // they can take a new anchor, which keeps K near the values of long z-chunks (a log-normal
   // density changes by decades along z).
   __shared__ T s_ext[2][kP3Warps];
+  const bool col_in = x0 + lane < f.nx;
   auto block_anchor = [&](int64_t z) -> T {
-    T mn = nxt[0].x, mx = nxt[0].x;
+    // (TMAP: start from the tile's first sample, which is in the field, and skip the zeros the
+    // tensor copies put outside it)
+    T mn = TMAP ? f.xp(z)[y0 * f.nx + x0] : nxt[0].x, mx = mn;
 #pragma unroll
-    for (int k = 1; k < KC; k++)
-      if (row_live(k)) { mn = tmin(mn, nxt[k].x); mx = tmax(mx, nxt[k].x); }
+    for (int k = TMAP ? 0 : 1; k < KC; k++)
+      if (row_live(k) && (!TMAP || (col_in && y0 + warp + kP3Warps * k < f.ny))) {
+        mn = tmin(mn, nxt[k].x);
+        mx = tmax(mx, nxt[k].x);
+      }
     mn = warp_min_t(mn);
     mx = warp_max_t(mx);
     if (lane == 0) { s_ext[0][warp] = mn; s_ext[1][warp] = mx; }
@@ -461,8 +536,15 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
       }
     }
     load(step + 1, warm || s == WZ - 1);
-    if (!full) return;                                   // no complete z-window yet
+    if (!full) {                                         // no complete z-window yet
+      if constexpr (TMAP) {                              // every thread has read its planes <= step + 1
+        __syncthreads();
+        tma_issue(step + Gm::kStages - 1);
+      }
+      return;
+    }
     __syncthreads();
+    if constexpr (TMAP) tma_issue(step + Gm::kStages - 1);
     const bool zok = zph == 0;                           // origin plane zb + step - WZ + 1
     zph = zph + 1 == p.sz ? 0 : zph + 1;
     // ---- (b) y-pass: the G origin rows of this warp (running sums over WY rows) ------------
@@ -593,13 +675,54 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
 
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no libcuda link): a float32
+// plane segment as a (nx, ny, planes) tensor with box (bx, by, 1), zeros outside.
+static bool p3_encode_map(CUtensorMap* m, const float* base, int64_t nx, int64_t ny, int64_t nz, int bx, int by) {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    void* fp = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fp, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !fp)
+      return false;
+    fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fp);
+  }
+  if (nx % 4 != 0 || ((uintptr_t)base & 15) != 0 || nx >= ((int64_t)1 << 31) || ny >= ((int64_t)1 << 31) ||
+      nz >= ((int64_t)1 << 31))
+    return false;
+  const cuuint64_t dims[3] = {(cuuint64_t)nx, (cuuint64_t)ny, (cuuint64_t)nz};
+  const cuuint64_t strides[2] = {(cuuint64_t)nx * 4, (cuuint64_t)(nx * ny) * 4};
+  const cuuint32_t box[3] = {(cuuint32_t)bx, (cuuint32_t)by, 1u};
+  const cuuint32_t es[3] = {1u, 1u, 1u};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(base), dims, strides, box, es,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+#ifndef CZC_P3_TMA
+#define CZC_P3_TMA 1
+#endif
+
 template <typename T, int WX, int WY, int WZ, int G>
 static cudaError_t launch_t(const Field3<T>& f, const SsimParams& p, double* parts,
                             DevResults* res, unsigned int* ticket, double* dbg, cudaStream_t st,
                             int64_t* nblocks_out) {
   using Gm = SsimGeom<T, WX, WY, WZ, G>;
-  auto kern = p3_kernel<T, WX, WY, WZ, G>;
-  cudaError_t e = set_smem_once<p3_kernel<T, WX, WY, WZ, G>>((int)Gm::smem);
+  // tensor-copy staging: float32, cubic 3-D windows, one plane segment (single GPU)
+  static const CUtensorMap no_map{};
+  CUtensorMap mx = no_map, my = no_map;
+  bool tma = false;
+  if constexpr (CZC_P3_TMA && std::is_same<T, float>::value && WY > 1 && WZ > 1) {
+    if (f.nseg == 1 && !nblocks_out) {
+      const int64_t nzs = f.zs[1] - f.zs[0];
+      tma = p3_encode_map(&mx, f.xs[0], f.nx, f.ny, nzs, Gm::BX, Gm::FY) &&
+            p3_encode_map(&my, f.ys[0], f.nx, f.ny, nzs, Gm::BX, Gm::FY);
+    }
+  }
+  auto kern = tma ? p3_kernel<T, WX, WY, WZ, G, true> : p3_kernel<T, WX, WY, WZ, G, false>;
+  const size_t smem_bytes = tma ? Gm::smem_tma : Gm::smem;
+  cudaError_t e = tma ? set_smem_once<p3_kernel<T, WX, WY, WZ, G, true>>((int)Gm::smem_tma)
+                      : set_smem_once<p3_kernel<T, WX, WY, WZ, G, false>>((int)Gm::smem);
   if (e != cudaSuccess) return e;
   int64_t zhi = f.zown1 < f.nz - WZ + 1 ? f.zown1 : f.nz - WZ + 1;
   const int64_t noz = zhi > f.zown0 ? zhi - f.zown0 : 1;
@@ -613,7 +736,9 @@ static cudaError_t launch_t(const Field3<T>& f, const SsimParams& p, double* par
     int d = 0;
     cudaGetDevice(&d);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, d);
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kP3Threads, Gm::smem) != cudaSuccess || occ < 1) occ = 1;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, p3_kernel<T, WX, WY, WZ, G, false>, kP3Threads, Gm::smem) !=
+            cudaSuccess || occ < 1)
+      occ = 1;
   }
   const int64_t slots = (int64_t)(sms > 0 ? sms : 148) * occ;
   const int64_t n0 = cdiv(noz, p.zchunk);
@@ -649,7 +774,7 @@ static cudaError_t launch_t(const Field3<T>& f, const SsimParams& p, double* par
             (unsigned)cdiv(noz, q.zchunk));
   if (nblocks_out) { *nblocks_out = (int64_t)grid.x * grid.y * grid.z; return cudaSuccess; }
   if (f.ny * f.nx >= (int64_t)1 << 31) return cudaErrorInvalidValue;   // 32-bit in-plane offsets
-  kern<<<grid, kP3Threads, Gm::smem, st>>>(f, q, parts, res, ticket, dbg);
+  kern<<<grid, kP3Threads, smem_bytes, st>>>(f, q, parts, res, ticket, dbg, mx, my);
   return cudaGetLastError();
 }
 

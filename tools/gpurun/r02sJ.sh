@@ -1,0 +1,7 @@
+python -m paper_conf_cluster_yudgtc21_b200.build > /dev/null 2>&1
+timeout 900 python -m pytest tests/test_gpu_ssim_cert.py tests/test_gpu_parity.py -q -x 2>&1 | tail -1
+python tools/ab_time.py C2 abtest/sst0.so abtest/sst1.so
+python tools/ab_time.py C3 abtest/sst0.so abtest/sst1.so
+for v in sst0 sst1; do
+  CZC_LIB=$PWD/abtest/$v.so timeout 600 python bench.py --steps 3 --warmup 2 --no-e2e --no-extra --no-f64 --no-cpu-baseline 2>/dev/null | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('$v', d['value'], d['ms_per_step'], d['per_pattern_ms'], d['ssim_exact_windows'])"
+done
