@@ -942,7 +942,7 @@ __device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, i
 template <typename T, int TM, bool VEC, bool TMAP>
 __global__ void __launch_bounds__(kPlThreads, pl_bps<T, TM>())
 ac_plane(Field3<T> s, double* __restrict__ parts, DevResults* __restrict__ res, unsigned int* __restrict__ ticket,
-         const __grid_constant__ CUtensorMap mapx, const __grid_constant__ CUtensorMap mapy) {
+         const __grid_constant__ CUtensorMap mapx, const __grid_constant__ CUtensorMap mapy, int64_t map_z0) {
   extern __shared__ __align__(128) unsigned char plane_smem[];
   using PT = PlaneTile<T, TM>;
   PT& sm = *reinterpret_cast<PT*>(plane_smem);
@@ -995,7 +995,7 @@ ac_plane(Field3<T> s, double* __restrict__ parts, DevResults* __restrict__ res, 
         // reads before the async-proxy writes
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         mbar_expect_tx(&s_bar, (uint32_t)(2 * HY * PT::PF * sizeof(T)));
-        const int zc = (int)(sz - s.zs[0]);
+        const int zc = (int)(sz - map_z0);               // plane within the mapped segment
         tma_load_3d(&sm.fx[0][0], &mapx, (int)sx0, (int)sy0, zc, &s_bar);
         tma_load_3d(&sm.fy[0][0], &mapy, (int)sx0, (int)sy0, zc, &s_bar);
       }
@@ -1271,15 +1271,19 @@ static cudaError_t launch_ac_t(const Field3<E>& s, int T, double* parts, DevResu
     bool done = false;
 #if CZC_AC_TMA
     if constexpr (sizeof(E) == 4) {
-      // one plane segment (single GPU): the windows arrive by tensor copies
-      if (pvec && s.nseg == 1) {
+      // the windows arrive by tensor copies; the owned planes lie in one segment (the whole field,
+      // or the local slab in slab mode, whose halo planes the in-plane lags never read): map it
+      int seg = -1;
+      for (int k = 0; k < s.nseg; k++)
+        if (s.zs[k] <= s.zown0 && s.zown1 <= s.zs[k + 1]) seg = k;
+      if (pvec && seg >= 0) {
         using PT = PlaneTile<E, TM>;
         CUtensorMap mx, my;
-        const int64_t nzs = s.zs[1] - s.zs[0];
-        if (encode_plane_map(&mx, s.xs[0], s.nx, s.ny, nzs, PT::PF, PT::HY) &&
-            encode_plane_map(&my, s.ys[0], s.nx, s.ny, nzs, PT::PF, PT::HY)) {
+        const int64_t nzs = s.zs[seg + 1] - s.zs[seg];
+        if (encode_plane_map(&mx, s.xs[seg], s.nx, s.ny, nzs, PT::PF, PT::HY) &&
+            encode_plane_map(&my, s.ys[seg], s.nx, s.ny, nzs, PT::PF, PT::HY)) {
           if ((e = set_smem_once<ac_plane<E, TM, true, true>>(psm)) != cudaSuccess) return e;
-          ac_plane<E, TM, true, true><<<g.pl, kPlThreads, psm, st>>>(s, pp, res, tickets + 1, mx, my);
+          ac_plane<E, TM, true, true><<<g.pl, kPlThreads, psm, st>>>(s, pp, res, tickets + 1, mx, my, s.zs[seg]);
           done = true;
         }
       }
@@ -1290,7 +1294,7 @@ static cudaError_t launch_ac_t(const Field3<E>& s, int T, double* parts, DevResu
       if ((e = pvec ? set_smem_once<ac_plane<E, TM, true, false>>(psm) : set_smem_once<ac_plane<E, TM, false, false>>(psm)) !=
           cudaSuccess)
         return e;
-      kern<<<g.pl, kPlThreads, psm, st>>>(s, pp, res, tickets + 1, no_map, no_map);
+      kern<<<g.pl, kPlThreads, psm, st>>>(s, pp, res, tickets + 1, no_map, no_map, 0);
     }
   } else if (g.rx) {
     bool done = false;
