@@ -34,9 +34,11 @@
 //       kSsimTau is recomputed exactly (two-pass, anchored at its own first sample) by its warp
 //       and counted in czc_result.n_ssim_exact (local anchors + bound +
 //       exact fallback).
-// K is one anchor per block (tile_anchor: the tile-centre sample of its first plane, or 0 for
-// tiles spanning decades or crossing zero).  Window extents are
-// compile-time (cubic 3-D, square 2-D, 1-D).
+// K is the block's anchor (tile_anchor: the tile-centre sample of its first plane, or 0 for
+// tiles spanning decades or crossing zero), re-chosen at every resync.  Window extents are
+// compile-time (cubic 3-D, square 2-D, 1-D).  Round 2: blocks walk long z-chunks where the grid
+// is large (launch_t's cost model), and on single-segment float32 fields the footprint planes
+// arrive by tensor copies (TMA) into a shared-memory ring instead of per-thread loads.
 #include <type_traits>
 
 #include <cuda.h>               // CUtensorMap (encoded through cudaGetDriverEntryPoint)
@@ -286,8 +288,6 @@ __device__ __forceinline__ double ssim_exact_window(const Field3<T> f, int64_t o
   return ((2.0 * mux * muy + C1) * (2.0 * cxy + C2)) / ((mux * mux + muy * muy + C1) * (vx + vy + C2));
 }
 
-// T = float: the x ring and the exchanged extrema are floats (exact); T = double: doubles, one
-// block per SM for the larger register ring.
 // 3-D tensor copy (TMA) of the box at (c0, c1, c2) into shared memory, completing on `bar`;
 // elements outside the tensor arrive as zeros
 __device__ __forceinline__ void p3_tma_3d(void* dst, const CUtensorMap* map, int c0, int c1, int c2, uint64_t* bar) {
@@ -296,6 +296,8 @@ __device__ __forceinline__ void p3_tma_3d(void* dst, const CUtensorMap* map, int
                : "memory");
 }
 
+// T = float: the x ring and the exchanged extrema are floats (exact); T = double: doubles, one
+// block per SM for the larger register ring.
 // TMAP (float32 fields in one plane segment): the footprint planes arrive by tensor copies issued
 // by one thread kStages - 1 planes ahead into a shared-memory ring (no per-thread addresses);
 // cells outside the field read zeros (they feed only masked windows, and the tile anchor skips
