@@ -1,3 +1,5 @@
+"""SSIM + P1 on a small C2-shaped field with and without per-kernel timing under the library in
+CZC_LIB: mean SSIM, window count, exact recomputes, kernel times (development aid)."""
 import os, sys
 sys.path.insert(0, os.getcwd())
 import torch, numpy as np

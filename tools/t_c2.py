@@ -1,3 +1,5 @@
+"""SSIM + P1 on a small and the full C2 shape under the library in CZC_LIB; prints the mean SSIM
+and exact recomputes or the error (development aid: tensor-copy bring-up)."""
 import os, sys
 sys.path.insert(0, os.getcwd())
 import torch
