@@ -298,15 +298,17 @@ __device__ __forceinline__ void p3_tma_3d(void* dst, const CUtensorMap* map, int
 
 // T = float: the x ring and the exchanged extrema are floats (exact); T = double: doubles, one
 // block per SM for the larger register ring.
-// TMAP (float32 fields in one plane segment): the footprint planes arrive by tensor copies issued
-// by one thread kStages - 1 planes ahead into a shared-memory ring (no per-thread addresses);
+// TMAP (float32 fields; in slab mode the local slab and its upper halo segment): the footprint
+// planes arrive by tensor copies issued by one thread kStages - 1 planes ahead into a
+// shared-memory ring (no per-thread addresses);
 // cells outside the field read zeros (they feed only masked windows, and the tile anchor skips
 // them).
 template <typename T, int WX, int WY, int WZ, int G, bool TMAP>
 __global__ void __launch_bounds__(kP3Threads, (kP3Warps <= 8 && SsimGeom<T, WX, WY, WZ, G>::KC * WZ * sizeof(T) <= 128) ? 2 : 1)
 p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __restrict__ res,
           unsigned int* __restrict__ ticket, double* __restrict__ dbg, const __grid_constant__ CUtensorMap mapx,
-          const __grid_constant__ CUtensorMap mapy) {
+          const __grid_constant__ CUtensorMap mapy, const __grid_constant__ CUtensorMap mapxh,
+          const __grid_constant__ CUtensorMap mapyh, int64_t tz0, int64_t tz1) {
   using Gm = SsimGeom<T, WX, WY, WZ, G>;
   constexpr int TX = Gm::TX, FY = Gm::FY, KC = Gm::KC, ZS = Gm::ZSTRIDE;
   constexpr double invM = 1.0 / (double)(WX * WY * WZ);
@@ -358,10 +360,14 @@ p3_kernel(Field3<T> f, SsimParams p, double* __restrict__ parts, DevResults* __r
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         mbar_expect_tx(&s_tbar[st], (uint32_t)((old ? 3 : 2) * Gm::box_bytes));
         unsigned char* d = smem_raw + Gm::ring_off + (size_t)3 * st * Gm::box_pitch;
-        const int zc = (int)(zb + n - f.zs[0]);
-        p3_tma_3d(d, &mapx, xs0, (int)y0, zc, &s_tbar[st]);
-        p3_tma_3d(d + Gm::box_pitch, &mapy, xs0, (int)y0, zc, &s_tbar[st]);
-        if (old) p3_tma_3d(d + 2 * Gm::box_pitch, &mapy, xs0, (int)y0, zc - WZ, &s_tbar[st]);
+        // planes below tz1 come from the segment mapped by (mapx, mapy) (from tz0), the others from
+        // the upper halo segment (mapxh, mapyh, from tz1); a leaving plane is always an owned one
+        const int64_t z = zb + n;
+        const bool hi = z >= tz1;
+        const int zc = (int)(hi ? z - tz1 : z - tz0);
+        p3_tma_3d(d, hi ? &mapxh : &mapx, xs0, (int)y0, zc, &s_tbar[st]);
+        p3_tma_3d(d + Gm::box_pitch, hi ? &mapyh : &mapy, xs0, (int)y0, zc, &s_tbar[st]);
+        if (old) p3_tma_3d(d + 2 * Gm::box_pitch, &mapy, xs0, (int)y0, (int)(z - WZ - tz0), &s_tbar[st]);
       }
     }
   };
@@ -712,13 +718,27 @@ static cudaError_t launch_t(const Field3<T>& f, const SsimParams& p, double* par
   using Gm = SsimGeom<T, WX, WY, WZ, G>;
   // tensor-copy staging: float32, cubic 3-D windows, one plane segment (single GPU)
   static const CUtensorMap no_map{};
-  CUtensorMap mx = no_map, my = no_map;
+  CUtensorMap mx = no_map, my = no_map, mxh = no_map, myh = no_map;
+  int64_t tz0 = 0, tz1 = 0;
   bool tma = false;
   if constexpr (CZC_P3_TMA && std::is_same<T, float>::value && WY > 1 && WZ > 1) {
-    if (f.nseg == 1 && !nblocks_out) {
-      const int64_t nzs = f.zs[1] - f.zs[0];
-      tma = p3_encode_map(&mx, f.xs[0], f.nx, f.ny, nzs, Gm::BX, Gm::FY) &&
-            p3_encode_map(&my, f.ys[0], f.nx, f.ny, nzs, Gm::BX, Gm::FY);
+    // the segment holding the owned planes (the whole field, or the local slab), and the upper
+    // halo segment after it when there is one (slab mode: the windows of the last owned planes)
+    int seg = -1;
+    for (int k = 0; k < f.nseg; k++)
+      if (f.zs[k] <= f.zown0 && f.zown1 <= f.zs[k + 1]) seg = k;
+    if (seg >= 0 && !nblocks_out) {
+      tz0 = f.zs[seg];
+      tz1 = f.zs[seg + 1];
+      tma = p3_encode_map(&mx, f.xs[seg], f.nx, f.ny, tz1 - tz0, Gm::BX, Gm::FY) &&
+            p3_encode_map(&my, f.ys[seg], f.nx, f.ny, tz1 - tz0, Gm::BX, Gm::FY);
+      mxh = mx;
+      myh = my;
+      if (tma && seg + 1 < f.nseg) {
+        const int64_t nh = f.zs[seg + 2] - f.zs[seg + 1];
+        tma = p3_encode_map(&mxh, f.xs[seg + 1], f.nx, f.ny, nh, Gm::BX, Gm::FY) &&
+              p3_encode_map(&myh, f.ys[seg + 1], f.nx, f.ny, nh, Gm::BX, Gm::FY);
+      }
     }
   }
   auto kern = tma ? p3_kernel<T, WX, WY, WZ, G, true> : p3_kernel<T, WX, WY, WZ, G, false>;
@@ -776,7 +796,7 @@ static cudaError_t launch_t(const Field3<T>& f, const SsimParams& p, double* par
             (unsigned)cdiv(noz, q.zchunk));
   if (nblocks_out) { *nblocks_out = (int64_t)grid.x * grid.y * grid.z; return cudaSuccess; }
   if (f.ny * f.nx >= (int64_t)1 << 31) return cudaErrorInvalidValue;   // 32-bit in-plane offsets
-  kern<<<grid, kP3Threads, smem_bytes, st>>>(f, q, parts, res, ticket, dbg, mx, my);
+  kern<<<grid, kP3Threads, smem_bytes, st>>>(f, q, parts, res, ticket, dbg, mx, my, mxh, myh, tz0, tz1);
   return cudaGetLastError();
 }
 
